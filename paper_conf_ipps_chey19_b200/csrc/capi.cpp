@@ -1,0 +1,162 @@
+// C ABI entry points for the GEMM, the leaf, plan introspection and the
+// partitioner (include/northup.h).
+#include <string.h>
+
+#include <chrono>
+
+#include "northup_internal.h"
+
+using namespace nu;
+
+struct northup_plan_s {
+  Plan plan;
+};
+
+static double now_ms() {
+  using namespace std::chrono;
+  return duration<double, std::milli>(steady_clock::now().time_since_epoch()).count();
+}
+
+extern "C" {
+
+int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
+                      int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t k_chunk,
+                      int npass, void* stream) {
+  if ((!A || !B) && M > 0 && N > 0 && K > 0) return fail(NU_EINVAL, "NULL operand");
+  if (!C && M > 0 && N > 0) return fail(NU_EINVAL, "NULL C");
+  return leaf_gemm_launch(A, lda, B, ldb, C, ldc, M, N, K, accumulate,
+                          k_chunk > 0 ? k_chunk : kDefaultKChunk, npass, static_cast<cudaStream_t>(stream));
+}
+
+int northup_gemm(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_buf_t C, int64_t M,
+                 int64_t N, int64_t K) {
+  return northup_gemm_ex(t, A, B, C, M, N, K, nullptr, nullptr);
+}
+
+static int zero_root_c(northup_tree_t t, northup_buf_t C, int64_t M, int64_t N) {
+  const uint64_t bytes = static_cast<uint64_t>(M) * N * 4;
+  if (C->storage == NU_HOST) {
+    memset(C->ptr, 0, bytes);
+    return 0;
+  }
+  if (C->storage == NU_HBM) {
+    cudaSetDevice(t->nodes[C->node].phys);
+    cudaError_t e = cudaMemset(C->ptr, 0, bytes);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    return e == cudaSuccess ? 0 : cuda_fail(e, "cudaMemset");
+  }
+  return fail(NU_ENOTSUP, "K == 0 on a FILE root");
+}
+
+int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_buf_t C, int64_t M,
+                    int64_t N, int64_t K, const northup_gemm_opts* o, northup_stats* s) {
+  const double t0 = now_ms();
+  if (!t || !A || !B || !C) return fail(NU_EINVAL, "NULL argument");
+  if (!t->finalized) return fail(NU_ESTATE, "tree not finalized");
+  if (t->busy) return fail(NU_ESTATE, "a northup_gemm is already in flight on this tree");
+  if (M < 0 || N < 0 || K < 0) return fail(NU_EINVAL, "negative dimension");
+  if (A->tree != t || B->tree != t || C->tree != t) return fail(NU_EINVAL, "buffer from another tree");
+  if (A->node != 0 || B->node != 0 || C->node != 0)
+    return fail(NU_EINVAL, "A, B and C must live at the root node (level 0)");
+  const uint64_t need_a = 4ull * M * K, need_b = 4ull * K * N, need_c = 4ull * M * N;
+  if (A->bytes < need_a || B->bytes < need_b || C->bytes < need_c)
+    return fail(NU_EINVAL, "buffer smaller than its matrix");
+  if (o && o->replicate_result && t->workers.size() > 1)
+    return fail(NU_ENOTSUP, "replicate_result needs the NCCL gather (not built in this version)");
+  northup_stats local{};
+  northup_stats* st = s ? s : &local;
+  *st = northup_stats{};
+  if (M == 0 || N == 0) return 0;
+  if (K == 0) return zero_root_c(t, C, M, N);
+  if (t->nodes[0].storage == NU_FILE)
+    return fail(NU_ENOTSUP, "FILE roots are not supported by northup_gemm in this version");
+
+  t->busy = true;
+  Plan plan;
+  const bool a_al = reinterpret_cast<uintptr_t>(A->ptr) % 16 == 0;
+  const bool b_al = reinterpret_cast<uintptr_t>(B->ptr) % 16 == 0;
+  int rc = build_plan_ex(t, M, N, K, o, a_al, b_al, &plan);
+  const double t1 = now_ms();
+  if (!rc) {
+    *st = plan.stats;
+    st->t_plan_ms = t1 - t0;
+    int prev = 0;
+    cudaGetDevice(&prev);
+    rc = execute_plan(t, plan, A->ptr, B->ptr, C->ptr, o, st);
+    cudaSetDevice(prev);
+  }
+  t->busy = false;
+  st->t_total_ms = now_ms() - t0;
+  return rc;
+}
+
+// ------------------------------------------------------------ plan API
+int northup_plan_create(northup_tree_t t, int64_t M, int64_t N, int64_t K,
+                        const northup_gemm_opts* opts, northup_plan_t* out) {
+  if (!t || !out) return fail(NU_EINVAL, "NULL argument");
+  northup_plan_s* p = new northup_plan_s();
+  int rc = build_plan(t, M, N, K, opts, &p->plan);
+  if (rc) {
+    delete p;
+    return rc;
+  }
+  *out = p;
+  return 0;
+}
+
+int northup_plan_num_ops(northup_plan_t p, int64_t* n) {
+  if (!p || !n) return fail(NU_EINVAL, "NULL argument");
+  *n = static_cast<int64_t>(p->plan.ops.size());
+  return 0;
+}
+
+int northup_plan_get_op(northup_plan_t p, int64_t i, northup_op* out) {
+  if (!p || !out || i < 0 || i >= static_cast<int64_t>(p->plan.ops.size()))
+    return fail(NU_EINVAL, "bad op index");
+  *out = p->plan.ops[i];
+  return 0;
+}
+
+int northup_plan_num_bufs(northup_plan_t p, int* n) {
+  if (!p || !n) return fail(NU_EINVAL, "NULL argument");
+  *n = static_cast<int>(p->plan.bufs.size());
+  return 0;
+}
+
+int northup_plan_get_buf(northup_plan_t p, int i, northup_plan_buf* out) {
+  if (!p || !out || i < 0 || i >= static_cast<int>(p->plan.bufs.size()))
+    return fail(NU_EINVAL, "bad buffer index");
+  const PlanBuf& b = p->plan.bufs[i];
+  out->kind = b.kind;
+  out->node = b.node;
+  out->worker = b.worker;
+  out->bytes = b.bytes;
+  return 0;
+}
+
+int northup_plan_stats(northup_plan_t p, northup_stats* out) {
+  if (!p || !out) return fail(NU_EINVAL, "NULL argument");
+  *out = p->plan.stats;
+  return 0;
+}
+
+int northup_plan_destroy(northup_plan_t p) {
+  delete p;
+  return 0;
+}
+
+// --------------------------------------------------------- partitioner
+int northup_partition(int G, int64_t M, int64_t N, int64_t K, int* Pr, int* Pc) {
+  (void)K;
+  if (!Pr || !Pc) return fail(NU_EINVAL, "NULL argument");
+  return partition_grid(G, M, N, Pr, Pc);
+}
+
+int northup_partition_region(int G, int64_t M, int64_t N, int64_t K, int r, int64_t* r0,
+                             int64_t* r1, int64_t* c0, int64_t* c1) {
+  (void)K;
+  if (!r0 || !r1 || !c0 || !c1) return fail(NU_EINVAL, "NULL argument");
+  return region_of(G, M, N, r, r0, r1, c0, c1);
+}
+
+}  // extern "C"

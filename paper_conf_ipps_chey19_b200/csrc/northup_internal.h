@@ -1,0 +1,116 @@
+// Internal declarations shared by the translation units of libnorthup.so.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "northup.h"
+
+namespace nu {
+
+constexpr int kMaxDevices = 64;
+constexpr int64_t kDefaultKChunk = 1024;   // TMEM accumulation length
+constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
+
+// Thread-local error message (northup_last_error).  Returns its argument so
+// call sites can write `return fail(NU_EINVAL, "...")`.
+void set_error(const char* fmt, ...) __attribute__((format(printf, 1, 2)));
+int fail(int code, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+int cuda_fail(cudaError_t e, const char* what);
+
+// ------------------------------------------------------------------ tree
+struct Node {
+  int id = -1;
+  int storage = NU_HOST;
+  int phys = -1;
+  int processor = NU_PROC_NONE;
+  uint64_t capacity = 0;    // bytes, 0 = unbounded
+  uint64_t used = 0;        // bytes allocated by the library at this node
+  int level = 0;
+  int parent = -1;
+  std::vector<int> children;
+  int64_t bm = 0, bn = 0, bk = 0;   // block override (set_block)
+  // HBM nodes: arena used for plan buffers (slots, C block, tail buffers).
+  void* arena = nullptr;
+  uint64_t arena_bytes = 0;
+  bool arena_owned = false;
+};
+
+}  // namespace nu
+
+struct northup_buf_s {
+  northup_tree_t tree = nullptr;
+  int node = -1;
+  int storage = NU_HOST;
+  void* ptr = nullptr;       // host / device pointer (NULL for files)
+  int fd = -1;               // file descriptor (NU_FILE)
+  uint64_t bytes = 0;
+  bool owned = false;        // library allocated (freed on release/destroy)
+  bool registered = false;   // cudaHostRegister'ed by us (wrap_host)
+  bool direct = false;       // fd opened with O_DIRECT
+  std::string path;
+};
+
+struct WorkerState;
+
+struct northup_tree_s {
+  std::vector<nu::Node> nodes;
+  bool finalized = false;
+  bool busy = false;
+  std::string file_dir = "/tmp";
+  std::vector<northup_buf_s*> bufs;
+  std::vector<WorkerState*> workers;   // one per HBM node (created at finalize)
+};
+
+namespace nu {
+
+// --------------------------------------------------------------- plan
+enum Stream { S_H2D = 0, S_COMP = 1, S_D2H = 2, S_IO = 3, S_D2D = 4, S_NUM = 5 };
+enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3 };
+
+struct PlanBuf {
+  int kind = B_ARENA;
+  int node = -1;
+  int worker = -1;
+  uint64_t bytes = 0;   // elements * 4 for arenas (planned footprint)
+};
+
+struct Plan {
+  int64_t M = 0, N = 0, K = 0;
+  int num_workers = 0;
+  std::vector<int> worker_node;      // HBM node id per worker
+  std::vector<PlanBuf> bufs;
+  std::vector<northup_op> ops;
+  northup_stats stats{};
+  int64_t kc = kDefaultKChunk;
+  int npass = 3;
+  bool root_is_device = false;
+};
+
+int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
+               const northup_gemm_opts* o, Plan* out);
+// a_aligned / b_aligned: the root-tier device pointers are 16-B aligned
+// (only consulted for an HBM root, where the leaf reads them in place).
+int build_plan_ex(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
+                  const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out);
+int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc);
+int region_of(int G, int64_t M, int64_t N, int r, int64_t* r0, int64_t* r1, int64_t* c0,
+              int64_t* c1);
+int validate_tree(const northup_tree_s* t);
+
+// --------------------------------------------------------------- leaf
+bool leaf_tma_legal(const void* p, int64_t ld);
+int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
+                     int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
+                     int npass, cudaStream_t stream);
+
+// --------------------------------------------------------------- executor
+int execute_plan(northup_tree_s* t, const Plan& plan, void* a, void* b, void* c,
+                 const northup_gemm_opts* o, northup_stats* st);
+int finalize_workers(northup_tree_s* t);
+void destroy_workers(northup_tree_s* t);
+
+}  // namespace nu

@@ -1,0 +1,564 @@
+// Planner: the recursive decomposition of §IV-A over the Northup
+// tree, unrolled into a per-GPU list of operations (Listing 3 P:204-221 with
+// the recursion depth fixed by the tree).
+//
+//   level l (root, pinned host)  --data_down-->  level l+1 (HBM of GPU w)
+//   level l+1 (HBM)              --TMA------->   SMEM/TMEM leaf (the kernel)
+//
+// Each op is COPY (data_down / data_up over PCIe), LEAF (compute_task at the
+// leaf, accumulating partial sums) or ZERO.  Dependencies between ops
+// are derived here from the byte ranges each op reads and writes, so the
+// executor only has to turn them into CUDA stream waits.
+//
+// Schedules at the HOST -> HBM edge:
+//   S2  C block resident in HBM, K panels of A and B stream through a ring of
+//       kSlots slots; the last `tail_k` of K is computed strip by strip with a
+//       resident B tail so each finished C strip drains (D2H) while the next
+//       strip computes ("staggered drain").
+//   S1  paper-literal row-shard reuse: row shard m of A stays in HBM
+//       while the column shards of B stream; each C block drains when done.
+#include <algorithm>
+#include <cmath>
+
+#include "northup_internal.h"
+
+namespace nu {
+
+static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static int64_t rup(int64_t a, int64_t b) { return cdiv(a, b) * b; }
+static int64_t pad_ld(int64_t n) { return std::max<int64_t>(32, rup(n, 32)); }  // 128-B rows
+
+// Nominal planning constants: useful 3xTF32 flop rate and the
+// PCIe Gen5 x16 per-direction bandwidth.  Only used to size the drain tail.
+static constexpr double kPlanFlops = 250e12;
+static constexpr double kPlanPcie = 50e9;
+
+int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc) {
+  if (G <= 0) return fail(NU_EINVAL, "G must be positive");
+  int best_r = 1, best_c = G;
+  int64_t best = -1;
+  for (int r = 1; r <= G; ++r) {
+    if (G % r) continue;
+    const int c = G / r;
+    // per-GPU H2D bytes ~ 4K (M/Pr + N/Pc); ties go to more row splits so
+    // C regions stay contiguous in the row-major root.
+    const int64_t cost = cdiv(M, r) + cdiv(N, c);
+    if (best < 0 || cost < best || (cost == best && r > best_r)) {
+      best = cost;
+      best_r = r;
+      best_c = c;
+    }
+  }
+  *Pr = best_r;
+  *Pc = best_c;
+  return 0;
+}
+
+static void split_range(int64_t n, int parts, int i, int64_t* lo, int64_t* hi) {
+  const int64_t step = cdiv(n, parts);
+  *lo = std::min<int64_t>(n, step * i);
+  *hi = std::min<int64_t>(n, *lo + step);
+}
+
+int region_of(int G, int64_t M, int64_t N, int r, int64_t* r0, int64_t* r1, int64_t* c0,
+              int64_t* c1) {
+  int Pr = 1, Pc = 1;
+  int rc = partition_grid(G, M, N, &Pr, &Pc);
+  if (rc) return rc;
+  if (r < 0 || r >= G) return fail(NU_EINVAL, "region index out of range");
+  split_range(M, Pr, r / Pc, r0, r1);
+  split_range(N, Pc, r % Pc, c0, c1);
+  return 0;
+}
+
+namespace {
+
+struct Access {
+  int op;
+  int stream;
+  int64_t lo, hi;
+  bool write;
+};
+
+struct Builder {
+  Plan* P;
+  std::vector<std::vector<Access>> hist;   // per buffer
+
+  int add_buf(int kind, int node, int worker, uint64_t bytes) {
+    PlanBuf b;
+    b.kind = kind;
+    b.node = node;
+    b.worker = worker;
+    b.bytes = bytes;
+    P->bufs.push_back(b);
+    hist.emplace_back();
+    return static_cast<int>(P->bufs.size()) - 1;
+  }
+
+  struct Acc {
+    int buf;
+    int64_t off, ld, rows, cols;
+    bool write;
+  };
+
+  void emit(northup_op op, std::initializer_list<Acc> accs) {
+    const int idx = static_cast<int>(P->ops.size());
+    int last[S_NUM];
+    for (int& x : last) x = -1;
+    for (const Acc& a : accs) {
+      if (a.rows <= 0 || a.cols <= 0) continue;
+      const int64_t lo = a.off, hi = a.off + (a.rows - 1) * a.ld + a.cols;
+      auto& h = hist[a.buf];
+      for (const Access& p : h) {
+        if (p.hi <= lo || hi <= p.lo) continue;
+        if (!a.write && !p.write) continue;
+        if (p.stream == op.stream) continue;   // same stream: ordered already
+        if (P->ops[p.op].worker != op.worker) continue;   // sibling regions are disjoint
+        last[p.stream] = std::max(last[p.stream], p.op);
+      }
+      h.push_back(Access{idx, op.stream, lo, hi, a.write});
+    }
+    op.ndeps = 0;
+    for (int s = 0; s < S_NUM; ++s)
+      if (last[s] >= 0) op.deps[op.ndeps++] = last[s];
+    P->ops.push_back(op);
+  }
+};
+
+northup_op make_copy(int worker, int stream, int src, int64_t src_off, int64_t src_ld, int dst,
+                     int64_t dst_off, int64_t dst_ld, int64_t rows, int64_t cols) {
+  northup_op o{};
+  o.op = NU_OP_COPY;
+  o.worker = worker;
+  o.stream = stream;
+  o.src_buf = src;
+  o.dst_buf = dst;
+  o.src_off = src_off;
+  o.dst_off = dst_off;
+  o.src_ld = src_ld;
+  o.dst_ld = dst_ld;
+  o.rows = rows;
+  o.cols = cols;
+  o.a_buf = o.b_buf = o.c_buf = -1;
+  return o;
+}
+
+northup_op make_leaf(int worker, int a, int64_t a_off, int64_t lda, int b, int64_t b_off,
+                     int64_t ldb, int c, int64_t c_off, int64_t ldc, int64_t m, int64_t n, int64_t k,
+                     int accumulate) {
+  northup_op o{};
+  o.op = NU_OP_LEAF;
+  o.worker = worker;
+  o.stream = S_COMP;
+  o.a_buf = a;
+  o.b_buf = b;
+  o.c_buf = c;
+  o.a_off = a_off;
+  o.b_off = b_off;
+  o.c_off = c_off;
+  o.lda = lda;
+  o.ldb = ldb;
+  o.ldc = ldc;
+  o.m = m;
+  o.n = n;
+  o.k = k;
+  o.accumulate = accumulate;
+  o.src_buf = o.dst_buf = -1;
+  return o;
+}
+
+struct EdgeCtx {
+  Builder* B;
+  int worker;
+  int hbm_node;
+  int A, Bb, C;            // user buffers (root tier)
+  int64_t lda, ldb, ldc;   // root leading dims
+  int64_t r0, r1, c0, c1;  // region
+  int64_t K;
+  uint64_t cap;            // HBM capacity (bytes)
+  int64_t kc;
+  int64_t obm, obn, obk;   // block override at the parent node
+  int sched;
+};
+
+// ---------------------------------------------------------------- S2
+struct S2Shape {
+  int64_t bm, bn, bk, tail, sr;
+  uint64_t bytes;
+};
+
+uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, int64_t sr) {
+  const int64_t kmain = K - tail;
+  uint64_t e = static_cast<uint64_t>(bm) * pad_ld(bn);                    // C block
+  if (kmain > 0)
+    e += static_cast<uint64_t>(kSlots) *
+         (static_cast<uint64_t>(bm) * pad_ld(bk) + static_cast<uint64_t>(bk) * pad_ld(bn));
+  if (tail > 0)
+    e += static_cast<uint64_t>(tail) * pad_ld(bn) +                          // B tail
+         static_cast<uint64_t>(kSlots) * sr * pad_ld(tail);                  // A strips
+  return e * 4;
+}
+
+int choose_s2(const EdgeCtx& x, S2Shape* out) {
+  const int64_t m = x.r1 - x.r0, n = x.c1 - x.c0, K = x.K;
+  const uint64_t cap = x.cap ? x.cap : (uint64_t(1) << 62);
+  int64_t bk = x.obk > 0 ? x.obk : std::max<int64_t>(x.kc, 4);
+  bk = std::min<int64_t>(bk, rup(K, 4));
+  // drain tail: strip compute must cover the strip's D2H: K_t >= 2 P / BW.
+  int64_t want_tail = rup(static_cast<int64_t>(2.0 * kPlanFlops / kPlanPcie), x.kc);
+  std::vector<int64_t> bms, bns;
+  int64_t bm0 = x.obm > 0 ? std::min(x.obm, m) : m;
+  int64_t bn0 = x.obn > 0 ? std::min(x.obn, n) : n;
+  for (int64_t v = bm0;; v = rup(cdiv(v, 2), 128)) {
+    bms.push_back(v);
+    if (v <= 128) break;
+  }
+  for (int64_t v = bn0;; v = rup(cdiv(v, 2), 256)) {
+    bns.push_back(v);
+    if (v <= 256) break;
+  }
+  // Prefer whole-region blocks (fewest H2D bytes), then the longest tail.
+  for (int64_t bn : bns) {
+    for (int64_t bm : bms) {
+      const int64_t tails[] = {std::min(K, want_tail), std::min(K, want_tail / 2),
+                               std::min(K, x.kc), 0};
+      for (int64_t tail : tails) {
+        if (tail < 0) continue;
+        int64_t strips = std::max<int64_t>(1, std::min<int64_t>(16, cdiv(bm, 1024)));
+        int64_t sr = rup(cdiv(bm, strips), 128);
+        sr = std::min(sr, bm);
+        const uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr);
+        if (bytes <= cap) {
+          *out = S2Shape{bm, bn, bk, tail, sr, bytes};
+          return 0;
+        }
+      }
+      // also try the minimum panel
+      if (bk > x.kc && x.obk <= 0) {
+        const uint64_t bytes = s2_bytes(bm, bn, x.kc, K, 0, 0);
+        if (bytes <= cap) {
+          *out = S2Shape{bm, bn, x.kc, 0, 0, bytes};
+          return 0;
+        }
+      }
+    }
+  }
+  return fail(NU_ENOMEM, "HBM node %d capacity %llu B is below the minimum block", x.hbm_node,
+              (unsigned long long)x.cap);
+}
+
+int build_s2(const EdgeCtx& x, northup_stats* st) {
+  S2Shape s;
+  int rc = choose_s2(x, &s);
+  if (rc) return rc;
+  Builder& B = *x.B;
+  const int w = x.worker;
+  const int64_t m = x.r1 - x.r0, n = x.c1 - x.c0, K = x.K;
+  const int arena = B.add_buf(B_ARENA, x.hbm_node, w, s.bytes);
+  // arena layout (elements)
+  const int64_t ldC = pad_ld(s.bn), ldA = pad_ld(s.bk), ldBs = pad_ld(s.bn), ldAt = pad_ld(s.tail);
+  int64_t off = 0;
+  const int64_t offC = off;
+  off += s.bm * ldC;
+  const int64_t kmain = K - s.tail;
+  int64_t offSA[kSlots], offSB[kSlots], offAT[kSlots], offBT = 0;
+  for (int i = 0; i < kSlots; ++i) {
+    offSA[i] = off;
+    off += kmain > 0 ? s.bm * ldA : 0;
+    offSB[i] = off;
+    off += kmain > 0 ? s.bk * ldBs : 0;
+  }
+  if (s.tail > 0) {
+    offBT = off;
+    off += s.tail * ldBs;
+    for (int i = 0; i < kSlots; ++i) {
+      offAT[i] = off;
+      off += s.sr * ldAt;
+    }
+  }
+  if (w == 0) {
+    st->bm = s.bm;
+    st->bn = s.bn;
+    st->bk = s.bk;
+    st->tail_k = s.tail;
+    st->strips = s.tail > 0 ? cdiv(s.bm, s.sr) : 0;
+    st->hbm_peak_bytes = s.bytes;
+    st->schedule = NU_SCHED_S2;
+  }
+  int panel_it = 0, strip_it = 0;
+  for (int64_t i0 = 0; i0 < m; i0 += s.bm) {
+    const int64_t bm = std::min(s.bm, m - i0);
+    for (int64_t j0 = 0; j0 < n; j0 += s.bn) {
+      const int64_t bn = std::min(s.bn, n - j0);
+      const int64_t gr = x.r0 + i0, gc = x.c0 + j0;   // global row/col of the block
+      // ---- main phase: K panels [0, kmain)
+      const int64_t npan = kmain > 0 ? cdiv(kmain, s.bk) : 0;
+      const int64_t ntail_pieces = s.tail > 0 ? cdiv(s.tail, s.bk) : 0;
+      int64_t pieces_done = 0;
+      auto load_tail_piece = [&](int64_t piece) {
+        const int64_t k0 = kmain + piece * s.bk, kk = std::min(s.bk, K - k0);
+        B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc, x.ldb, arena, offBT + (k0 - kmain) * ldBs,
+                         ldBs, kk, bn),
+               {{x.Bb, k0 * x.ldb + gc, x.ldb, kk, bn, false},
+                {arena, offBT + (k0 - kmain) * ldBs, ldBs, kk, bn, true}});
+        st->bytes_h2d += static_cast<uint64_t>(kk) * bn * 4;
+      };
+      for (int64_t p = 0; p < npan; ++p, ++panel_it) {
+        const int sl = panel_it % kSlots;
+        const int64_t k0 = p * s.bk, kk = std::min(s.bk, kmain - k0);
+        B.emit(make_copy(w, S_H2D, x.A, gr * x.lda + k0, x.lda, arena, offSA[sl], ldA, bm, kk),
+               {{x.A, gr * x.lda + k0, x.lda, bm, kk, false}, {arena, offSA[sl], ldA, bm, kk, true}});
+        B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc, x.ldb, arena, offSB[sl], ldBs, kk, bn),
+               {{x.Bb, k0 * x.ldb + gc, x.ldb, kk, bn, false},
+                {arena, offSB[sl], ldBs, kk, bn, true}});
+        st->bytes_h2d += static_cast<uint64_t>(bm) * kk * 4 + static_cast<uint64_t>(kk) * bn * 4;
+        B.emit(make_leaf(w, arena, offSA[sl], ldA, arena, offSB[sl], ldBs, arena, offC, ldC, bm, bn,
+                         kk, p > 0 ? 1 : 0),
+               {{arena, offSA[sl], ldA, bm, kk, false},
+                {arena, offSB[sl], ldBs, kk, bn, false},
+                {arena, offC, ldC, bm, bn, true}});
+        st->leaf_launches++;
+        // interleave the B-tail pieces over the main phase so they overlap compute
+        while (pieces_done < ntail_pieces && (pieces_done + 1) * npan <= (p + 1) * ntail_pieces) {
+          load_tail_piece(pieces_done++);
+        }
+      }
+      while (pieces_done < ntail_pieces) load_tail_piece(pieces_done++);
+      if (s.tail > 0) {
+        // ---- tail phase: strips of C finish and drain one by one
+        for (int64_t r = 0; r < bm; r += s.sr, ++strip_it) {
+          const int64_t rr = std::min(s.sr, bm - r);
+          const int sl = strip_it % kSlots;
+          B.emit(make_copy(w, S_H2D, x.A, (gr + r) * x.lda + kmain, x.lda, arena, offAT[sl], ldAt, rr,
+                           s.tail),
+                 {{x.A, (gr + r) * x.lda + kmain, x.lda, rr, s.tail, false},
+                  {arena, offAT[sl], ldAt, rr, s.tail, true}});
+          st->bytes_h2d += static_cast<uint64_t>(rr) * s.tail * 4;
+          B.emit(make_leaf(w, arena, offAT[sl], ldAt, arena, offBT, ldBs, arena, offC + r * ldC, ldC,
+                           rr, bn, s.tail, kmain > 0 ? 1 : 0),
+                 {{arena, offAT[sl], ldAt, rr, s.tail, false},
+                  {arena, offBT, ldBs, s.tail, bn, false},
+                  {arena, offC + r * ldC, ldC, rr, bn, true}});
+          st->leaf_launches++;
+          B.emit(make_copy(w, S_D2H, arena, offC + r * ldC, ldC, x.C, (gr + r) * x.ldc + gc, x.ldc, rr,
+                           bn),
+                 {{arena, offC + r * ldC, ldC, rr, bn, false},
+                  {x.C, (gr + r) * x.ldc + gc, x.ldc, rr, bn, true}});
+          st->bytes_d2h += static_cast<uint64_t>(rr) * bn * 4;
+        }
+      } else {
+        B.emit(make_copy(w, S_D2H, arena, offC, ldC, x.C, gr * x.ldc + gc, x.ldc, bm, bn),
+               {{arena, offC, ldC, bm, bn, false}, {x.C, gr * x.ldc + gc, x.ldc, bm, bn, true}});
+        st->bytes_d2h += static_cast<uint64_t>(bm) * bn * 4;
+      }
+    }
+  }
+  return 0;
+}
+
+// ---------------------------------------------------------------- S1
+int build_s1(const EdgeCtx& x, northup_stats* st) {
+  Builder& B = *x.B;
+  const int w = x.worker;
+  const int64_t m = x.r1 - x.r0, n = x.c1 - x.c0, K = x.K;
+  const uint64_t cap = x.cap ? x.cap : (uint64_t(1) << 62);
+  int64_t bm = x.obm > 0 ? std::min(x.obm, m) : std::min<int64_t>(m, 4096);
+  int64_t bn = x.obn > 0 ? std::min(x.obn, n) : std::min<int64_t>(n, 4096);
+  int64_t bk = x.obk > 0 ? std::min(x.obk, rup(K, 4)) : std::min<int64_t>(rup(K, 4), x.kc);
+  auto bytes_of = [&](int64_t bm_, int64_t bn_, int64_t bk_) -> uint64_t {
+    return 4ull * (2ull * bm_ * pad_ld(K)             // two row shards (next prefetches)
+                   + 2ull * bm_ * pad_ld(bn_)         // double-buffered C block
+                   + uint64_t(kSlots) * bk_ * pad_ld(bn_));
+  };
+  while (bytes_of(bm, bn, bk) > cap) {
+    if (bm > 128 && x.obm <= 0) bm = rup(cdiv(bm, 2), 128);
+    else if (bn > 256 && x.obn <= 0) bn = rup(cdiv(bn, 2), 256);
+    else return fail(NU_ENOMEM, "HBM node %d capacity too small for S1 blocks", x.hbm_node);
+  }
+  const uint64_t bytes = bytes_of(bm, bn, bk);
+  const int arena = B.add_buf(B_ARENA, x.hbm_node, w, bytes);
+  const int64_t ldAs = pad_ld(K), ldC = pad_ld(bn), ldB = pad_ld(bn);
+  int64_t off = 0, offAs[2], offC[2], offB[kSlots];
+  for (int i = 0; i < 2; ++i) { offAs[i] = off; off += bm * ldAs; }
+  for (int i = 0; i < 2; ++i) { offC[i] = off; off += bm * ldC; }
+  for (int i = 0; i < kSlots; ++i) { offB[i] = off; off += bk * ldB; }
+  if (w == 0) {
+    st->bm = bm;
+    st->bn = bn;
+    st->bk = bk;
+    st->hbm_peak_bytes = bytes;
+    st->schedule = NU_SCHED_S1;
+  }
+  int shard = 0, cblk = 0, pit = 0;
+  for (int64_t i0 = 0; i0 < m; i0 += bm, ++shard) {
+    const int64_t rm = std::min(bm, m - i0);
+    const int64_t gr = x.r0 + i0;
+    const int as = shard & 1;
+    // row shard m moves to level l+1 once and stays
+    B.emit(make_copy(w, S_H2D, x.A, gr * x.lda, x.lda, arena, offAs[as], ldAs, rm, K),
+           {{x.A, gr * x.lda, x.lda, rm, K, false}, {arena, offAs[as], ldAs, rm, K, true}});
+    st->bytes_h2d += static_cast<uint64_t>(rm) * K * 4;
+    for (int64_t j0 = 0; j0 < n; j0 += bn, ++cblk) {
+      const int64_t cn = std::min(bn, n - j0);
+      const int64_t gc = x.c0 + j0;
+      const int cb = cblk & 1;
+      for (int64_t k0 = 0; k0 < K; k0 += bk, ++pit) {
+        const int64_t kk = std::min(bk, K - k0);
+        const int sl = pit % kSlots;
+        B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc, x.ldb, arena, offB[sl], ldB, kk, cn),
+               {{x.Bb, k0 * x.ldb + gc, x.ldb, kk, cn, false}, {arena, offB[sl], ldB, kk, cn, true}});
+        st->bytes_h2d += static_cast<uint64_t>(kk) * cn * 4;
+        B.emit(make_leaf(w, arena, offAs[as] + k0, ldAs, arena, offB[sl], ldB, arena, offC[cb], ldC,
+                         rm, cn, kk, k0 > 0 ? 1 : 0),
+               {{arena, offAs[as] + k0, ldAs, rm, kk, false},
+                {arena, offB[sl], ldB, kk, cn, false},
+                {arena, offC[cb], ldC, rm, cn, true}});
+        st->leaf_launches++;
+      }
+      B.emit(make_copy(w, S_D2H, arena, offC[cb], ldC, x.C, gr * x.ldc + gc, x.ldc, rm, cn),
+             {{arena, offC[cb], ldC, rm, cn, false}, {x.C, gr * x.ldc + gc, x.ldc, rm, cn, true}});
+      st->bytes_d2h += static_cast<uint64_t>(rm) * cn * 4;
+    }
+  }
+  return 0;
+}
+
+// In-HBM (single-node HBM tree, CS4): the leaf runs directly on the caller's
+// device buffers; operands whose layout TMA cannot address are first copied
+// into padded arena buffers (R16 layout transformation during move_data).
+int build_in_hbm(Builder& B, int node, int64_t M, int64_t N, int64_t K, int A, int Bb, int C,
+                 bool a_ok, bool b_ok, northup_stats* st) {
+  const int64_t ldA = pad_ld(K), ldB = pad_ld(N);
+  uint64_t bytes = 0;
+  if (!a_ok) bytes += 4ull * M * ldA;
+  if (!b_ok) bytes += 4ull * K * ldB;
+  int arena = -1;
+  int64_t offA = 0, offB = a_ok ? 0 : M * ldA;
+  if (bytes) arena = B.add_buf(B_ARENA, node, 0, bytes);
+  int a = A, b = Bb;
+  int64_t la = K, lb = N, oa = 0, ob = 0;
+  if (!a_ok) {
+    B.emit(make_copy(0, S_COMP, A, 0, K, arena, offA, ldA, M, K),
+           {{A, 0, K, M, K, false}, {arena, offA, ldA, M, K, true}});
+    st->bytes_d2d += 4ull * M * K;
+    a = arena, la = ldA, oa = offA;
+  }
+  if (!b_ok) {
+    B.emit(make_copy(0, S_COMP, Bb, 0, N, arena, offB, ldB, K, N),
+           {{Bb, 0, N, K, N, false}, {arena, offB, ldB, K, N, true}});
+    st->bytes_d2d += 4ull * K * N;
+    b = arena, lb = ldB, ob = offB;
+  }
+  B.emit(make_leaf(0, a, oa, la, b, ob, lb, C, 0, N, M, N, K, 0),
+         {{a, oa, la, M, K, false}, {b, ob, lb, K, N, false}, {C, 0, N, M, N, true}});
+  st->leaf_launches++;
+  st->bm = M;
+  st->bn = N;
+  st->bk = K;
+  st->hbm_peak_bytes = bytes;
+  st->schedule = NU_SCHED_AUTO;
+  return 0;
+}
+
+}  // namespace
+
+// Which HBM nodes compute, and what sits above them.
+int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K, const northup_gemm_opts* o,
+               Plan* out) {
+  return build_plan_ex(t, M, N, K, o, true, true, out);
+}
+
+int build_plan_ex(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
+                  const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out) {
+  int rc = validate_tree(t);
+  if (rc) return rc;
+  if (M < 0 || N < 0 || K < 0) return fail(NU_EINVAL, "negative dimension");
+  Plan& P = *out;
+  P = Plan();
+  P.M = M;
+  P.N = N;
+  P.K = K;
+  P.kc = (o && o->k_chunk > 0) ? o->k_chunk : kDefaultKChunk;
+  if (P.kc % 4) return fail(NU_EINVAL, "k_chunk must be a multiple of 4");
+  P.npass = (o && o->npass == 1) ? 1 : 3;
+  const int sched = o ? o->schedule : NU_SCHED_AUTO;
+  if (sched < NU_SCHED_AUTO || sched > NU_SCHED_S2) return fail(NU_EINVAL, "unknown schedule");
+  Builder B;
+  B.P = &P;
+  const int A = B.add_buf(B_USER_A, 0, -1, 4ull * M * K);
+  const int Bb = B.add_buf(B_USER_B, 0, -1, 4ull * K * N);
+  const int C = B.add_buf(B_USER_C, 0, -1, 4ull * M * N);
+  northup_stats& st = P.stats;
+  st = northup_stats{};
+  const nu::Node& root = t->nodes[0];
+
+  if (root.storage == NU_HBM) {
+    // single-node HBM tree (or HBM -> SMEM leaf): the in-HBM reference (CS4)
+    P.root_is_device = true;
+    P.num_workers = 1;
+    P.worker_node.push_back(0);
+    st.num_gpus = 1;
+    if (M == 0 || N == 0 || K == 0) return 0;
+    // Layout legality is decided by the executor against real pointers; the
+    // plan assumes dense ld = K / N and records whether those are TMA-legal.
+    rc = build_in_hbm(B, 0, M, N, K, A, Bb, C, a_aligned && K % 4 == 0, b_aligned && N % 4 == 0,
+                      &st);
+    st.ops = static_cast<int64_t>(P.ops.size());
+    return rc;
+  }
+  if (root.storage == NU_FILE)
+    return fail(NU_ENOTSUP, "FILE roots are planned by the staging engine (northup_gemm_file)");
+  if (root.storage != NU_HOST) return fail(NU_EINVAL, "root must be FILE, HOST or HBM");
+
+  // HOST root: its children must be the HBM siblings (branch parallelism).
+  std::vector<int> hbm;
+  for (int c : root.children) {
+    if (t->nodes[c].storage != NU_HBM)
+      return fail(NU_ENOTSUP, "HOST root children must be HBM nodes (node %d is not)", c);
+    hbm.push_back(c);
+  }
+  if (hbm.empty()) return fail(NU_EINVAL, "HOST root has no HBM child");
+  const int G = static_cast<int>(hbm.size());
+  P.num_workers = G;
+  P.worker_node = hbm;
+  st.num_gpus = G;
+  if (M == 0 || N == 0 || K == 0) return 0;
+  for (int w = 0; w < G; ++w) {
+    EdgeCtx x;
+    x.B = &B;
+    x.worker = w;
+    x.hbm_node = hbm[w];
+    x.A = A;
+    x.Bb = Bb;
+    x.C = C;
+    x.lda = K;
+    x.ldb = N;
+    x.ldc = N;
+    rc = region_of(G, M, N, w, &x.r0, &x.r1, &x.c0, &x.c1);
+    if (rc) return rc;
+    if (x.r1 <= x.r0 || x.c1 <= x.c0) continue;   // more GPUs than rows/cols
+    x.K = K;
+    x.cap = t->nodes[hbm[w]].capacity;
+    x.kc = P.kc;
+    x.obm = root.bm;
+    x.obn = root.bn;
+    x.obk = root.bk;
+    x.sched = sched;
+    int use = sched;
+    if (use == NU_SCHED_AUTO) {
+      // P:299's row-shard reuse when the caller fixed blocks smaller than the
+      // region (cfg1's 64 x 64 blocks); otherwise the C-resident schedule.
+      const bool small_blocks = (root.bm > 0 && root.bm < x.r1 - x.r0) ||
+                                (root.bn > 0 && root.bn < x.c1 - x.c0);
+      use = small_blocks ? NU_SCHED_S1 : NU_SCHED_S2;
+    }
+    rc = use == NU_SCHED_S1 ? build_s1(x, &st) : build_s2(x, &st);
+    if (rc) return rc;
+  }
+  st.ops = static_cast<int64_t>(P.ops.size());
+  for (const northup_op& op : P.ops)
+    if (op.op == NU_OP_COPY) st.copies++;
+  return 0;
+}
+
+}  // namespace nu

@@ -1,0 +1,228 @@
+"""Host-side tests of the C ABI (no GPU): the library loads and exports every
+symbol include/northup.h declares; the tree (Listing 1) validates and
+answers queries; the planner's op lists compute C = A.B exactly when replayed
+by a CPU simulator in ANY order the dependencies allow (so the dependencies
+are sufficient), move the closed-form number of bytes, and stay within node
+capacities; the partitioner picks the grids of SURVEY.md §8(e)."""
+import random
+
+import numpy as np
+import pytest
+
+import nugen
+import paper_conf_ipps_chey19_b200 as nu
+
+GiB = 1 << 30
+
+
+def test_library_exports_every_header_symbol():
+    syms = nu.header_symbols()
+    assert len(syms) >= 35
+    L = nu.lib()
+    missing = [s for s in syms if not hasattr(L, s)]
+    assert not missing
+    assert nu.version() == 100
+
+
+def test_tree_queries_and_levels():
+    t = nu.Tree()
+    root = t.add_node(-1, nu.NU_HOST)
+    h0 = t.add_node(root, nu.NU_HBM, 0, 8 * GiB)
+    s0 = t.add_node(h0, nu.NU_SMEM, 0, 227 * 1024, nu.NU_PROC_SM100)
+    h1 = t.add_node(root, nu.NU_HBM, 1, 8 * GiB, nu.NU_PROC_SM100)
+    assert [t.get_level(n) for n in (root, h0, s0, h1)] == [0, 1, 2, 1]
+    assert t.get_max_treelevel() == 2
+    assert t.get_children_list(root) == [h0, h1]
+    assert t.get_parent(s0) == h0 and t.get_parent(root) == -1
+    assert t.fetch_node_type(h1) == nu.NU_HBM
+    info = t.node_info(s0)
+    assert info["is_leaf"] == 1 and info["processor_type"] == nu.NU_PROC_SM100
+    txt = t.print()
+    assert "HOST" in txt and "SMEM" in txt and "(leaf)" in txt and txt.count("\n") == 4
+    t.destroy()
+
+
+def test_tree_errors():
+    t = nu.Tree()
+    root = t.add_node(-1, nu.NU_HOST)
+    with pytest.raises(nu.NorthupError) as e:
+        t.add_node(-1, nu.NU_HOST)            # a second root
+    assert e.value.code == nu.NU_EINVAL
+    with pytest.raises(nu.NorthupError):
+        t.add_node(17, nu.NU_HBM, 0)          # unknown parent
+    with pytest.raises(nu.NorthupError):
+        t.set_block(root, 64, 64, 30)         # bk not a multiple of 4
+    h = t.add_node(root, nu.NU_HBM, 0)        # leaf without a processor
+    with pytest.raises(nu.NorthupError) as e:
+        t.finalize()
+    assert e.value.code == nu.NU_EINVAL and "processor" in str(e.value)
+    t.destroy()
+    t = nu.Tree()
+    h = t.add_node(-1, nu.NU_HBM, 0)
+    t.add_node(h, nu.NU_HOST, -1, 0, nu.NU_PROC_SM100)   # edge to slower memory
+    with pytest.raises(nu.NorthupError):
+        t.finalize()
+    t.destroy()
+
+
+def test_gemm_needs_finalized_tree():
+    t, _ = nu.host_tree(1)
+    with pytest.raises(nu.NorthupError):
+        nu.check(nu.lib().northup_gemm(t.handle, None, None, None, 4, 4, 4))
+    t.destroy()
+
+
+@pytest.mark.parametrize("G,M,N,grid", [(2, 65536, 65536, (2, 1)), (4, 65536, 65536, (2, 2)),
+                                         (8, 65536, 65536, (4, 2)), (8, 1048576, 4096, (8, 1)),
+                                         (1, 10, 10, (1, 1)), (3, 300, 900, (1, 3))])
+def test_partition_grid(G, M, N, grid):
+    assert nu.partition(G, M, N) == grid
+    seen = np.zeros((M // 64 + 1, N // 64 + 1), dtype=int) if M * N > 1e6 else np.zeros((M, N), int)
+    if M * N <= 1e6:
+        for r in range(G):
+            r0, r1, c0, c1 = nu.partition_region(G, M, N, 0, r)
+            seen[r0:r1, c0:c1] += 1
+        assert (seen == 1).all()
+
+
+# ------------------------------------------------------------ plan simulator
+def simulate(plan: nu.Plan, A, B, M, N, K, rng=None):
+    """Replay the plan's ops on host arrays (float64, exact on integers).
+    With `rng`, ops run in a random order consistent with the dependencies
+    and with in-order execution per (worker, stream)."""
+    bufs = plan.bufs()
+    ops = plan.ops()
+    mem = []
+    for b in bufs:
+        if b["kind"] == 0:
+            mem.append(A.astype(np.float64).ravel().copy())
+        elif b["kind"] == 1:
+            mem.append(B.astype(np.float64).ravel().copy())
+        elif b["kind"] == 2:
+            mem.append(np.full(M * N, np.nan))
+        else:
+            mem.append(np.full(b["bytes"] // 4, np.nan))
+
+    def view(buf, off, ld, rows, cols):
+        return np.lib.stride_tricks.as_strided(mem[buf][off:], shape=(rows, cols),
+                                               strides=(ld * 8, 8), writeable=True)
+
+    def run(op):
+        if op["op"] == nu.NU_OP_COPY:
+            view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
+                view(op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
+        elif op["op"] == nu.NU_OP_LEAF:
+            a = view(op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
+            b = view(op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"])
+            c = view(op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])
+            prod = a @ b
+            c[...] = (c + prod) if op["accumulate"] else prod
+        else:
+            view(op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])[...] = 0
+
+    if rng is None:
+        for op in ops:
+            run(op)
+    else:
+        queues = {}
+        for i, op in enumerate(ops):
+            queues.setdefault((op["worker"], op["stream"]), []).append(i)
+        done = set()
+        while len(done) < len(ops):
+            ready = [q for q in queues.values() if q and all(d in done for d in ops[q[0]]["deps"])]
+            assert ready, "deadlock: dependencies form a cycle"
+            q = rng.choice(ready)
+            i = q.pop(0)
+            run(ops[i])
+            done.add(i)
+    return mem[[b["kind"] for b in bufs].index(2)].reshape(M, N)
+
+
+def _plan_case(M, N, K, G=1, cap=0, block=None, sched=nu.NU_SCHED_AUTO, kc=0):
+    t, _ = nu.host_tree(G, cap)
+    if block:
+        t.set_block(0, *block)
+    p = t.plan(M, N, K, nu.make_opts(schedule=sched, k_chunk=kc))
+    return t, p
+
+
+@pytest.mark.parametrize("M,N,K,G,cap,block,sched,kc", [
+    (256, 256, 256, 1, 0, (64, 64, 64), nu.NU_SCHED_AUTO, 0),     # cfg1 shape (S1)
+    (300, 200, 130, 1, 0, None, nu.NU_SCHED_AUTO, 0),             # ragged, S2 all-tail
+    (513, 300, 777, 2, 0, None, nu.NU_SCHED_S2, 64),              # S2, 2 GPUs, small kc
+    (400, 520, 1000, 1, 600_000, None, nu.NU_SCHED_S2, 32),       # capacity forces blocks
+    (200, 300, 150, 4, 0, (64, 96, 40), nu.NU_SCHED_S1, 0),       # S1 on 4 GPUs
+    (1, 1, 1, 1, 0, None, nu.NU_SCHED_AUTO, 0),
+])
+def test_plan_simulation_exact(M, N, K, G, cap, block, sched, kc):
+    A = nugen.fill(M, K, 3, 1, "int")
+    B = nugen.fill(K, N, 3, 2, "int")
+    ref = A.astype(np.float64) @ B.astype(np.float64)
+    t, p = _plan_case(M, N, K, G, cap, block, sched, kc)
+    assert np.array_equal(simulate(p, A, B, M, N, K), ref)
+    for seed in range(4):
+        C = simulate(p, A, B, M, N, K, rng=random.Random(seed))
+        assert np.array_equal(C, ref), f"order seed {seed} broke a dependency"
+    if cap:
+        assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
+    t.destroy()
+
+
+def test_plan_bytes_closed_forms():
+    # S2 with a whole-region C block: every A and B byte crosses PCIe once,
+    # C comes back once (H2D = 4K(r + c), D2H = 4rc).
+    M, N, K = 4096, 2048, 8192
+    t, p = _plan_case(M, N, K, sched=nu.NU_SCHED_S2)
+    s = p.stats()
+    assert s["bytes_h2d"] == 4 * K * (M + N) and s["bytes_d2h"] == 4 * M * N
+    assert s["bm"] == M and s["bn"] == N and s["schedule"] == nu.NU_SCHED_S2
+    t.destroy()
+    # S1 (paper-literal): A once, B once per row shard: 4MK + 4KN ceil(M/bm)
+    M, N, K, bm = 256, 256, 256, 64
+    t, p = _plan_case(M, N, K, block=(bm, 64, 64))
+    s = p.stats()
+    assert s["schedule"] == nu.NU_SCHED_S1
+    assert s["bytes_h2d"] == 4 * M * K + 4 * K * N * (M // bm) and s["bytes_d2h"] == 4 * M * N
+    assert s["leaf_launches"] == (M // 64) * (N // 64) * (K // 64)
+    t.destroy()
+
+
+def test_cfg3_plan_shape():
+    """cfg3: 32768^3, 8 GiB HBM cap -> C resident, staggered drain, footprint <= cap."""
+    M = N = K = 32768
+    t, p = _plan_case(M, N, K, cap=8 * GiB)
+    s = p.stats()
+    assert s["schedule"] == nu.NU_SCHED_S2 and s["bm"] == M and s["bn"] == N
+    assert 0 < s["tail_k"] < K and s["tail_k"] % 1024 == 0 and s["strips"] >= 8
+    assert s["hbm_peak_bytes"] <= 8 * GiB
+    assert s["bytes_h2d"] == 4 * K * (M + N) and s["bytes_d2h"] == 4 * M * N
+    ks = [op["k"] for op in p.ops() if op["op"] == nu.NU_OP_LEAF]
+    assert all(k % 1024 == 0 for k in ks)            # panel edges on k_chunk multiples
+    t.destroy()
+
+
+def test_capacity_below_minimum_block():
+    t, _ = nu.host_tree(1, 4096)
+    with pytest.raises(nu.NorthupError) as e:
+        t.plan(1024, 1024, 1024)
+    assert e.value.code == nu.NU_ENOMEM
+    t.destroy()
+
+
+def test_hbm_root_plan_is_one_leaf():
+    t = nu.hbm_tree(0)
+    p = t.plan(8192, 8192, 8192)
+    ops = p.ops()
+    assert len(ops) == 1 and ops[0]["op"] == nu.NU_OP_LEAF and ops[0]["k"] == 8192
+    p2 = t.plan(100, 30, 7)    # K % 4 != 0: A is staged into a padded arena copy
+    kinds = [o["op"] for o in p2.ops()]
+    assert kinds == [nu.NU_OP_COPY, nu.NU_OP_COPY, nu.NU_OP_LEAF][:len(kinds)] or \
+        kinds == [nu.NU_OP_COPY, nu.NU_OP_LEAF]
+    t.destroy()
+
+
+def test_data_api_host_only_errors():
+    t, _ = nu.host_tree(1)
+    with pytest.raises(nu.NorthupError):
+        t.alloc(64, 2)     # SMEM node: managed by the leaf kernel
+    t.destroy()

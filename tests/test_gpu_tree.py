@@ -1,0 +1,167 @@
+"""End-to-end parity of northup_gemm through the C ABI: HOST root -> HBM ->
+SMEM/TMEM leaf (and the in-HBM single-node tree), against the fp64 oracle on
+the same seeded inputs."""
+import ctypes
+
+import numpy as np
+import pytest
+import torch
+
+import nugen
+import oracle
+import paper_conf_ipps_chey19_b200 as nu
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+GiB = 1 << 30
+
+
+def host_view(buf, rows, cols):
+    n = rows * cols
+    if n == 0:
+        return np.zeros((rows, cols), np.float32)
+    arr = (ctypes.c_float * n).from_address(buf.ptr)
+    return np.ctypeslib.as_array(arr).reshape(rows, cols)
+
+
+class HostProblem:
+    """A, B, C allocated at the HOST root through Table I's alloc()."""
+
+    def __init__(self, tree, M, N, K, seed, kind="uniform"):
+        self.M, self.N, self.K = M, N, K
+        self.A = tree.alloc(4 * M * K, 0)
+        self.B = tree.alloc(4 * K * N, 0)
+        self.C = tree.alloc(4 * M * N, 0)
+        self.a = host_view(self.A, M, K)
+        self.b = host_view(self.B, K, N)
+        self.c = host_view(self.C, M, N)
+        nugen.fill(M, K, seed, nugen.MAT_A, kind, out=self.a)
+        nugen.fill(K, N, seed, nugen.MAT_B, kind, out=self.b)
+        if M * N:
+            self.c[...] = np.nan
+
+
+def run_host(M, N, K, G=1, cap=0, block=None, kind="uniform", seed=1, **opt):
+    t, _ = nu.host_tree(G, cap, devices=[0] * G)     # G "virtual siblings" on GPU 0 (T5)
+    if block:
+        t.set_block(0, *block)
+    t.finalize()
+    p = HostProblem(t, M, N, K, seed, kind)
+    st = t.gemm(p.A, p.B, p.C, M, N, K, nu.make_opts(**opt))
+    C = p.c.copy()
+    a, b = p.a.copy(), p.b.copy()
+    t.destroy()
+    return C, a, b, st
+
+
+def check(C, a, b, kind):
+    ref = oracle.gemm(a, b)
+    if kind == "int":
+        assert np.array_equal(C.astype(np.float64), ref)
+    else:
+        e, where = oracle.normwise_err(C, ref, oracle.row_norms(a), oracle.col_norms(b))
+        assert e <= TOL, (e, where)
+
+
+def test_cfg1_two_level_tree_64_blocks():
+    """BASELINE.json configs[0]: 256^3, host DRAM -> 1 GPU leaf, 64 x 64 blocks."""
+    for kind in ("uniform", "int"):
+        C, a, b, st = run_host(256, 256, 256, block=(64, 64, 64), kind=kind)
+        check(C, a, b, kind)
+        assert st["schedule"] == nu.NU_SCHED_S1 and st["leaf_launches"] == 64
+
+
+@pytest.mark.parametrize("M,N,K,G,cap,sched,kc", [
+    (300, 200, 130, 1, 0, 0, 0),
+    (1, 1, 1, 1, 0, 0, 0),
+    (513, 777, 2100, 1, 0, nu.NU_SCHED_S2, 256),
+    (1000, 1200, 3000, 1, 6_000_000, nu.NU_SCHED_S2, 512),   # capacity -> several C blocks
+    (640, 900, 1500, 2, 0, 0, 0),                            # 2 siblings, one device
+    (500, 700, 333, 4, 0, nu.NU_SCHED_S1, 0),
+    (2048, 2048, 12288, 1, 0, nu.NU_SCHED_S2, 1024),         # main phase + drain tail
+])
+@pytest.mark.parametrize("kind", ["uniform", "int"])
+def test_host_root_gemm(M, N, K, G, cap, sched, kc, kind):
+    C, a, b, st = run_host(M, N, K, G=G, cap=cap, schedule=sched, k_chunk=kc, kind=kind)
+    check(C, a, b, kind)
+    assert st["num_gpus"] == G
+
+
+def test_zero_k_and_empty():
+    C, a, b, st = run_host(7, 9, 0)
+    assert (C == 0).all()
+    run_host(0, 5, 5)
+    run_host(5, 0, 5)
+
+
+def test_in_hbm_tree_and_cross_tier_bitwise():
+    """CS4: the single-node HBM tree runs the same leaf; with K-panel edges on
+    k_chunk multiples the out-of-core result is bitwise identical (§8(c) (4))."""
+    M, N, K = 1536, 1024, 6144
+    C_ooc, a, b, st = run_host(M, N, K, schedule=nu.NU_SCHED_S2, k_chunk=1024)
+    assert st["tail_k"] > 0 and st["leaf_launches"] > 1
+    dev = torch.device("cuda:0")
+    Ad = torch.from_numpy(a).to(dev)
+    Bd = torch.from_numpy(b).to(dev)
+    Cd = torch.full((M, N), float("nan"), device=dev)
+    t = nu.hbm_tree(0)
+    t.finalize()
+    bA = t.wrap_device(0, Ad.data_ptr(), Ad.numel() * 4)
+    bB = t.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4)
+    bC = t.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4)
+    t.gemm(bA, bB, bC, M, N, K, nu.make_opts(k_chunk=1024))
+    torch.cuda.synchronize()
+    C_hbm = Cd.cpu().numpy()
+    t.destroy()
+    check(C_hbm, a, b, "uniform")
+    assert np.array_equal(C_hbm, C_ooc)
+
+
+def test_in_hbm_unaligned_operands_staged():
+    """K % 4 != 0: the HBM root stages A into a padded arena (R16)."""
+    M, N, K = 130, 66, 37
+    a = nugen.fill(M, K, 5, 1, "int")
+    b = nugen.fill(K, N, 5, 2, "int")
+    dev = torch.device("cuda:0")
+    Ad, Bd = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
+    Cd = torch.zeros((M, N), device=dev)
+    t = nu.hbm_tree(0)
+    t.finalize()
+    st = t.gemm(t.wrap_device(0, Ad.data_ptr(), Ad.numel() * 4),
+                t.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4),
+                t.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4), M, N, K)
+    assert st["bytes_d2d"] > 0
+    assert np.array_equal(Cd.cpu().numpy().astype(np.float64), oracle.gemm(a, b))
+    t.destroy()
+
+
+def test_cross_g_bitwise():
+    """Same K-panel sequence on G = 1 / 2 / 4 siblings gives identical C."""
+    M, N, K = 1024, 768, 4096
+    outs = [run_host(M, N, K, G=G, schedule=nu.NU_SCHED_S2, k_chunk=1024)[0] for G in (1, 2, 4)]
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
+
+
+def test_data_api_round_trip():
+    """Table I: alloc at HOST and HBM, move_data down and up, byte exact."""
+    t, hbm = nu.host_tree(1)
+    t.finalize()
+    h = t.alloc(1 << 20, 0)
+    d = t.alloc(1 << 20, hbm[0])
+    back = t.alloc(1 << 20, 0)
+    x = host_view(h, 256, 1024)
+    x[...] = nugen.fill(256, 1024, 9, 1)
+    t.move_data_down(d, h, 1 << 20, 0, 0)
+    t.move_data_up(back, d, 1 << 20, 0)
+    assert np.array_equal(host_view(back, 256, 1024), x)
+    assert t.node_info(hbm[0])["used"] >= 1 << 20
+    t.destroy()
+
+
+def test_hbm_capacity_enforced():
+    t, hbm = nu.host_tree(1, 1 << 20)
+    t.finalize()
+    with pytest.raises(nu.NorthupError) as e:
+        t.alloc(2 << 20, hbm[0])
+    assert e.value.code == nu.NU_ENOMEM
+    t.destroy()
