@@ -69,6 +69,8 @@ struct Params {
   int tiles_m, tiles_n;
   int vec_ok;         // C base and ldc allow 16-byte vector access
   int npass;          // 3 = 3xTF32 (product path), 1 = plain TF32 (negative test)
+  int b_kmajor;       // debug: B given as N x K (K-major) instead of K x N
+  float* dbg;         // debug: dump of stage 0 after the split (NULL in production)
 };
 
 // ---------------------------------------------------------------- PTX helpers
@@ -142,21 +144,27 @@ __device__ __forceinline__ void tc_fence_after() {
 }
 
 // UMMA shared-memory matrix descriptor (sm_100): start>>4 [0,14), LBO>>4
-// [16,30), SBO>>4 [32,46), version=1 [46,48), layout [61,64) (2 = SWIZZLE_128B).
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+// [16,30), SBO>>4 [32,46), version=1 [46,48), layout [61,64):
+//   2 = SWIZZLE_128B (K-major A: 16-B granules XOR row%8),
+//   1 = SWIZZLE_128B_BASE32B (MN-major 32-bit B: 32-B granules XOR row%4 —
+//       the only MN-major smem layout the tensor core accepts for tf32).
+constexpr uint32_t LAYOUT_SW128 = 2;
+constexpr uint32_t LAYOUT_SW128_BASE32B = 1;
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo,
+                                              uint32_t layout = LAYOUT_SW128) {
   uint64_t d = 0;
   d |= static_cast<uint64_t>((saddr >> 4) & 0x3FFFu);
   d |= static_cast<uint64_t>((lbo >> 4) & 0x3FFFu) << 16;
   d |= static_cast<uint64_t>((sbo >> 4) & 0x3FFFu) << 32;
   d |= static_cast<uint64_t>(1) << 46;
-  d |= static_cast<uint64_t>(2) << 61;
+  d |= static_cast<uint64_t>(layout) << 61;
   return d;
 }
 
 // Instruction descriptor, kind::tf32: D f32 [4,6)=1, A tf32 [7,10)=2,
 // B tf32 [10,13)=2, A K-major [15]=0, B MN-major [16]=1, N>>3 [17,23), M>>4 [24,29).
-__host__ __device__ constexpr uint32_t idesc_tf32(int m, int n) {
-  return (1u << 4) | (2u << 7) | (2u << 10) | (0u << 15) | (1u << 16) |
+__host__ __device__ constexpr uint32_t idesc_tf32(int m, int n, uint32_t b_mn_major = 1) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | (0u << 15) | (b_mn_major << 16) |
          (static_cast<uint32_t>(n >> 3) << 17) | (static_cast<uint32_t>(m >> 4) << 24);
 }
 
@@ -263,16 +271,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           const uint32_t sa = smem_u32(smem + s * STAGE_BYTES);
           const uint32_t sb = sa + A_BYTES;
           tma_load_2d(sa, &tmA, full, kb * BK, mb * BM);
+          if (p.b_kmajor) {
+            tma_load_2d(sb, &tmB, full, kb * BK, nb * BN);
+          } else {
 #pragma unroll
-          for (int c = 0; c < BN / B_CHUNK; ++c)
-            tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, nb * BN + c * B_CHUNK, kb * BK);
+            for (int c = 0; c < BN / B_CHUNK; ++c)
+              tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, nb * BN + c * B_CHUNK, kb * BK);
+          }
         }
       }
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------- MMA issuer
     if (lane == 0) {
-      const uint32_t idesc = idesc_tf32(BM, BN);
+      const uint32_t idesc = idesc_tf32(BM, BN, p.b_kmajor ? 0u : 1u);
       uint32_t it = 0, chunk_it = 0;
       for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
         for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
@@ -293,12 +305,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 #pragma unroll
             for (int k = 0; k < BK / UMMA_K; ++k) {
               // A: K-major SW128, advance 32 B per k-step inside the atom row.
-              // B: MN-major SW128, LBO = stride between 32-column chunks,
-              //    SBO = 8-row group stride; advance one 8-row group per k-step.
+              // B: MN-major SW128_BASE32B, LBO = stride between 32-column
+              //    chunks, SBO = stride between 4-row atoms (512 B); a k-step
+              //    (8 rows) advances 1024 B.
               const uint64_t dah = umma_desc(a_hi + k * 32, 16, 1024);
               const uint64_t dal = umma_desc(a_lo + k * 32, 16, 1024);
-              const uint64_t dbh = umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 1024);
-              const uint64_t dbl = umma_desc(b_lo + k * 1024, B_CHUNK_BYTES, 1024);
+              const uint64_t dbh = p.b_kmajor ? umma_desc(b_hi + k * 32, 16, 1024)
+                                              : umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512,
+                                                          LAYOUT_SW128_BASE32B);
+              const uint64_t dbl = p.b_kmajor ? umma_desc(b_lo + k * 32, 16, 1024)
+                                              : umma_desc(b_lo + k * 1024, B_CHUNK_BYTES, 512,
+                                                          LAYOUT_SW128_BASE32B);
               const uint32_t first = (kb == kb0 && k == 0) ? 0u : 1u;
               if (p.npass == 3) {
                 umma_tf32(tmem_d, dal, dbh, idesc, first);   // small terms first
@@ -340,6 +357,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             raw[i] = h;
             lo[i] = l;
           }
+        }
+        if (p.dbg && blockIdx.x == 0 && it == 0) {
+          __syncwarp();
+          asm volatile("bar.sync 1, 128;" ::: "memory");
+          const float* src = reinterpret_cast<const float*>(smem + s * STAGE_BYTES);
+          for (int i = tid; i < STAGE_BYTES / 4; i += XFORM_THREADS) p.dbg[i] = src[i];
         }
         fence_proxy_async_smem();   // generic-proxy writes -> visible to tcgen05 reads
         mbar_arrive(bar_xform + 8 * s);
@@ -433,14 +456,15 @@ static int get_encode() {
 }
 
 static int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t outer,
-                     uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer) {
+                     uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer,
+                     CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   cuuint64_t dims[2] = {inner, outer};
   cuuint64_t strides[1] = {ld_elems * 4};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims,
-                        strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                        CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d): base=%p inner=%llu outer=%llu ld=%llu", (int)r,
@@ -455,9 +479,20 @@ bool leaf_tma_legal(const void* p, int64_t ld) {
   return (reinterpret_cast<uintptr_t>(p) % 16 == 0) && (ld % 4 == 0) && ld > 0;
 }
 
+int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
+                         int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
+                         int npass, int b_kmajor, float* dbg, cudaStream_t stream);
+
 int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                      int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                      int npass, cudaStream_t stream) {
+  return leaf_gemm_launch_dbg(A, lda, B, ldb, C, ldc, M, N, K, accumulate, kc, npass, 0, nullptr,
+                              stream);
+}
+
+int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
+                         int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
+                         int npass, int b_kmajor, float* dbg, cudaStream_t stream) {
   using namespace leaf;
   if (M < 0 || N < 0 || K < 0) return set_error("negative dimension"), NU_EINVAL;
   if (M == 0 || N == 0) return 0;
@@ -470,12 +505,18 @@ int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, f
     return set_error("dimension exceeds int32 TMA coordinates"), NU_EINVAL;
   if (!leaf_tma_legal(A, lda) || !leaf_tma_legal(B, ldb))
     return set_error("leaf operands need 16-B aligned base and ld %% 4 == 0"), NU_EINVAL;
-  if (lda < K || ldb < N || ldc < N) return set_error("leading dimension too small"), NU_EINVAL;
+  if (lda < K || ldb < (b_kmajor ? K : N) || ldc < N)
+    return set_error("leading dimension too small"), NU_EINVAL;
   int rc = get_encode();
   if (rc) return rc;
   CUtensorMap tmA, tmB;
   if ((rc = encode_2d(&tmA, A, K, M, lda, BK, BM))) return rc;
-  if ((rc = encode_2d(&tmB, B, N, K, ldb, B_CHUNK, BK))) return rc;
+  if (b_kmajor) {
+    if ((rc = encode_2d(&tmB, B, K, N, ldb, BK, BN))) return rc;
+  } else {
+    if ((rc = encode_2d(&tmB, B, N, K, ldb, B_CHUNK, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)))
+      return rc;
+  }
 
   if (kc <= 0) kc = K;
   int64_t kbpc = (kc + BK - 1) / BK;
@@ -494,6 +535,8 @@ int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, f
   p.tiles_n = static_cast<int>((N + BN - 1) / BN);
   p.vec_ok = (reinterpret_cast<uintptr_t>(C) % 16 == 0) && (ldc % 4 == 0);
   p.npass = npass == 1 ? 1 : 3;
+  p.b_kmajor = b_kmajor;
+  p.dbg = dbg;
 
   int dev = 0;
   cudaGetDevice(&dev);
@@ -521,3 +564,12 @@ int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, f
 }
 
 }  // namespace nu
+
+// Debug entry (not part of northup.h): B K-major variant and a stage dump.
+extern "C" int northup_debug_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb,
+                                       float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
+                                       int accumulate, int64_t kc, int npass, int b_kmajor,
+                                       float* dbg, void* stream) {
+  return nu::leaf_gemm_launch_dbg(A, lda, B, ldb, C, ldc, M, N, K, accumulate, kc, npass, b_kmajor,
+                                  dbg, static_cast<cudaStream_t>(stream));
+}
