@@ -1,0 +1,428 @@
+#!/usr/bin/env python
+"""Benchmark of the Northup out-of-core recursive GEMM on B200 (BASELINE.json
+metric: "out-of-core GEMM TFLOP/s at 1/2/4/8 B200; % slowdown vs in-HBM;
+roofline frac").
+
+One step = one northup_gemm call = one pass of the whole hot path:
+  value : the GEMM with A, B, C already resident in HBM (single-node HBM tree,
+          CS4 — the paper's in-memory baseline);
+  e2e   : the same GEMM through the C ABI from pinned HOST buffers
+          (HOST -> HBM (8 GiB cap) -> SMEM/TMEM), every H2D/D2H inside the
+          timed region — the out-of-core number.  slowdown = t_e2e/t_value - 1.
+
+N = 1 runs BASELINE configs[2] (cfg3: 32768^3, 8 GiB HBM cap).  Under torchrun
+(N > 1) every rank runs its C region of configs[3] (cfg4: 65536 x 65536 x
+32768, pinned-host root) — disjoint C subtrees, no data-path collective.
+
+`--impl reference` times the fp64 CPU oracle (the only reference this paper
+has) on a bounded sample of the same workload, on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+GiB = 1 << 30
+METRIC = "out-of-core GEMM TFLOP/s at 1/2/4/8 B200; % slowdown vs in-HBM; roofline frac"
+CONFIGS = {
+    "cfg1": dict(M=256, N=256, K=256, cap=0, block=(64, 64, 64),
+                 desc="256x256x256 fp32, host DRAM -> 1 GPU leaf, 64x64 blocks"),
+    "cfg2": dict(M=8192, N=8192, K=8192, cap=0, block=None,
+                 desc="8192^3 fp32 (in-HBM reference point)"),
+    "cfg3": dict(M=32768, N=32768, K=32768, cap=8 * GiB, block=None,
+                 desc="32768^3 fp32, pinned host -> HBM (8 GiB cap) -> SMEM/TMEM, 1 GPU"),
+    "cfg4": dict(M=65536, N=65536, K=32768, cap=8 * GiB, block=None,
+                 desc="65536x65536x32768 fp32, pinned-host root (no NVMe on the box), C subtrees over G GPUs"),
+    "cfg5": dict(M=1048576, N=4096, K=4096, cap=8 * GiB, block=None,
+                 desc="tall-skinny 1048576x4096x4096 fp32, A streamed from host"),
+}
+NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25      # B200_PROFILING.md nominal dense ratio
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 9:
+                self.rows.append(parts)
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        def num(x):
+            try:
+                return float(x)
+            except ValueError:
+                return None
+        sm = [num(r[1]) for r in self.rows if num(r[1])]
+        mx = [num(r[2]) for r in self.rows if num(r[2])]
+        pw = [num(r[3]) for r in self.rows if num(r[3])]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if r[5 + i].lower().startswith("active")})
+        loaded = sorted(sm)[len(sm) // 2:] if sm else []
+        return {"sm_mhz": statistics.median(loaded) if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "power_w_max": max(pw) if pw else None,
+                "samples": len(self.rows), "reasons": reasons}
+
+
+# ------------------------------------------------------------------ peaks
+def measured_peaks() -> dict:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"bf16_burst": d["bf16_tflops"], "bf16_sustained": d.get("bf16_tflops_sustained",
+                d["bf16_tflops"]), "hbm_gbs": d["hbm_gbs"], "source": "measured"}
+    return {"bf16_burst": 1590.0, "bf16_sustained": 1400.0, "hbm_gbs": 6650.0, "source": "fallback"}
+
+
+def host_array(ptr: int, rows: int, cols: int):
+    import numpy as np
+    n = rows * cols
+    return np.ctypeslib.as_array((ctypes.c_float * n).from_address(ptr)).reshape(rows, cols)
+
+
+# ------------------------------------------------------------- CPU oracle leg
+def cpu_baseline(cfg: dict, a_host, b_host, c_gpu, budget_s: float) -> dict:
+    """The fp64 oracle timed on a bounded sample (full rows of C) on the host
+    cores; also reports the normwise error of the GPU's C on those rows."""
+    import numpy as np
+    import oracle
+    M, N, K = cfg["M"], cfg["N"], cfg["K"]
+    cores = oracle.threads()
+    rng = np.random.default_rng(12345)
+    rows = np.sort(rng.choice(M, size=min(M, cores), replace=False))
+    t0 = time.perf_counter()
+    ref = oracle.gemm_rows(a_host, b_host, rows)
+    dt = time.perf_counter() - t0
+    done = [(rows, ref)]
+    nrows, elapsed = len(rows), dt
+    # grow the sample up to the time budget (whole multiples of `cores` rows)
+    if dt > 0 and dt < budget_s / 2:
+        reps = max(1, int((budget_s - dt) / dt))
+        more = np.sort(rng.choice(M, size=min(M, reps * cores), replace=False))
+        t0 = time.perf_counter()
+        ref2 = oracle.gemm_rows(a_host, b_host, more)
+        elapsed += time.perf_counter() - t0
+        nrows += len(more)
+        done.append((more, ref2))
+    flops = 2.0 * nrows * N * K
+    out = {"value": flops / elapsed / 1e12, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+           "sample": f"{nrows} full rows of C ({nrows}x{N}x{K} fp64 triple loop), {elapsed:.1f} s",
+           "seconds": elapsed}
+    if c_gpu is not None:
+        cn = oracle.col_norms(b_host)
+        worst = 0.0
+        for rws, rf in done:
+            a_s = np.ascontiguousarray(a_host[rws])
+            e, _ = oracle.normwise_err(np.ascontiguousarray(c_gpu[rws]), rf, oracle.row_norms(a_s), cn)
+            worst = max(worst, e)
+        out["gpu_normwise_err_on_sample"] = worst
+        out["gpu_parity_ok"] = bool(worst <= 1e-5)
+    return out
+
+
+# -------------------------------------------------------------------- ours
+def run_ours(args, rank: int, world: int, local_rank: int):
+    import numpy as np
+    import torch
+    import nugen
+    import paper_conf_ipps_chey19_b200 as nu
+
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    name = args.config or ("cfg3" if world == 1 else "cfg4")
+    cfg = dict(CONFIGS[name])
+    if args.quick:
+        cfg.update(M=cfg["M"] // 4, N=cfg["N"] // 4, K=cfg["K"] // 4, cap=cfg["cap"] // 4)
+    M, N, K = cfg["M"], cfg["N"], cfg["K"]
+    r0, r1, c0, c1 = nu.partition_region(world, M, N, K, rank) if world > 1 else (0, M, 0, N)
+    m, n = r1 - r0, c1 - c0
+    seed = int(name[-1])
+    kc = args.k_chunk
+
+    # --- the out-of-core tree: HOST root -> HBM (cap) -> SMEM/TMEM leaf
+    t, hbm = nu.host_tree(1, cfg["cap"], devices=[local_rank])
+    if cfg["block"]:
+        t.set_block(0, *cfg["block"])
+    t.finalize()
+    tg = time.perf_counter()
+    Ab, Bb, Cb = t.alloc(4 * m * K, 0), t.alloc(4 * K * n, 0), t.alloc(4 * m * n, 0)
+    a = host_array(Ab.ptr, m, K)
+    b = host_array(Bb.ptr, K, n)
+    c = host_array(Cb.ptr, m, n)
+    nugen.fill(m, K, seed, nugen.MAT_A, "uniform", out=a, i0=r0, ncols=K)
+    nugen.fill(K, n, seed, nugen.MAT_B, "uniform", out=b, j0=c0, ncols=N)
+    log(f"[rank {rank}] {name} region {m}x{n}x{K}: inputs generated in pinned host memory "
+        f"in {time.perf_counter() - tg:.1f} s")
+
+    # --- the in-HBM tree (value): same GEMM, operands resident in HBM
+    th = nu.hbm_tree(local_rank)
+    th.finalize()
+    Ad = torch.from_numpy(a).to(dev)
+    Bd = torch.from_numpy(b).to(dev)
+    Cd = torch.empty((m, n), dtype=torch.float32, device=dev)
+    hA = th.wrap_device(0, Ad.data_ptr(), Ad.numel() * 4)
+    hB = th.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4)
+    hC = th.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4)
+    opts = nu.make_opts(k_chunk=kc)
+    stream = torch.cuda.current_stream(dev)
+
+    def barrier():
+        torch.cuda.synchronize(dev)
+        if dist is not None:
+            dist.barrier()
+
+    def timed(fn, steps, warmup):
+        for _ in range(warmup):
+            fn()
+        barrier()
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        evs[0].record(stream)
+        for i in range(steps):
+            fn()
+            evs[i + 1].record(stream)
+        barrier()
+        per = [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
+        total = evs[0].elapsed_time(evs[-1])
+        if dist is not None:
+            x = torch.tensor([total], dtype=torch.float64, device=dev)
+            dist.all_reduce(x, op=dist.ReduceOp.MAX)
+            total = float(x.item())
+        return total, per
+
+    # value: in-HBM (the leaf runs on the current torch stream; one launch/step)
+    def step_hbm():
+        nu.leaf_gemm(Ad, Bd, Cd, k_chunk=kc, stream=stream)
+
+    ooc_stats = {}
+
+    def step_ooc():
+        ooc_stats.update(t.gemm(Ab, Bb, Cb, m, n, K, opts))
+
+    with ClockSampler(local_rank) as clk:
+        t_hbm, per_hbm = timed(step_hbm, args.steps, args.warmup)
+        t_ooc, per_ooc = timed(step_ooc, args.steps, args.warmup)
+    c_hbm = Cd.cpu().numpy()
+    c_ooc = c.copy()
+    bitwise_cross_tier = bool(np.array_equal(c_hbm, c_ooc))
+    # the single-node HBM tree through the C ABI must give the same bits
+    th.gemm(hA, hB, hC, m, n, K, opts)
+    torch.cuda.synchronize(dev)
+    bitwise_tree_vs_leaf = bool(torch.equal(Cd, torch.from_numpy(c_hbm).to(dev)))
+
+    flops_total = 2.0 * M * N * K
+    ms_hbm = t_hbm / args.steps
+    ms_ooc = t_ooc / args.steps
+    value = flops_total / (ms_hbm * 1e-3) / 1e12
+    e2e = flops_total / (ms_ooc * 1e-3) / 1e12
+    peaks = measured_peaks()
+    p_tf32 = peaks["bf16_sustained"] * NOMINAL_TF32_OVER_BF16
+    p_eff = p_tf32 / 3.0
+    leaf_ms = statistics.mean(per_hbm)
+    achieved = 2.0 * m * n * K / (leaf_ms * 1e-3) / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tj = json.load(f)
+        if (tj.get("M"), tj.get("N"), tj.get("K")) == (m, n, K):
+            traffic = tj.get("dram_bytes")
+
+    result = None
+    if rank == 0:
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = cpu_baseline(dict(cfg, M=m, N=n), a, b, c_ooc, args.cpu_budget)
+        result = {
+            "metric": METRIC,
+            "value": round(value, 3),
+            "unit": "TFLOP/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": round(ms_hbm, 3),
+            "higher_is_better": True,
+            "scaling": "strong" if world > 1 else "weak",
+            "vs_baseline": None,
+            "dtype": "f32 (3xTF32 tcgen05, fp32 accumulate)",
+            "data": "synthetic (counter-hash uniform [-1,1) fp32, seed = config index)",
+            "config": {
+                "workload": f"{name}: {cfg['desc']}" + (" [quick: /4 sizes]" if args.quick else ""),
+                "M": M, "N": N, "K": K, "hbm_cap_bytes": cfg["cap"], "k_chunk": kc or 1024,
+                "region_per_gpu": [m, n, K],
+                "parallelism": f"C subtrees {nu.partition(world, M, N)} over {world} GPU(s)" if world > 1 else "1 GPU",
+                "schedule": {1: "S1", 2: "S2"}.get(ooc_stats.get("schedule"), "auto"),
+                "blocks": [ooc_stats.get("bm"), ooc_stats.get("bn"), ooc_stats.get("bk")],
+                "drain_tail_k": ooc_stats.get("tail_k"), "drain_strips": ooc_stats.get("strips"),
+                "hbm_footprint_bytes": ooc_stats.get("hbm_peak_bytes"),
+                "l2": "inputs (>= 4 GiB each) exceed the 126 MB L2; no flush needed",
+            },
+            "e2e": {"value": round(e2e, 3), "unit": "TFLOP/s",
+                    "h2d_bytes_per_step": int(ooc_stats.get("bytes_h2d", 0)),
+                    "d2h_bytes_per_step": int(ooc_stats.get("bytes_d2h", 0)),
+                    "ms_per_step": round(ms_ooc, 3),
+                    "leaf_launches_per_step": int(ooc_stats.get("leaf_launches", 0))},
+            "slowdown_pct_vs_in_hbm": round(100.0 * (ms_ooc / ms_hbm - 1.0), 2),
+            "paper_context": {"avg_ooc_slowdown_pct": 17, "dmm_ooc_gap_pct": 5,
+                              "note": "APU + SSD, OpenCL fp32 (PAPER.md P:10, P:381); context only"},
+            "roofline": {"bound": "tensor", "achieved": round(achieved, 3),
+                         "peak": round(p_eff, 3), "unit": "TFLOP/s",
+                         "frac": round(achieved / p_eff, 4), "traffic": traffic,
+                         "peak_basis": (f"3xTF32 useful ceiling = {peaks['source']} bf16 sustained "
+                                        f"{peaks['bf16_sustained']} TF/s x nominal tf32/bf16 "
+                                        f"{NOMINAL_TF32_OVER_BF16:.3f} / 3 MMAs"),
+                         "tensor_pipe_frac_of_tf32_peak": round(3 * achieved / p_tf32, 4),
+                         "kernel": "nu::leaf::leaf_gemm_kernel", "launch": [m, n, K],
+                         "ms_per_launch": round(leaf_ms, 3)},
+            "gpu_launches": args.steps + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
+            "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise_cross_tier,
+                       "bitwise_tree_vs_leaf": bitwise_tree_vs_leaf},
+            "clocks": clk.summary(),
+        }
+        if cpu is not None:
+            result["cpu_baseline"] = {k: cpu[k] for k in ("value", "unit", "cores", "kind", "sample")}
+            result["parity"]["oracle_normwise_err_rows"] = cpu.get("gpu_normwise_err_on_sample")
+            result["parity"]["oracle_ok"] = cpu.get("gpu_parity_ok")
+    th.destroy()
+    t.destroy()
+    return result
+
+
+# --------------------------------------------------------------- reference
+def run_reference(args):
+    """The fp64 CPU oracle as the reference arm (bounded sample per step)."""
+    import numpy as np
+    import nugen
+    import oracle
+    name = args.config or "cfg3"
+    cfg = dict(CONFIGS[name])
+    if args.quick:
+        cfg.update(M=cfg["M"] // 4, N=cfg["N"] // 4, K=cfg["K"] // 4)
+    M, N, K = cfg["M"], cfg["N"], cfg["K"]
+    seed = int(name[-1])
+    cores = oracle.threads()
+    b = nugen.fill(K, N, seed, nugen.MAT_B)
+    rng = np.random.default_rng(7)
+
+    def step(nrows):
+        rows = np.sort(rng.choice(M, size=nrows, replace=False))
+        a = np.empty((nrows, K), dtype=np.float32)
+        for i, r in enumerate(rows):
+            nugen.fill(1, K, seed, nugen.MAT_A, out=a[i:i + 1], i0=int(r), ncols=K)
+        t0 = time.perf_counter()
+        oracle.gemm(a, b)
+        return time.perf_counter() - t0
+
+    dt = step(cores)
+    nrows = cores * max(1, int(args.ref_step_s / max(dt, 1e-3)))
+    for _ in range(args.warmup):
+        step(cores)
+    times = [step(nrows) for _ in range(args.steps)]
+    total = sum(times)
+    flops = 2.0 * nrows * N * K * args.steps
+    v = flops / total / 1e12
+    return {
+        "impl": "reference", "metric": METRIC, "value": round(v, 6), "unit": "TFLOP/s",
+        "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * total / args.steps, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{name}: {cfg['desc']}", "M": M, "N": N, "K": K},
+        "cpu_baseline": {"value": round(v, 6), "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{nrows} full rows of C per step ({nrows}x{N}x{K})"},
+        "e2e": {"value": round(v, 6), "unit": "TFLOP/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default=None, choices=sorted(CONFIGS))
+    ap.add_argument("--k-chunk", type=int, default=1024)
+    ap.add_argument("--quick", action="store_true", help="sizes / 4 (smoke-testing the bench)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--ref-step-s", type=float, default=5.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("warning: the timing rules ask for >= 3 warm-up steps")
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank == 0:
+            print(json.dumps(run_reference(args)), flush=True)
+        return
+
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    res = run_ours(args, rank, world, local_rank)
+    if rank == 0 and res is not None:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
