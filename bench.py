@@ -300,7 +300,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
             "data": "synthetic (counter-hash uniform [-1,1) fp32, seed = config index)",
             "config": {
                 "workload": f"{name}: {cfg['desc']}" + (" [quick: /4 sizes]" if args.quick else ""),
-                "M": M, "N": N, "K": K, "hbm_cap_bytes": cfg["cap"], "k_chunk": kc or 1024,
+                "M": M, "N": N, "K": K, "hbm_cap_bytes": cfg["cap"], "k_chunk": kc or 2048,
                 "region_per_gpu": [m, n, K],
                 "parallelism": f"C subtrees {nu.partition(world, M, N)} over {world} GPU(s)" if world > 1 else "1 GPU",
                 "schedule": {1: "S1", 2: "S2"}.get(ooc_stats.get("schedule"), "auto"),
@@ -324,7 +324,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                                         f"{peaks['bf16_sustained']} TF/s x nominal tf32/bf16 "
                                         f"{NOMINAL_TF32_OVER_BF16:.3f} / 3 MMAs"),
                          "tensor_pipe_frac_of_tf32_peak": round(3 * achieved / p_tf32, 4),
-                         "kernel": "nu::leaf::leaf_gemm_kernel", "launch": [m, n, K],
+                         "kernel": "nu::leaf::sm2::leaf_gemm_2sm_kernel", "launch": [m, n, K],
                          "ms_per_launch": round(leaf_ms, 3)},
             "gpu_launches": args.steps + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
             "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise_cross_tier,
@@ -393,7 +393,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default=None, choices=sorted(CONFIGS))
-    ap.add_argument("--k-chunk", type=int, default=1024)
+    ap.add_argument("--k-chunk", type=int, default=2048)
     ap.add_argument("--quick", action="store_true", help="sizes / 4 (smoke-testing the bench)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

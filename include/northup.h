@@ -171,7 +171,7 @@ int northup_release(northup_tree_t t, northup_buf_t b);
 typedef struct {
   int schedule;         /* NU_SCHED_AUTO / S1 / S2 */
   int replicate_result; /* 1: after the join, all-gather C to every GPU's HBM (NCCL) */
-  int64_t k_chunk;      /* TMEM accumulation length in K (0 = library default, 1024) */
+  int64_t k_chunk;      /* TMEM accumulation length in K (0 = library default, 2048) */
   int npass;            /* 3 = 3xTF32 (default, 0 means 3); 1 = plain TF32 (tests only) */
   int resident;         /* 1: run the plan with operands already resident (in-HBM timing) */
   int collect_timing;   /* 1: record per-stage CUDA-event timings into the stats */
@@ -212,7 +212,7 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
  * C = A.B (accumulate = 0) or C += A.B (accumulate = 1), row-major, on `stream`
  * (a cudaStream_t, NULL = legacy default) of the CURRENT device. A and B need a
  * 16-byte-aligned base and lda, ldb multiples of 4 (TMA); C any alignment.
- * k_chunk = TMEM accumulation length (0 = 1024); npass 3 = 3xTF32, 1 = TF32.
+ * k_chunk = TMEM accumulation length (0 = 2048); npass 3 = 3xTF32, 1 = TF32.
  * Asynchronous: returns after the launch. */
 int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                       int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t k_chunk,

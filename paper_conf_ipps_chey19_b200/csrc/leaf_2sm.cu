@@ -1,0 +1,412 @@
+// Leaf kernel v1: a CTA pair (thread-block cluster of 2 on one TPC) computes
+// a 256 x 256 tile of C with tcgen05.mma.cta_group::2 (UMMA M = 256).
+//
+// Same contract and arithmetic as v0 (leaf_sm100.cu: 3xTF32, TMEM
+// accumulation per k_chunk, fp32 RN epilogue add), but each CTA stages only
+// its half of the operands: CTA r holds A rows [r*128, r*128+128) and B
+// columns [r*128, r*128+128) of the pair tile.  The leader CTA (rank 0)
+// issues the MMAs, which read both CTAs' shared memory, so each SM's shared
+// memory supplies 8 KiB per k8 step instead of 12 KiB.
+//
+// The tensor core truncates the low 13 mantissa bits of an fp32 operand fed
+// as tf32 (probed on the box: tools/debug_leaf.py, R19), so the raw
+// TMA tile IS the hi operand; the split only writes lo = x - trunc(x).  Raw
+// tiles live in an RS-deep ring, lo tiles in an LS-deep ring.  Per k8 step
+// the three MMAs run as (hi.lo, hi.hi, lo.hi) with the A collector keeping
+// A_hi between the first two (one A read saved).
+//
+// Synchronisation across the pair:
+//   full[s]    (each CTA)  own TMA bytes landed               -> own split warps
+//   rempty[s]  (each CTA)  leader's commit, multicast          -> own TMA producer
+//   xform[j]   (leader)    both CTAs' lo tile written (cnt 2)  -> MMA issuer
+//   lempty[j]  (each CTA)  leader's commit, multicast          -> own split warps
+//   tfull[a]   (each CTA)  leader's commit, multicast          -> own epilogue
+//   tempty[a]  (leader)    both CTAs drained TMEM (count 2)    -> MMA issuer
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "leaf_common.cuh"
+#include "northup_internal.h"
+
+namespace nu {
+namespace leaf {
+namespace sm2 {
+
+constexpr int BM = 256;                            // pair tile rows (UMMA M)
+constexpr int BN = 256;                            // pair tile cols (UMMA N)
+constexpr int BM_CTA = 128;                        // rows of A per CTA
+constexpr int BN_CTA = 128;                        // cols of B per CTA
+constexpr int RS = 4;                              // raw (TMA) ring depth
+constexpr int LS = 2;                              // lo (split) ring depth
+constexpr int A_BYTES = BM_CTA * BK * 4;           // 16 KiB
+constexpr int B_BYTES = BN_CTA * BK * 4;           // 16 KiB
+constexpr int TMA_BYTES = A_BYTES + B_BYTES;       // per CTA per stage
+constexpr int STAGE_BYTES = TMA_BYTES;             // one raw or one lo stage
+constexpr int NUM_THREADS = 320;
+constexpr int XFORM_THREADS = 128;
+constexpr int EPI_THREADS = 128;
+constexpr int TMEM_COLS = 512;                     // 2 accumulators x 256 columns
+constexpr int BAR_BYTES = 1024;
+constexpr int SMEM_BYTES = (RS + LS) * STAGE_BYTES + BAR_BYTES + 1024;
+static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+
+__device__ __forceinline__ uint32_t mapa(uint32_t saddr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+
+// Arrive on a barrier of another CTA of the cluster (address from mapa).
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "r"(a));
+  return v;
+}
+
+__device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+
+// Wait with cluster-scope acquire (the phase may be completed by the peer CTA).
+__device__ __forceinline__ void mbar_wait_cluster(uint32_t bar, uint32_t parity) {
+  uint32_t done = 0;
+  uint64_t t0 = 0;
+  for (uint32_t it = 0;; ++it) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    if (done) return;
+    if ((it & 1023u) == 0) {
+      const uint64_t t = globaltimer();
+      if (it == 0) t0 = t;
+      else if (t - t0 > 4000000000ull) __trap();
+    }
+  }
+}
+
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+
+__device__ __forceinline__ void named_bar(uint32_t id, uint32_t count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void umma_tf32_2sm(uint32_t tmem_d, uint64_t da, uint64_t db,
+                                              uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+__device__ __forceinline__ void umma_tf32_2sm_afill(uint32_t tmem_d, uint64_t da, uint64_t db,
+                                                    uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32.collector::a::fill [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+__device__ __forceinline__ void umma_tf32_2sm_alast(uint32_t tmem_d, uint64_t da, uint64_t db,
+                                                    uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32.collector::a::lastuse [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+// Arrive on the same barrier offset in both CTAs of the pair once the MMAs
+// issued so far have completed.
+__device__ __forceinline__ void umma_commit_pair(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
+      " [%0], %1;" ::"r"(bar),
+      "h"(static_cast<uint16_t>(3))
+      : "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
+    leaf_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tmA,
+                         const __grid_constant__ CUtensorMap tmB, const Params p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint8_t* raw_base = smem;                          // RS raw stages
+  uint8_t* lo_base = smem + RS * STAGE_BYTES;         // LS lo stages
+  uint8_t* bars = smem + (RS + LS) * STAGE_BYTES;
+  const uint32_t bar_full = smem_u32(bars);
+  const uint32_t bar_rempty = bar_full + 8 * RS;
+  const uint32_t bar_xform = bar_rempty + 8 * RS;
+  const uint32_t bar_lempty = bar_xform + 8 * LS;
+  const uint32_t bar_tfull = bar_lempty + 8 * LS;
+  const uint32_t bar_tempty = bar_tfull + 16;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (2 * RS + 2 * LS + 4));
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+
+  if (threadIdx.x == 0) {
+    prefetch_tmap(&tmA);
+    prefetch_tmap(&tmB);
+    for (int s = 0; s < RS; ++s) {
+      mbar_init(bar_full + 8 * s, 1);
+      mbar_init(bar_rempty + 8 * s, 1);
+    }
+    for (int j = 0; j < LS; ++j) {
+      mbar_init(bar_xform + 8 * j, 2 * XFORM_THREADS);
+      mbar_init(bar_lempty + 8 * j, 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(bar_tfull + 8 * a, 1);
+      mbar_init(bar_tempty + 8 * a, 2 * EPI_THREADS);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  const int cid = blockIdx.x >> 1;
+  const int nclusters = gridDim.x >> 1;
+  const int num_tiles = p.tiles_m * p.tiles_n;
+  const int nkb = (p.K + BK - 1) / BK;
+  const int nchunks = (nkb + p.kb_per_chunk - 1) / p.kb_per_chunk;
+
+  if (warp == 0) {
+    // ------------------------------------------------------ TMA producer (own half)
+    if (lane == 0) {
+      uint32_t it = 0;
+      for (int t = cid; t < num_tiles; t += nclusters) {
+        int mb, nb;
+        tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
+        const int row0 = mb * BM + rank * BM_CTA;
+        const int col0 = nb * BN + rank * BN_CTA;
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const uint32_t s = it % RS, use = it / RS;
+          mbar_wait(bar_rempty + 8 * s, (use & 1) ^ 1);
+          const uint32_t full = bar_full + 8 * s;
+          mbar_arrive_expect_tx(full, TMA_BYTES);
+          const uint32_t sa = smem_u32(raw_base + s * STAGE_BYTES);
+          const uint32_t sb = sa + A_BYTES;
+          tma_load_2d(sa, &tmA, full, kb * BK, row0);
+#pragma unroll
+          for (int c = 0; c < BN_CTA / B_CHUNK; ++c)
+            tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------ MMA issuer (leader CTA only)
+    if (leader && lane == 0) {
+      const uint32_t idesc = idesc_tf32(BM, BN, 1u);
+      uint32_t it = 0, chunk_it = 0;
+      for (int t = cid; t < num_tiles; t += nclusters) {
+        for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
+          const uint32_t acc = chunk_it & 1, ause = chunk_it >> 1;
+          mbar_wait_cluster(bar_tempty + 8 * acc, (ause & 1) ^ 1);
+          tc_fence_after();
+          const uint32_t tmem_d = tmem_base + acc * BN;
+          const int kb0 = ch * p.kb_per_chunk;
+          const int kb1 = min(nkb, kb0 + p.kb_per_chunk);
+          for (int kb = kb0; kb < kb1; ++kb, ++it) {
+            const uint32_t s = it % RS;
+            const uint32_t j = it % LS, juse = it / LS;
+            mbar_wait_cluster(bar_xform + 8 * j, juse & 1);
+            tc_fence_after();
+            const uint32_t a_hi = smem_u32(raw_base + s * STAGE_BYTES);
+            const uint32_t b_hi = a_hi + A_BYTES;
+            const uint32_t a_lo = smem_u32(lo_base + j * STAGE_BYTES);
+            const uint32_t b_lo = a_lo + A_BYTES;
+#pragma unroll
+            for (int k = 0; k < BK / UMMA_K; ++k) {
+              const uint64_t dah = umma_desc(a_hi + k * 32, 16, 1024);
+              const uint64_t dal = umma_desc(a_lo + k * 32, 16, 1024);
+              const uint64_t dbh = umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
+              const uint64_t dbl = umma_desc(b_lo + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
+              const uint32_t first = (kb == kb0 && k == 0) ? 0u : 1u;
+              if (p.npass == 3) {
+                umma_tf32_2sm_afill(tmem_d, dah, dbl, idesc, first);
+                umma_tf32_2sm_alast(tmem_d, dah, dbh, idesc, 1u);
+                umma_tf32_2sm(tmem_d, dal, dbh, idesc, 1u);
+              } else {
+                umma_tf32_2sm(tmem_d, dah, dbh, idesc, first);
+              }
+            }
+            umma_commit_pair(bar_rempty + 8 * s);
+            umma_commit_pair(bar_lempty + 8 * j);
+          }
+          umma_commit_pair(bar_tfull + 8 * acc);
+        }
+      }
+    }
+  } else if (warp < 6) {
+    // ---------------------------------------------------- transform (own half)
+    const int tid = threadIdx.x - 64;
+    const uint32_t xform_leader0 = mapa(bar_xform, 0);
+    uint32_t it = 0;
+    for (int t = cid; t < num_tiles; t += nclusters) {
+      for (int kb = 0; kb < nkb; ++kb, ++it) {
+        const uint32_t s = it % RS, use = it / RS;
+        const uint32_t j = it % LS, juse = it / LS;
+        mbar_wait(bar_full + 8 * s, use & 1);
+        mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
+        const uint32_t raw = smem_u32(raw_base + s * STAGE_BYTES);
+        const uint32_t lo = smem_u32(lo_base + j * STAGE_BYTES);
+        if (p.npass == 3) {
+          uint4 x[TMA_BYTES / 16 / XFORM_THREADS];
+#pragma unroll
+          for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u)
+            x[u] = lds128(raw + (tid + u * XFORM_THREADS) * 16);
+#pragma unroll
+          for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u) {
+            uint4 l;   // lo = x - trunc13(x): exact in fp32
+            l.x = __float_as_uint(__uint_as_float(x[u].x) - __uint_as_float(x[u].x & 0xFFFFE000u));
+            l.y = __float_as_uint(__uint_as_float(x[u].y) - __uint_as_float(x[u].y & 0xFFFFE000u));
+            l.z = __float_as_uint(__uint_as_float(x[u].z) - __uint_as_float(x[u].z & 0xFFFFE000u));
+            l.w = __float_as_uint(__uint_as_float(x[u].w) - __uint_as_float(x[u].w & 0xFFFFE000u));
+            sts128(lo + (tid + u * XFORM_THREADS) * 16, l);
+          }
+        }
+        fence_proxy_async_smem();   // generic st.shared -> visible to the tensor core
+        mbar_arrive_cluster(xform_leader0 + 8 * j);
+      }
+    }
+  } else {
+    // ------------------------------------------------------ epilogue (own rows)
+    const int q = warp & 3;
+    const int row_in_tile = rank * BM_CTA + q * 32 + lane;
+    const uint32_t tempty_leader0 = mapa(bar_tempty, 0);
+    uint32_t chunk_it = 0;
+    for (int t = cid; t < num_tiles; t += nclusters) {
+      int mb, nb;
+      tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
+      const int row = mb * BM + row_in_tile;
+      const bool row_ok = row < p.M;
+      float* crow = p.C + static_cast<int64_t>(row) * p.ldc;
+      for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
+        const uint32_t acc = chunk_it & 1, ause = chunk_it >> 1;
+        mbar_wait(bar_tfull + 8 * acc, ause & 1);
+        tc_fence_after();
+        const bool add = (ch > 0) || p.accumulate;
+#pragma unroll 1
+        for (int c = 0; c < BN / 32; ++c) {
+          uint32_t v[32];
+          __syncwarp();
+          tmem_ld32(tmem_base + (static_cast<uint32_t>(q * 32) << 16) + acc * BN + c * 32, v);
+          const int col0 = nb * BN + c * 32;
+          if (row_ok && col0 < p.N) {
+            float* dst = crow + col0;
+            if (p.vec_ok && col0 + 32 <= p.N) {
+#pragma unroll
+              for (int j = 0; j < 32; j += 4) {
+                float4 o = make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]),
+                                       __uint_as_float(v[j + 2]), __uint_as_float(v[j + 3]));
+                if (add) {
+                  const float4 c4 = *reinterpret_cast<const float4*>(dst + j);
+                  o.x = c4.x + o.x;
+                  o.y = c4.y + o.y;
+                  o.z = c4.z + o.z;
+                  o.w = c4.w + o.w;
+                }
+                *reinterpret_cast<float4*>(dst + j) = o;
+              }
+            } else {
+              const int ncol = min(32, p.N - col0);
+#pragma unroll
+              for (int j = 0; j < 32; ++j) {
+                if (j < ncol) {
+                  float o = __uint_as_float(v[j]);
+                  if (add) o = dst[j] + o;
+                  dst[j] = o;
+                }
+              }
+            }
+          }
+        }
+        __syncwarp();
+        tc_fence_before();
+        mbar_arrive_cluster(tempty_leader0 + 8 * acc);
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "n"(TMEM_COLS)
+                 : "memory");
+  }
+}
+
+}  // namespace sm2
+
+int launch_sm2(LaunchArgs& a) {
+  using namespace sm2;
+  int rc;
+  CUtensorMap tmA, tmB;
+  Params& p = a.p;
+  if (p.b_kmajor || p.dbg) return fail(NU_ENOTSUP, "debug options are 1sm-only");
+  if ((rc = encode_2d(&tmA, a.A, p.K, p.M, a.lda, BK, BM_CTA))) return rc;
+  if ((rc = encode_2d(&tmB, a.B, p.N, p.K, a.ldb, B_CHUNK, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)))
+    return rc;
+  p.tiles_m = (p.M + BM - 1) / BM;
+  p.tiles_n = (p.N + BN - 1) / BN;
+  static std::atomic<int> configured[kMaxDevices];
+  if (!configured[a.dev].load()) {
+    cudaError_t e = cudaFuncSetAttribute(leaf_gemm_2sm_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    if (e != cudaSuccess) return fail(NU_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+    configured[a.dev].store(1);
+  }
+  const int tiles = p.tiles_m * p.tiles_n;
+  const int pairs = a.sms / 2;
+  const int grid = 2 * (tiles < pairs ? tiles : pairs);
+  leaf_gemm_2sm_kernel<<<grid, NUM_THREADS, SMEM_BYTES, a.stream>>>(tmA, tmB, p);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : fail(NU_ECUDA, "leaf (2sm) launch: %s", cudaGetErrorString(e));
+}
+
+}  // namespace leaf
+}  // namespace nu

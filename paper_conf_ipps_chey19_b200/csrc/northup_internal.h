@@ -12,8 +12,10 @@
 namespace nu {
 
 constexpr int kMaxDevices = 64;
-constexpr int64_t kDefaultKChunk = 1024;   // TMEM accumulation length
+constexpr int64_t kDefaultKChunk = 2048;   // TMEM accumulation length (R20)
 constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
+constexpr int kRasterBand = 16;            // n-blocks per raster band in the leaf
+constexpr int64_t kPanelChunks = 1;        // leaf K-panel launches, in k_chunks (0 = one launch)
 
 // Thread-local error message (northup_last_error).  Returns its argument so
 // call sites can write `return fail(NU_EINVAL, "...")`.
@@ -106,6 +108,9 @@ bool leaf_tma_legal(const void* p, int64_t ld);
 int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                      int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                      int npass, cudaStream_t stream);
+int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
+                         int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
+                         int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream);
 
 // --------------------------------------------------------------- executor
 int execute_plan(northup_tree_s* t, const Plan& plan, void* a, void* b, void* c,

@@ -248,7 +248,7 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
 }
 
 int build_s2(const EdgeCtx& x, northup_stats* st) {
-  S2Shape s;
+  S2Shape s{};
   int rc = choose_s2(x, &s);
   if (rc) return rc;
   Builder& B = *x.B;
