@@ -15,7 +15,7 @@ import os
 import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libnorthup.so")
+LIB_PATH = os.environ.get("NORTHUP_LIB_PATH") or os.path.join(_HERE, "libnorthup.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "northup.h")
 
 # status codes / enums (include/northup.h)

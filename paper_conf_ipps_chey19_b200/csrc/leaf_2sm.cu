@@ -39,17 +39,28 @@ constexpr int BM = 256;                            // pair tile rows (UMMA M)
 constexpr int BN = 256;                            // pair tile cols (UMMA N)
 constexpr int BM_CTA = 128;                        // rows of A per CTA
 constexpr int BN_CTA = 128;                        // cols of B per CTA
-constexpr int RS = 4;                              // raw (TMA) ring depth
-constexpr int LS = 2;                              // lo (split) ring depth
+#ifndef NU_LEAF_RS
+#define NU_LEAF_RS 4
+#endif
+#ifndef NU_LEAF_LS
+#define NU_LEAF_LS 3
+#endif
+constexpr int RS = NU_LEAF_RS;                     // raw (TMA) ring depth
+constexpr int LS = NU_LEAF_LS;                     // lo (split) ring depth
 constexpr int A_BYTES = BM_CTA * BK * 4;           // 16 KiB
 constexpr int B_BYTES = BN_CTA * BK * 4;           // 16 KiB
 constexpr int TMA_BYTES = A_BYTES + B_BYTES;       // per CTA per stage
 constexpr int STAGE_BYTES = TMA_BYTES;             // one raw or one lo stage
-constexpr int NUM_THREADS = 320;
-constexpr int XFORM_THREADS = 128;
+#ifndef NU_LEAF_XFORM_WARPS
+#define NU_LEAF_XFORM_WARPS 4
+#endif
+constexpr int XFORM_WARPS = NU_LEAF_XFORM_WARPS;   // split warps (2 .. 2+XFORM_WARPS-1)
+constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
+constexpr int EPI_WARP0 = 2 + XFORM_WARPS;         // 4 epilogue warps follow
 constexpr int EPI_THREADS = 128;
+constexpr int NUM_THREADS = 32 * (EPI_WARP0 + 4);
 constexpr int TMEM_COLS = 512;                     // 2 accumulators x 256 columns
-constexpr int BAR_BYTES = 1024;
+constexpr int BAR_BYTES = 256;
 constexpr int SMEM_BYTES = (RS + LS) * STAGE_BYTES + BAR_BYTES + 1024;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 
@@ -184,7 +195,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       mbar_init(bar_rempty + 8 * s, 1);
     }
     for (int j = 0; j < LS; ++j) {
-      mbar_init(bar_xform + 8 * j, 2 * XFORM_THREADS);
+      mbar_init(bar_xform + 8 * j, 2);   // one elected arrive per CTA
       mbar_init(bar_lempty + 8 * j, 1);
     }
     for (int a = 0; a < 2; ++a) {
@@ -239,10 +250,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     if (leader && lane == 0) {
       const uint32_t idesc = idesc_tf32(BM, BN, 1u);
       uint32_t it = 0, chunk_it = 0;
+      long long w_xf = 0, w_te = 0, t_beg = clock64();   // profile mode (p.dbg)
       for (int t = cid; t < num_tiles; t += nclusters) {
         for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
           const uint32_t acc = chunk_it & 1, ause = chunk_it >> 1;
+          long long c0 = clock64();
           mbar_wait_cluster(bar_tempty + 8 * acc, (ause & 1) ^ 1);
+          w_te += clock64() - c0;
           tc_fence_after();
           const uint32_t tmem_d = tmem_base + acc * BN;
           const int kb0 = ch * p.kb_per_chunk;
@@ -250,7 +264,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           for (int kb = kb0; kb < kb1; ++kb, ++it) {
             const uint32_t s = it % RS;
             const uint32_t j = it % LS, juse = it / LS;
-            mbar_wait_cluster(bar_xform + 8 * j, juse & 1);
+            c0 = clock64();
+            if (!(p.b_kmajor & 1)) mbar_wait_cluster(bar_xform + 8 * j, juse & 1);   // exp. 1: no wait
+            w_xf += clock64() - c0;
             tc_fence_after();
             const uint32_t a_hi = smem_u32(raw_base + s * STAGE_BYTES);
             const uint32_t b_hi = a_hi + A_BYTES;
@@ -277,21 +293,33 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           umma_commit_pair(bar_tfull + 8 * acc);
         }
       }
+      if (p.dbg) {
+        float* d = p.dbg + 8 * cid;
+        d[0] = static_cast<float>(clock64() - t_beg);
+        d[1] = static_cast<float>(w_xf);
+        d[2] = static_cast<float>(w_te);
+        d[3] = static_cast<float>(it);
+      }
     }
-  } else if (warp < 6) {
+  } else if (warp < EPI_WARP0) {
     // ---------------------------------------------------- transform (own half)
     const int tid = threadIdx.x - 64;
     const uint32_t xform_leader0 = mapa(bar_xform, 0);
     uint32_t it = 0;
+    long long w_full = 0, w_lem = 0;
     for (int t = cid; t < num_tiles; t += nclusters) {
       for (int kb = 0; kb < nkb; ++kb, ++it) {
         const uint32_t s = it % RS, use = it / RS;
         const uint32_t j = it % LS, juse = it / LS;
+        long long c0 = clock64();
         mbar_wait(bar_full + 8 * s, use & 1);
+        long long c1 = clock64();
         mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
+        w_full += c1 - c0;
+        w_lem += clock64() - c1;
         const uint32_t raw = smem_u32(raw_base + s * STAGE_BYTES);
         const uint32_t lo = smem_u32(lo_base + j * STAGE_BYTES);
-        if (p.npass == 3) {
+        if (p.npass == 3 && !(p.b_kmajor & 2)) {   // exp. 2: skip the split work
           uint4 x[TMA_BYTES / 16 / XFORM_THREADS];
 #pragma unroll
           for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u)
@@ -307,8 +335,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           }
         }
         fence_proxy_async_smem();   // generic st.shared -> visible to the tensor core
-        mbar_arrive_cluster(xform_leader0 + 8 * j);
+        named_bar(1, XFORM_THREADS);
+        if (tid == 0) mbar_arrive_cluster(xform_leader0 + 8 * j);
       }
+    }
+    if (p.dbg && tid == 0) {
+      float* d = p.dbg + 8 * cid + 4 + 2 * rank;
+      d[0] = static_cast<float>(w_full);
+      d[1] = static_cast<float>(w_lem);
     }
   } else {
     // ------------------------------------------------------ epilogue (own rows)
@@ -387,7 +421,7 @@ int launch_sm2(LaunchArgs& a) {
   int rc;
   CUtensorMap tmA, tmB;
   Params& p = a.p;
-  if (p.b_kmajor || p.dbg) return fail(NU_ENOTSUP, "debug options are 1sm-only");
+  // (2sm: b_kmajor is reused as an experiment bit field by tools/mma_prof.py)
   if ((rc = encode_2d(&tmA, a.A, p.K, p.M, a.lda, BK, BM_CTA))) return rc;
   if ((rc = encode_2d(&tmB, a.B, p.N, p.K, a.ldb, B_CHUNK, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)))
     return rc;
@@ -410,3 +444,70 @@ int launch_sm2(LaunchArgs& a) {
 
 }  // namespace leaf
 }  // namespace nu
+
+// --------------------------------------------------------------------------
+// Debug: raw tensor-core rate of the 2-CTA tf32 MMA (M=256, N=256, K=8) on
+// fixed shared-memory operands, no pipeline — calibrates the 128-clk model.
+namespace nu {
+namespace leaf {
+namespace sm2 {
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1)
+    mma_rate_kernel(int n_mma, int mode, long long* out) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  __shared__ uint64_t bar;
+  __shared__ uint32_t slot;
+  const int warp = threadIdx.x >> 5;
+  const uint32_t rank = cluster_ctarank();
+  for (int i = threadIdx.x; i < 65536 / 4; i += blockDim.x) reinterpret_cast<float*>(smem)[i] = 0.f;
+  if (threadIdx.x == 0) {
+    mbar_init(smem_u32(&bar), 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&slot)), "n"(256) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem = slot;
+  if (rank == 0 && threadIdx.x == 0) {
+    const uint32_t idesc = idesc_tf32(256, 256, 1u);
+    const uint32_t a = smem_u32(smem), b = a + 16384, a2 = a + 32768, b2 = a + 49152;
+    long long t0 = clock64();
+    for (int i = 0; i < n_mma; ++i) {
+      const uint64_t da = umma_desc((mode & 1) && (i % 3 == 2) ? a2 : a, 16, 1024);
+      const uint64_t db = umma_desc((mode & 2) && (i % 3 == 0) ? b2 : b, B_CHUNK_BYTES, 512,
+                                    LAYOUT_SW128_BASE32B);
+      umma_tf32_2sm(tmem, da, db, idesc, i > 0);
+    }
+    umma_commit_pair(smem_u32(&bar));
+    mbar_wait(smem_u32(&bar), 0);
+    out[0] = clock64() - t0;
+  } else if (rank == 1 && threadIdx.x == 0) {
+    mbar_wait(smem_u32(&bar), 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(256)
+                 : "memory");
+  }
+}
+}  // namespace sm2
+}  // namespace leaf
+}  // namespace nu
+
+extern "C" int northup_debug_mma_rate(int n_mma, int mode, int grid, long long* out_dev) {
+  cudaFuncSetAttribute(nu::leaf::sm2::mma_rate_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       70 * 1024);
+  nu::leaf::sm2::mma_rate_kernel<<<grid, 128, 70 * 1024>>>(n_mma, mode, out_dev);
+  cudaError_t e = cudaDeviceSynchronize();
+  return e == cudaSuccess ? 0 : nu::fail(NU_ECUDA, "mma_rate: %s", cudaGetErrorString(e));
+}
