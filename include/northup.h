@@ -175,7 +175,9 @@ typedef struct {
   int npass;            /* 3 = 3xTF32 (default, 0 means 3); 1 = plain TF32 (tests only) */
   int resident;         /* 1: run the plan with operands already resident (in-HBM timing) */
   int collect_timing;   /* 1: record per-stage CUDA-event timings into the stats */
-  int reserved[8];
+  int64_t a_panel_k;    /* FILE root only: A is stored K-panel-major (R15 preprocessing,
+                           see northup_file_tile_kpanels) with this panel width; 0 = row-major */
+  int reserved[6];
 } northup_gemm_opts;
 
 typedef struct {
@@ -225,6 +227,8 @@ int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, 
 #define NU_OP_COPY 0
 #define NU_OP_LEAF 1
 #define NU_OP_ZERO 2
+#define NU_OP_IO_READ 3  /* file -> DRAM staging (pread), host I/O thread */
+#define NU_OP_IO_WRITE 4 /* DRAM staging -> file (pwrite), host I/O thread */
 typedef struct {
   int op;
   int worker;   /* GPU worker index (0 .. num_gpus-1) */
@@ -235,7 +239,7 @@ typedef struct {
   int64_t src_off, dst_off, src_ld, dst_ld, rows, cols; /* COPY, element units */
   int64_t a_off, b_off, c_off, lda, ldb, ldc, m, n, k;  /* LEAF, element units */
   int ndeps;
-  int deps[8];  /* indices of earlier ops this op must wait for (pruned per stream) */
+  int deps[16]; /* indices of earlier ops this op must wait for (pruned per worker and stream) */
 } northup_op;
 
 typedef struct {
@@ -258,6 +262,16 @@ int northup_plan_get_buf(northup_plan_t p, int i, northup_plan_buf* out);
 /* Same statistics the executor reports, predicted from the plan (bytes, blocks). */
 int northup_plan_stats(northup_plan_t p, northup_stats* out);
 int northup_plan_destroy(northup_plan_t p);
+
+/* ------------------------------------------- file-root preprocessing (R15) */
+/* P:353 "preprocessing the original file and reorganizing it ... for chunking":
+ * rewrite a row-major M x K fp32 matrix file `src` as K-panel-major `dst`
+ * (panel p = columns [p*panel_k, (p+1)*panel_k), row-major inside, panels
+ * stored one after another; the last panel may be narrower), so that each
+ * K panel of A is one sequential read.  Host-only; a one-time cost reported
+ * separately from the GEMM (reading R15). */
+int northup_file_tile_kpanels(const char* src, const char* dst, int64_t M, int64_t K,
+                              int64_t panel_k);
 
 /* -------------------------------------------------------- partitioner */
 /* The 2-D grid Pr x Pc = G that minimises per-GPU H2D bytes 4K(M/Pr + N/Pc),

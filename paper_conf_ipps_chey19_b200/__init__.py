@@ -23,7 +23,7 @@ NU_OK, NU_EINVAL, NU_ENOMEM, NU_EIO, NU_ECUDA, NU_ENCCL, NU_ESTATE, NU_ENOTSUP =
 NU_FILE, NU_HOST, NU_HBM, NU_SMEM = 0, 1, 2, 3
 NU_PROC_NONE, NU_PROC_SM100 = 0, 1
 NU_SCHED_AUTO, NU_SCHED_S1, NU_SCHED_S2 = 0, 1, 2
-NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO = 0, 1, 2
+NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO, NU_OP_IO_READ, NU_OP_IO_WRITE = 0, 1, 2, 3, 4
 STREAM_NAMES = {0: "h2d", 1: "compute", 2: "d2h", 3: "io", 4: "d2d"}
 STATUS_NAMES = {0: "NU_OK", -1: "NU_EINVAL", -2: "NU_ENOMEM", -3: "NU_EIO", -4: "NU_ECUDA",
                 -5: "NU_ENCCL", -6: "NU_ESTATE", -7: "NU_ENOTSUP"}
@@ -48,7 +48,8 @@ class NodeInfo(ctypes.Structure):
 class GemmOpts(ctypes.Structure):
     _fields_ = [("schedule", ctypes.c_int), ("replicate_result", ctypes.c_int),
                 ("k_chunk", ctypes.c_int64), ("npass", ctypes.c_int), ("resident", ctypes.c_int),
-                ("collect_timing", ctypes.c_int), ("reserved", ctypes.c_int * 8)]
+                ("collect_timing", ctypes.c_int), ("a_panel_k", ctypes.c_int64),
+                ("reserved", ctypes.c_int * 6)]
 
 
 class Stats(ctypes.Structure):
@@ -76,7 +77,7 @@ class Op(ctypes.Structure):
                 ("cols", ctypes.c_int64), ("a_off", ctypes.c_int64), ("b_off", ctypes.c_int64),
                 ("c_off", ctypes.c_int64), ("lda", ctypes.c_int64), ("ldb", ctypes.c_int64),
                 ("ldc", ctypes.c_int64), ("m", ctypes.c_int64), ("n", ctypes.c_int64),
-                ("k", ctypes.c_int64), ("ndeps", ctypes.c_int), ("deps", ctypes.c_int * 8)]
+                ("k", ctypes.c_int64), ("ndeps", ctypes.c_int), ("deps", ctypes.c_int * 16)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "deps"}
@@ -135,6 +136,7 @@ _SIGS = {
     "northup_partition": [_int, _i64, _i64, _i64, _pint, _pint],
     "northup_partition_region": [_int, _i64, _i64, _i64, _int, ctypes.POINTER(_i64),
                                  ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i64)],
+    "northup_file_tile_kpanels": [ctypes.c_char_p, ctypes.c_char_p, _i64, _i64, _i64],
     "northup_version": [],
     "northup_device_count": [],
 }
@@ -216,6 +218,11 @@ def leaf_gemm(A, B, C, accumulate: bool = False, k_chunk: int = 0, npass: int = 
                       npass, stream)
 
 
+def file_tile_kpanels(src: str, dst: str, M: int, K: int, panel_k: int) -> None:
+    """R15 preprocessing: row-major A file -> K-panel-major file."""
+    check(lib().northup_file_tile_kpanels(src.encode(), dst.encode(), M, K, panel_k))
+
+
 def partition(G: int, M: int, N: int, K: int = 0) -> tuple[int, int]:
     pr, pc = ctypes.c_int(), ctypes.c_int()
     check(lib().northup_partition(G, M, N, K, ctypes.byref(pr), ctypes.byref(pc)))
@@ -229,8 +236,10 @@ def partition_region(G: int, M: int, N: int, K: int, r: int) -> tuple[int, int, 
 
 
 def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 3,
-              collect_timing: bool = False, replicate_result: bool = False) -> GemmOpts:
+              collect_timing: bool = False, replicate_result: bool = False,
+              a_panel_k: int = 0) -> GemmOpts:
     o = GemmOpts()
+    o.a_panel_k = a_panel_k
     o.schedule = schedule
     o.k_chunk = k_chunk
     o.npass = npass

@@ -1,6 +1,11 @@
 // C ABI entry points for the GEMM, the leaf, plan introspection and the
 // partitioner (include/northup.h).
+#include <errno.h>
+#include <stdio.h>
 #include <string.h>
+
+#include <algorithm>
+#include <vector>
 
 #include <chrono>
 
@@ -68,8 +73,9 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
   *st = northup_stats{};
   if (M == 0 || N == 0) return 0;
   if (K == 0) return zero_root_c(t, C, M, N);
-  if (t->nodes[0].storage == NU_FILE)
-    return fail(NU_ENOTSUP, "FILE roots are not supported by northup_gemm in this version");
+  if (t->nodes[0].storage == NU_FILE &&
+      (A->storage != NU_FILE || B->storage != NU_FILE || C->storage != NU_FILE))
+    return fail(NU_EINVAL, "a FILE root needs A, B and C as files (northup_open_file / alloc)");
 
   t->busy = true;
   Plan plan;
@@ -82,7 +88,7 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
     st->t_plan_ms = t1 - t0;
     int prev = 0;
     cudaGetDevice(&prev);
-    rc = execute_plan(t, plan, A->ptr, B->ptr, C->ptr, o, st);
+    rc = execute_plan(t, plan, A, B, C, o, st);
     cudaSetDevice(prev);
   }
   t->busy = false;
@@ -143,6 +149,46 @@ int northup_plan_stats(northup_plan_t p, northup_stats* out) {
 int northup_plan_destroy(northup_plan_t p) {
   delete p;
   return 0;
+}
+
+// ------------------------------------------- file preprocessing (R15)
+int northup_file_tile_kpanels(const char* src, const char* dst, int64_t M, int64_t K,
+                              int64_t panel_k) {
+  if (!src || !dst || M < 0 || K < 0 || panel_k <= 0) return fail(NU_EINVAL, "bad arguments");
+  FILE* in = fopen(src, "rb");
+  if (!in) return fail(NU_EIO, "open %s: %s", src, strerror(errno));
+  FILE* out = fopen(dst, "wb");
+  if (!out) {
+    fclose(in);
+    return fail(NU_EIO, "open %s: %s", dst, strerror(errno));
+  }
+  // Stream row blocks of A; scatter each row's panel pieces to their panels.
+  const int64_t rows_per = std::max<int64_t>(1, (256ll << 20) / std::max<int64_t>(1, K * 4));
+  std::vector<float> buf(static_cast<size_t>(rows_per * K));
+  int rc = 0;
+  for (int64_t r0 = 0; r0 < M && !rc; r0 += rows_per) {
+    const int64_t nr = std::min(rows_per, M - r0);
+    if (fread(buf.data(), 4, static_cast<size_t>(nr * K), in) != static_cast<size_t>(nr * K)) {
+      rc = fail(NU_EIO, "short read from %s", src);
+      break;
+    }
+    for (int64_t k0 = 0; k0 < K && !rc; k0 += panel_k) {
+      const int64_t w = std::min(panel_k, K - k0);
+      // panel p starts at element k0 * M; row r of the panel at + r * w
+      if (fseeko(out, static_cast<off_t>((k0 * M + r0 * w) * 4), SEEK_SET) != 0) {
+        rc = fail(NU_EIO, "seek %s: %s", dst, strerror(errno));
+        break;
+      }
+      for (int64_t r = 0; r < nr; ++r)
+        if (fwrite(buf.data() + r * K + k0, 4, static_cast<size_t>(w), out) != static_cast<size_t>(w)) {
+          rc = fail(NU_EIO, "write %s: %s", dst, strerror(errno));
+          break;
+        }
+    }
+  }
+  fclose(in);
+  if (fclose(out) != 0 && !rc) rc = fail(NU_EIO, "close %s: %s", dst, strerror(errno));
+  return rc;
 }
 
 // --------------------------------------------------------- partitioner

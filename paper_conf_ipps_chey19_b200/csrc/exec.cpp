@@ -7,7 +7,22 @@
 // another stream becomes a cudaStreamWaitEvent, so transfers of later
 // chunks overlap the computation of earlier ones ("overlapping computation
 // and communications (i.e. OpenCL/CUDA streams) at the leaf node").
+//
+// A FILE root adds a host I/O thread (file <-> DRAM staging, Listing 4):
+//   CUDA op waiting for an I/O op  -> the worker thread blocks before issuing it
+//   I/O op waiting for a CUDA op   -> the I/O thread waits until the op has been
+//                                     issued, then cudaEventSynchronize.
+// All dependencies point backwards in plan order, which every thread follows,
+// so the waits cannot deadlock.
+#include <errno.h>
+#include <fcntl.h>
+#include <string.h>
+#include <unistd.h>
+
+#include <atomic>
 #include <chrono>
+#include <condition_variable>
+#include <mutex>
 #include <thread>
 
 #include "northup_internal.h"
@@ -72,18 +87,33 @@ static int ensure_arena(northup_tree_s* t, int node, uint64_t bytes) {
     return fail(NU_ENOMEM, "node %d: plan needs %llu B, capacity %llu B (%llu in use)", node,
                 (unsigned long long)bytes, (unsigned long long)n.capacity,
                 (unsigned long long)other);
-  cudaSetDevice(n.phys);
-  if (n.arena) {
-    cudaFree(n.arena);
-    n.used -= n.arena_bytes;
-    n.arena = nullptr;
-    n.arena_bytes = 0;
-  }
-  cudaError_t e = cudaMalloc(&n.arena, bytes);
-  if (e != cudaSuccess) {
-    n.arena = nullptr;
-    return fail(NU_ENOMEM, "cudaMalloc(%llu) for node %d arena: %s", (unsigned long long)bytes, node,
-                cudaGetErrorString(e));
+  if (n.storage == NU_HOST) {
+    if (n.arena) {
+      cudaFreeHost(n.arena);
+      n.used -= n.arena_bytes;
+      n.arena = nullptr;
+      n.arena_bytes = 0;
+    }
+    cudaError_t e = cudaHostAlloc(&n.arena, bytes, cudaHostAllocPortable);
+    if (e != cudaSuccess) {
+      n.arena = nullptr;
+      return fail(NU_ENOMEM, "cudaHostAlloc(%llu) for staging node %d: %s", (unsigned long long)bytes,
+                  node, cudaGetErrorString(e));
+    }
+  } else {
+    cudaSetDevice(n.phys);
+    if (n.arena) {
+      cudaFree(n.arena);
+      n.used -= n.arena_bytes;
+      n.arena = nullptr;
+      n.arena_bytes = 0;
+    }
+    cudaError_t e = cudaMalloc(&n.arena, bytes);
+    if (e != cudaSuccess) {
+      n.arena = nullptr;
+      return fail(NU_ENOMEM, "cudaMalloc(%llu) for node %d arena: %s", (unsigned long long)bytes,
+                  node, cudaGetErrorString(e));
+    }
   }
   n.arena_bytes = bytes;
   n.arena_owned = true;
@@ -94,11 +124,34 @@ static int ensure_arena(northup_tree_s* t, int node, uint64_t bytes) {
 struct RunCtx {
   northup_tree_s* t;
   const Plan* plan;
-  std::vector<char*> base;             // per plan buffer
+  std::vector<char*> base;             // per plan buffer (host/device pointers)
+  std::vector<const northup_buf_s*> file;   // per plan buffer: file handle or NULL
   const std::vector<char>* needs_event;
   const northup_gemm_opts* o;
   bool timing;
+  // cross-thread progress (FILE roots)
+  std::mutex m;
+  std::condition_variable cv;
+  std::vector<char> issued;            // CUDA op: event recorded
+  std::vector<char> io_done;           // I/O op: finished
+  std::atomic<bool> abort{false};
+  double io_ms = 0;
 };
+
+static void mark(RunCtx& c, std::vector<char>& v, size_t i) {
+  {
+    std::lock_guard<std::mutex> g(c.m);
+    v[i] = 1;
+  }
+  c.cv.notify_all();
+}
+
+// Wait until flag i is set (or the run aborted).  Returns false on abort.
+static bool wait_flag(RunCtx& c, std::vector<char>& v, size_t i) {
+  std::unique_lock<std::mutex> g(c.m);
+  c.cv.wait(g, [&] { return v[i] || c.abort.load(); });
+  return v[i] != 0;
+}
 
 static int run_worker(RunCtx& c, int wi, double* busy) {
   const Plan& P = *c.plan;
@@ -126,6 +179,11 @@ static int run_worker(RunCtx& c, int wi, double* busy) {
     if (op.worker != wi) continue;
     cudaStream_t s = w->streams[op.stream];
     for (int d = 0; d < op.ndeps; ++d) {
+      const northup_op& q = P.ops[op.deps[d]];
+      if (q.stream == S_IO) {
+        if (!wait_flag(c, c.io_done, op.deps[d])) return fail(NU_EIO, "aborted: file I/O failed");
+        continue;
+      }
       e = cudaStreamWaitEvent(s, w->events[op.deps[d]], 0);
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent");
     }
@@ -155,6 +213,7 @@ static int run_worker(RunCtx& c, int wi, double* busy) {
     if ((*c.needs_event)[i]) {
       e = cudaEventRecord(w->events[i], s);
       if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+      mark(c, c.issued, i);
     }
   }
   for (cudaStream_t s : w->streams) {
@@ -173,59 +232,142 @@ static int run_worker(RunCtx& c, int wi, double* busy) {
   return 0;
 }
 
-int execute_plan(northup_tree_s* t, const Plan& P, void* a, void* b, void* c,
-                 const northup_gemm_opts* o, northup_stats* st) {
+// Positional file I/O of a rows x cols fp32 block (element offsets / leading
+// dimensions); O_DIRECT when the file has a direct descriptor and
+// buffer, offset and length are 4 KiB aligned, else buffered I/O.
+static int file_block(const northup_buf_s* f, bool write, char* mem, int64_t mem_ld,
+                      int64_t file_off, int64_t file_ld, int64_t rows, int64_t cols) {
+  auto io = [&](char* p, uint64_t bytes, uint64_t off) -> int {
+    int fd = f->fd;
+    if (f->direct_fd >= 0 && reinterpret_cast<uintptr_t>(p) % 4096 == 0 && bytes % 4096 == 0 &&
+        off % 4096 == 0)
+      fd = f->direct_fd;
+    while (bytes) {
+      ssize_t r = write ? pwrite(fd, p, bytes, static_cast<off_t>(off))
+                        : pread(fd, p, bytes, static_cast<off_t>(off));
+      if (r < 0) {
+        if (errno == EINTR) continue;
+        return fail(NU_EIO, "%s(%s): %s", write ? "pwrite" : "pread", f->path.c_str(), strerror(errno));
+      }
+      if (r == 0) return fail(NU_EIO, "%s(%s): short transfer", write ? "pwrite" : "pread", f->path.c_str());
+      p += r;
+      bytes -= static_cast<uint64_t>(r);
+      off += static_cast<uint64_t>(r);
+    }
+    return 0;
+  };
+  if (mem_ld == cols && file_ld == cols)
+    return io(mem, static_cast<uint64_t>(rows * cols) * 4, static_cast<uint64_t>(file_off) * 4);
+  for (int64_t r = 0; r < rows; ++r) {
+    int rc = io(mem + r * mem_ld * 4, static_cast<uint64_t>(cols) * 4,
+                static_cast<uint64_t>(file_off + r * file_ld) * 4);
+    if (rc) return rc;
+  }
+  return 0;
+}
+
+static int run_io(RunCtx& c) {
+  const Plan& P = *c.plan;
+  const auto t0 = std::chrono::steady_clock::now();
+  for (size_t i = 0; i < P.ops.size(); ++i) {
+    const northup_op& op = P.ops[i];
+    if (op.stream != S_IO) continue;
+    for (int d = 0; d < op.ndeps; ++d) {
+      const northup_op& q = P.ops[op.deps[d]];
+      if (q.stream == S_IO) continue;
+      if (!wait_flag(c, c.issued, op.deps[d])) return fail(NU_ECUDA, "aborted: a GPU worker failed");
+      WorkerState* w = worker_for_node(c.t, P.worker_node[q.worker]);
+      cudaSetDevice(w->device);
+      cudaError_t e = cudaEventSynchronize(w->events[op.deps[d]]);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize (I/O thread)");
+    }
+    int rc;
+    if (op.op == NU_OP_IO_READ)
+      rc = file_block(c.file[op.src_buf], false, c.base[op.dst_buf] + op.dst_off * 4, op.dst_ld,
+                      op.src_off, op.src_ld, op.rows, op.cols);
+    else
+      rc = file_block(c.file[op.dst_buf], true, c.base[op.src_buf] + op.src_off * 4, op.src_ld,
+                      op.dst_off, op.dst_ld, op.rows, op.cols);
+    if (rc) return rc;
+    mark(c, c.io_done, i);
+  }
+  // O_SYNC semantics of P:242: C is durable when northup_gemm returns.
+  for (size_t b = 0; b < c.file.size(); ++b)
+    if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0)
+      return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(errno));
+  c.io_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return 0;
+}
+
+int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf_s* b,
+                 northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st) {
   RunCtx ctx;
   ctx.t = t;
   ctx.plan = &P;
   ctx.o = o;
   ctx.timing = o && o->collect_timing;
   ctx.base.resize(P.bufs.size(), nullptr);
+  ctx.file.resize(P.bufs.size(), nullptr);
   for (size_t i = 0; i < P.bufs.size(); ++i) {
     const PlanBuf& pb = P.bufs[i];
-    switch (pb.kind) {
-      case B_USER_A: ctx.base[i] = static_cast<char*>(a); break;
-      case B_USER_B: ctx.base[i] = static_cast<char*>(b); break;
-      case B_USER_C: ctx.base[i] = static_cast<char*>(c); break;
-      default: {
-        int rc = ensure_arena(t, pb.node, pb.bytes);
-        if (rc) return rc;
-        ctx.base[i] = static_cast<char*>(t->nodes[pb.node].arena);
-      }
+    northup_buf_s* ub = pb.kind == B_USER_A ? a : pb.kind == B_USER_B ? b : pb.kind == B_USER_C ? c : nullptr;
+    if (ub) {
+      ctx.base[i] = static_cast<char*>(ub->ptr);
+      if (ub->storage == NU_FILE) ctx.file[i] = ub;
+      continue;
     }
+    int rc = ensure_arena(t, pb.node, pb.bytes);
+    if (rc) return rc;
+    ctx.base[i] = static_cast<char*>(t->nodes[pb.node].arena);
   }
   // Only record an event where some later op on another stream waits for it.
   std::vector<char> needs(P.ops.size(), 0);
-  for (const northup_op& op : P.ops)
+  bool has_io = false;
+  for (const northup_op& op : P.ops) {
     for (int d = 0; d < op.ndeps; ++d) needs[op.deps[d]] = 1;
+    has_io |= op.stream == S_IO;
+  }
   ctx.needs_event = &needs;
+  ctx.issued.assign(P.ops.size(), 0);
+  ctx.io_done.assign(P.ops.size(), 0);
 
   const int W = P.num_workers;
-  std::vector<int> rcs(W, 0);
+  std::vector<int> rcs(W + 1, 0);
+  std::vector<std::string> errs(W + 1);
   std::vector<std::vector<double>> busy(W, std::vector<double>(S_NUM, 0.0));
-  std::string first_err;
-  if (W == 1) {
-    rcs[0] = run_worker(ctx, 0, busy[0].data());
-    if (rcs[0]) first_err = northup_last_error();
+  auto worker_body = [&](int wi) {
+    rcs[wi] = run_worker(ctx, wi, busy[wi].data());
+    if (rcs[wi]) {
+      errs[wi] = northup_last_error();
+      ctx.abort = true;
+      ctx.cv.notify_all();
+    }
+  };
+  auto io_body = [&] {
+    rcs[W] = run_io(ctx);
+    if (rcs[W]) {
+      errs[W] = northup_last_error();
+      ctx.abort = true;
+      ctx.cv.notify_all();
+    }
+  };
+  if (W == 1 && !has_io) {
+    worker_body(0);
   } else {
     std::vector<std::thread> th;
-    std::vector<std::string> errs(W);
-    for (int wi = 0; wi < W; ++wi)
-      th.emplace_back([&, wi] {
-        rcs[wi] = run_worker(ctx, wi, busy[wi].data());
-        if (rcs[wi]) errs[wi] = northup_last_error();
-      });
+    for (int wi = 0; wi < W; ++wi) th.emplace_back(worker_body, wi);
+    if (has_io) th.emplace_back(io_body);
     for (auto& x : th) x.join();
-    for (int wi = 0; wi < W; ++wi)
-      if (rcs[wi] && first_err.empty()) first_err = errs[wi];
   }
-  for (int wi = 0; wi < W; ++wi) {
-    if (rcs[wi]) return fail(rcs[wi], "worker %d: %s", wi, first_err.c_str());
-    if (st) {
+  for (int wi = 0; wi <= W; ++wi)
+    if (rcs[wi]) return fail(rcs[wi], "%s %d: %s", wi < W ? "worker" : "I/O thread", wi, errs[wi].c_str());
+  if (st) {
+    for (int wi = 0; wi < W; ++wi) {
       st->t_h2d_ms += busy[wi][S_H2D];
       st->t_compute_ms += busy[wi][S_COMP];
       st->t_d2h_ms += busy[wi][S_D2H] + busy[wi][S_D2D];
     }
+    st->t_io_ms = ctx.io_ms;
   }
   return 0;
 }

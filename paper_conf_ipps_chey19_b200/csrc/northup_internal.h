@@ -49,6 +49,7 @@ struct northup_buf_s {
   int storage = NU_HOST;
   void* ptr = nullptr;       // host / device pointer (NULL for files)
   int fd = -1;               // file descriptor (NU_FILE)
+  int direct_fd = -1;        // O_DIRECT descriptor when the file system allows it
   uint64_t bytes = 0;
   bool owned = false;        // library allocated (freed on release/destroy)
   bool registered = false;   // cudaHostRegister'ed by us (wrap_host)
@@ -71,7 +72,7 @@ namespace nu {
 
 // --------------------------------------------------------------- plan
 enum Stream { S_H2D = 0, S_COMP = 1, S_D2H = 2, S_IO = 3, S_D2D = 4, S_NUM = 5 };
-enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3 };
+enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3, B_DRAM = 4 };
 
 struct PlanBuf {
   int kind = B_ARENA;
@@ -90,6 +91,7 @@ struct Plan {
   int64_t kc = kDefaultKChunk;
   int npass = 3;
   bool root_is_device = false;
+  bool file_root = false;
 };
 
 int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
@@ -113,8 +115,8 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
                          int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream);
 
 // --------------------------------------------------------------- executor
-int execute_plan(northup_tree_s* t, const Plan& plan, void* a, void* b, void* c,
-                 const northup_gemm_opts* o, northup_stats* st);
+int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,
+                 northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
 int finalize_workers(northup_tree_s* t);
 void destroy_workers(northup_tree_s* t);
 

@@ -103,26 +103,44 @@ struct Builder {
 
   void emit(northup_op op, std::initializer_list<Acc> accs) {
     const int idx = static_cast<int>(P->ops.size());
-    int last[S_NUM];
-    for (int& x : last) x = -1;
+    // latest conflicting op per (worker, stream); ops on the op's own
+    // (worker, stream) queue are ordered already.
+    std::vector<std::pair<int, int>> last;   // (key, op)
     for (const Acc& a : accs) {
       if (a.rows <= 0 || a.cols <= 0) continue;
       const int64_t lo = a.off, hi = a.off + (a.rows - 1) * a.ld + a.cols;
+      const bool user = P->bufs[a.buf].kind != B_ARENA && P->bufs[a.buf].kind != B_DRAM;
       auto& h = hist[a.buf];
       for (const Access& p : h) {
         if (p.hi <= lo || hi <= p.lo) continue;
         if (!a.write && !p.write) continue;
-        if (p.stream == op.stream) continue;   // same stream: ordered already
-        if (P->ops[p.op].worker != op.worker) continue;   // sibling regions are disjoint
-        last[p.stream] = std::max(last[p.stream], p.op);
+        const northup_op& q = P->ops[p.op];
+        if (q.worker == op.worker && q.stream == op.stream) continue;
+        // root-tier regions of different siblings are disjoint by construction
+        // (their 2-D bounding intervals may still overlap)
+        if (user && q.worker != op.worker && q.stream != S_IO && op.stream != S_IO) continue;
+        const int key = q.worker * S_NUM + q.stream;
+        bool found = false;
+        for (auto& kv : last)
+          if (kv.first == key) {
+            kv.second = std::max(kv.second, p.op);
+            found = true;
+          }
+        if (!found) last.emplace_back(key, p.op);
       }
       h.push_back(Access{idx, op.stream, lo, hi, a.write});
     }
     op.ndeps = 0;
-    for (int s = 0; s < S_NUM; ++s)
-      if (last[s] >= 0) op.deps[op.ndeps++] = last[s];
+    for (auto& kv : last) {
+      if (op.ndeps >= 16) {
+        overflow = true;
+        break;
+      }
+      op.deps[op.ndeps++] = kv.second;
+    }
     P->ops.push_back(op);
   }
+  bool overflow = false;
 };
 
 northup_op make_copy(int worker, int stream, int src, int64_t src_off, int64_t src_ld, int dst,
@@ -460,6 +478,135 @@ int build_in_hbm(Builder& B, int node, int64_t M, int64_t N, int64_t K, int A, i
   return 0;
 }
 
+
+// FILE root (S§8(a) a3): FILE -> HOST staging -> G x HBM -> SMEM/TMEM.
+// K panels of A and B are read from the files into a ring of DRAM staging
+// slots shared by all siblings (each file byte is read once per C-block round),
+// every sibling copies its rows / columns of the panel to its HBM slots and
+// accumulates into its resident C block; finished C blocks drain HBM -> DRAM
+// strip by strip and are written back to the C file (Listing 4 file_write).
+northup_op make_io(int io_worker, int op, int src, int64_t src_off, int64_t src_ld, int dst,
+                   int64_t dst_off, int64_t dst_ld, int64_t rows, int64_t cols) {
+  northup_op o = make_copy(io_worker, S_IO, src, src_off, src_ld, dst, dst_off, dst_ld, rows, cols);
+  o.op = op;
+  return o;
+}
+
+int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std::vector<int>& hbm,
+                    int64_t M, int64_t N, int64_t K, int A, int Bb, int C, int64_t kc,
+                    int64_t a_panel_k, northup_stats* st) {
+  const int G = static_cast<int>(hbm.size());
+  const int io = G;   // the I/O pseudo-worker
+  const int64_t bk = a_panel_k > 0 ? a_panel_k : kc;
+  // per-worker regions and one common C-block shape that fits every HBM node
+  std::vector<int64_t> r0(G), r1(G), c0(G), c1(G);
+  int64_t mmax = 0, nmax = 0;
+  uint64_t cap = uint64_t(1) << 62;
+  for (int w = 0; w < G; ++w) {
+    int rc = region_of(G, M, N, w, &r0[w], &r1[w], &c0[w], &c1[w]);
+    if (rc) return rc;
+    mmax = std::max(mmax, r1[w] - r0[w]);
+    nmax = std::max(nmax, c1[w] - c0[w]);
+    if (t->nodes[hbm[w]].capacity) cap = std::min<uint64_t>(cap, t->nodes[hbm[w]].capacity);
+  }
+  auto hbm_bytes = [&](int64_t bm, int64_t bn) {
+    return 4ull * (uint64_t(bm) * pad_ld(bn) +
+                   uint64_t(kSlots) * (uint64_t(bm) * pad_ld(bk) + uint64_t(bk) * pad_ld(bn)));
+  };
+  int64_t bm = mmax, bn = nmax;
+  while (hbm_bytes(bm, bn) > cap) {
+    if (bm > 128) bm = rup(cdiv(bm, 2), 128);
+    else if (bn > 256) bn = rup(cdiv(bn, 2), 256);
+    else return fail(NU_ENOMEM, "HBM capacity %llu B below the minimum block", (unsigned long long)cap);
+  }
+  const int64_t nbr = cdiv(mmax, bm), nbc = cdiv(nmax, bn), rounds = nbr * nbc;
+  const int64_t sr = std::min<int64_t>(bm, rup(cdiv(bm, 8), 128));   // drain strip rows
+  // DRAM staging: R panel slots (A panel M x bk, B panel bk x N) + 2 C strips per GPU
+  const uint64_t dcap = t->nodes[staging].capacity ? t->nodes[staging].capacity : uint64_t(1) << 62;
+  const uint64_t panel_e = uint64_t(M) * bk + uint64_t(bk) * N;
+  const uint64_t cstage_e = uint64_t(G) * 2 * sr * bn;
+  int R = kSlots;
+  while (R > 1 && 4ull * (R * panel_e + cstage_e) > dcap) --R;
+  if (4ull * (R * panel_e + cstage_e) > dcap)
+    return fail(NU_ENOMEM, "staging node %d capacity %llu B below one panel + C strips", staging,
+                (unsigned long long)dcap);
+  const int dram = B.add_buf(B_DRAM, staging, -1, 4ull * (R * panel_e + cstage_e));
+  std::vector<int> arena(G);
+  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+  const int64_t ldC = pad_ld(bn), ldA = pad_ld(bk), ldB = pad_ld(bn);
+  const int64_t offC = 0;
+  int64_t offSA[kSlots], offSB[kSlots];
+  for (int i = 0, off = 0; i < kSlots; ++i) {
+    offSA[i] = offC + bm * ldC + i * (bm * ldA + bk * ldB);
+    offSB[i] = offSA[i] + bm * ldA;
+    (void)off;
+  }
+  auto slotA = [&](int s) { return int64_t(s) * int64_t(panel_e); };
+  auto slotB = [&](int s) { return int64_t(s) * int64_t(panel_e) + M * bk; };
+  auto cst = [&](int w, int j) { return int64_t(R) * int64_t(panel_e) + (int64_t(w) * 2 + j) * sr * bn; };
+  st->bm = bm;
+  st->bn = bn;
+  st->bk = bk;
+  st->hbm_peak_bytes = hbm_bytes(bm, bn);
+  st->schedule = NU_SCHED_S2;
+  const int64_t npan = cdiv(K, bk);
+  int64_t gp = 0;               // global panel counter (DRAM ring)
+  std::vector<int64_t> hslot(G, 0), cstrip(G, 0);
+  for (int64_t r = 0; r < rounds; ++r) {
+    const int64_t bi = r / nbc, bj = r % nbc;
+    for (int64_t p = 0; p < npan; ++p, ++gp) {
+      const int s = static_cast<int>(gp % R);
+      const int64_t k0 = p * bk, kk = std::min(bk, K - k0);
+      // file -> DRAM: one sequential read per panel when A is K-panel-major
+      if (a_panel_k > 0)
+        B.emit(make_io(io, NU_OP_IO_READ, A, k0 * M, kk, dram, slotA(s), kk, M, kk),
+               {{A, k0 * M, kk, M, kk, false}, {dram, slotA(s), kk, M, kk, true}});
+      else
+        B.emit(make_io(io, NU_OP_IO_READ, A, k0, K, dram, slotA(s), kk, M, kk),
+               {{A, k0, K, M, kk, false}, {dram, slotA(s), kk, M, kk, true}});
+      B.emit(make_io(io, NU_OP_IO_READ, Bb, k0 * N, N, dram, slotB(s), N, kk, N),
+             {{Bb, k0 * N, N, kk, N, false}, {dram, slotB(s), N, kk, N, true}});
+      st->bytes_file_read += 4ull * (uint64_t(M) * kk + uint64_t(kk) * N);
+      for (int w = 0; w < G; ++w) {
+        const int64_t i0 = bi * bm, j0 = bj * bn;
+        const int64_t m = std::min(bm, (r1[w] - r0[w]) - i0), n = std::min(bn, (c1[w] - c0[w]) - j0);
+        if (m <= 0 || n <= 0) continue;
+        const int64_t gr = r0[w] + i0, gc = c0[w] + j0;
+        const int sl = static_cast<int>(hslot[w]++ % kSlots);
+        B.emit(make_copy(w, S_H2D, dram, slotA(s) + gr * kk, kk, arena[w], offSA[sl], ldA, m, kk),
+               {{dram, slotA(s) + gr * kk, kk, m, kk, false}, {arena[w], offSA[sl], ldA, m, kk, true}});
+        B.emit(make_copy(w, S_H2D, dram, slotB(s) + gc, N, arena[w], offSB[sl], ldB, kk, n),
+               {{dram, slotB(s) + gc, N, kk, n, false}, {arena[w], offSB[sl], ldB, kk, n, true}});
+        st->bytes_h2d += 4ull * (uint64_t(m) * kk + uint64_t(kk) * n);
+        B.emit(make_leaf(w, arena[w], offSA[sl], ldA, arena[w], offSB[sl], ldB, arena[w], offC, ldC,
+                         m, n, kk, p > 0 ? 1 : 0),
+               {{arena[w], offSA[sl], ldA, m, kk, false},
+                {arena[w], offSB[sl], ldB, kk, n, false},
+                {arena[w], offC, ldC, m, n, true}});
+        st->leaf_launches++;
+      }
+    }
+    // drain: HBM -> DRAM strips -> C file (Listing 4: file_write)
+    for (int w = 0; w < G; ++w) {
+      const int64_t i0 = bi * bm, j0 = bj * bn;
+      const int64_t m = std::min(bm, (r1[w] - r0[w]) - i0), n = std::min(bn, (c1[w] - c0[w]) - j0);
+      if (m <= 0 || n <= 0) continue;
+      const int64_t gr = r0[w] + i0, gc = c0[w] + j0;
+      for (int64_t q = 0; q < m; q += sr) {
+        const int64_t rr = std::min(sr, m - q);
+        const int j = static_cast<int>(cstrip[w]++ % 2);
+        B.emit(make_copy(w, S_D2H, arena[w], offC + q * ldC, ldC, dram, cst(w, j), n, rr, n),
+               {{arena[w], offC + q * ldC, ldC, rr, n, false}, {dram, cst(w, j), n, rr, n, true}});
+        st->bytes_d2h += 4ull * rr * n;
+        B.emit(make_io(io, NU_OP_IO_WRITE, dram, cst(w, j), n, C, (gr + q) * N + gc, N, rr, n),
+               {{dram, cst(w, j), n, rr, n, false}, {C, (gr + q) * N + gc, N, rr, n, true}});
+        st->bytes_file_write += 4ull * rr * n;
+      }
+    }
+  }
+  return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
+}
+
 }  // namespace
 
 // Which HBM nodes compute, and what sits above them.
@@ -506,8 +653,29 @@ int build_plan_ex(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
     st.ops = static_cast<int64_t>(P.ops.size());
     return rc;
   }
-  if (root.storage == NU_FILE)
-    return fail(NU_ENOTSUP, "FILE roots are planned by the staging engine (northup_gemm_file)");
+  if (root.storage == NU_FILE) {
+    // FILE -> HOST (DRAM staging) -> HBM siblings
+    if (root.children.size() != 1 || t->nodes[root.children[0]].storage != NU_HOST)
+      return fail(NU_ENOTSUP, "a FILE root needs exactly one HOST staging child (no GDS edge)");
+    const int staging = root.children[0];
+    std::vector<int> hbm;
+    for (int c : t->nodes[staging].children) {
+      if (t->nodes[c].storage != NU_HBM)
+        return fail(NU_ENOTSUP, "staging node children must be HBM nodes (node %d is not)", c);
+      hbm.push_back(c);
+    }
+    if (hbm.empty()) return fail(NU_EINVAL, "staging node has no HBM child");
+    P.num_workers = static_cast<int>(hbm.size());
+    P.worker_node = hbm;
+    st.num_gpus = P.num_workers;
+    P.file_root = true;
+    if (M == 0 || N == 0 || K == 0) return 0;
+    rc = build_file_root(B, t, staging, hbm, M, N, K, A, Bb, C, P.kc, o ? o->a_panel_k : 0, &st);
+    st.ops = static_cast<int64_t>(P.ops.size());
+    for (const northup_op& op : P.ops)
+      if (op.op == NU_OP_COPY || op.op == NU_OP_IO_READ || op.op == NU_OP_IO_WRITE) st.copies++;
+    return rc;
+  }
   if (root.storage != NU_HOST) return fail(NU_EINVAL, "root must be FILE, HOST or HBM");
 
   // HOST root: its children must be the HBM siblings (branch parallelism).

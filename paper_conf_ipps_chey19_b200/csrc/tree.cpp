@@ -179,8 +179,12 @@ int northup_tree_destroy(northup_tree_t t) {
   destroy_workers(t);
   for (Node& n : t->nodes) {
     if (n.arena_owned && n.arena) {
-      cudaSetDevice(n.phys);
-      cudaFree(n.arena);
+      if (n.storage == NU_HOST) {
+        cudaFreeHost(n.arena);
+      } else {
+        cudaSetDevice(n.phys);
+        cudaFree(n.arena);
+      }
     }
     n.arena = nullptr;
   }
@@ -369,6 +373,7 @@ int northup_alloc(northup_tree_t t, uint64_t bytes, int node, northup_buf_t* out
       return fail(NU_EIO, "ftruncate(%s): %s", path, strerror(err));
     }
     b->fd = fd;
+    b->direct_fd = open(path, O_RDWR | O_DIRECT);
     b->path = path;
   } else {
     delete b;
@@ -459,6 +464,7 @@ int northup_open_file(northup_tree_t t, int node, const char* path, uint64_t byt
     }
   }
   b->fd = fd;
+  b->direct_fd = open(path, O_RDWR | O_DIRECT);   // -1 where O_DIRECT is unsupported (tmpfs)
   b->bytes = bytes;
   b->path = path;
   t->bufs.push_back(b);
@@ -578,6 +584,7 @@ int northup_release(northup_tree_t t, northup_buf_t b) {
     }
     if (b->storage == NU_FILE) {
       if (b->fd >= 0) close(b->fd);
+      if (b->direct_fd >= 0) close(b->direct_fd);
       if (!b->path.empty()) unlink(b->path.c_str());
       b->fd = -1;
     }
@@ -585,6 +592,7 @@ int northup_release(northup_tree_t t, northup_buf_t b) {
   } else {
     if (b->registered && b->ptr) cudaHostUnregister(b->ptr);
     if (b->storage == NU_FILE && b->fd >= 0) close(b->fd);
+    if (b->storage == NU_FILE && b->direct_fd >= 0) close(b->direct_fd);
   }
   delete b;
   return 0;

@@ -86,7 +86,13 @@ def test_partition_grid(G, M, N, grid):
 
 
 # ------------------------------------------------------------ plan simulator
-def simulate(plan: nu.Plan, A, B, M, N, K, rng=None):
+def kpanels(A, P):
+    """A (M x K) in the K-panel-major file layout of northup_file_tile_kpanels."""
+    M, K = A.shape
+    return np.concatenate([A[:, k0:k0 + P].ravel() for k0 in range(0, K, P)]) if K else A.ravel()
+
+
+def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
     """Replay the plan's ops on host arrays (float64, exact on integers).
     With `rng`, ops run in a random order consistent with the dependencies
     and with in-order execution per (worker, stream)."""
@@ -95,7 +101,7 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None):
     mem = []
     for b in bufs:
         if b["kind"] == 0:
-            mem.append(A.astype(np.float64).ravel().copy())
+            mem.append((a_layout if a_layout is not None else A.ravel()).astype(np.float64).copy())
         elif b["kind"] == 1:
             mem.append(B.astype(np.float64).ravel().copy())
         elif b["kind"] == 2:
@@ -108,7 +114,7 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None):
                                                strides=(ld * 8, 8), writeable=True)
 
     def run(op):
-        if op["op"] == nu.NU_OP_COPY:
+        if op["op"] in (nu.NU_OP_COPY, nu.NU_OP_IO_READ, nu.NU_OP_IO_WRITE):
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
                 view(op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
         elif op["op"] == nu.NU_OP_LEAF:
@@ -226,3 +232,46 @@ def test_data_api_host_only_errors():
     with pytest.raises(nu.NorthupError):
         t.alloc(64, 2)     # SMEM node: managed by the leaf kernel
     t.destroy()
+
+
+def file_tree(G, cap=0, staging_cap=0):
+    t = nu.Tree()
+    root = t.add_node(-1, nu.NU_FILE)
+    st = t.add_node(root, nu.NU_HOST, -1, staging_cap)
+    for g in range(G):
+        h = t.add_node(st, nu.NU_HBM, 0, cap)
+        t.add_node(h, nu.NU_SMEM, 0, 227 * 1024, nu.NU_PROC_SM100)
+    return t
+
+
+@pytest.mark.parametrize("M,N,K,G,cap,panel", [
+    (300, 200, 130, 1, 0, 0),          # row-major A file
+    (256, 384, 512, 2, 0, 128),        # K-panel-major A, two siblings
+    (400, 520, 700, 2, 700_000, 64),   # HBM capacity forces several C-block rounds
+    (130, 70, 33, 4, 0, 16),           # ragged last panel, 2 x 2 grid
+])
+def test_file_root_plan_simulation(M, N, K, G, cap, panel):
+    A = nugen.fill(M, K, 4, 1, "int")
+    B = nugen.fill(K, N, 4, 2, "int")
+    ref = A.astype(np.float64) @ B.astype(np.float64)
+    t = file_tree(G, cap)
+    p = t.plan(M, N, K, nu.make_opts(k_chunk=64, a_panel_k=panel))
+    ops = p.ops()
+    assert any(o["op"] == nu.NU_OP_IO_READ for o in ops) and any(o["op"] == nu.NU_OP_IO_WRITE for o in ops)
+    lay = kpanels(A, panel) if panel else None
+    assert np.array_equal(simulate(p, A, B, M, N, K, a_layout=lay), ref)
+    for seed in range(4):
+        C = simulate(p, A, B, M, N, K, rng=random.Random(seed), a_layout=lay)
+        assert np.array_equal(C, ref), f"order seed {seed} broke a dependency"
+    s = p.stats()
+    assert s["bytes_file_write"] == 4 * M * N
+    t.destroy()
+
+
+def test_file_tile_kpanels_round_trip(tmp_path):
+    M, K, P = 37, 101, 16
+    A = nugen.fill(M, K, 5, 1)
+    src, dst = tmp_path / "a.bin", tmp_path / "a_tiled.bin"
+    A.tofile(src)
+    nu.file_tile_kpanels(str(src), str(dst), M, K, P)
+    assert np.array_equal(np.fromfile(dst, dtype=np.float32), kpanels(A, P).astype(np.float32))
