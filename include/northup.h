@@ -108,6 +108,12 @@ int northup_tree_set_block(northup_tree_t t, int node, int64_t bm, int64_t bn, i
  * node instead of cudaMalloc. The arena must stay valid until destroy. */
 int northup_tree_set_arena(northup_tree_t t, int node, void* dev_ptr, uint64_t bytes);
 
+/* Register the caller-owned device buffer (M x N fp32, row-major) that
+ * receives the whole C on this HBM node when northup_gemm_ex runs with
+ * opts->replicate_result (S§8(e): NCCL over NVLink for distinct devices,
+ * device copies for siblings aliasing one device).  NULL unregisters. */
+int northup_tree_set_replica(northup_tree_t t, int node, void* dev_ptr, uint64_t bytes);
+
 /* Validate the tree (P:95 level rule: every path from the root ends in a leaf
  * with a processor; storage levels only get faster towards the leaves), create
  * streams/events for every HBM node, and prepare the per-node arenas.
@@ -170,7 +176,8 @@ int northup_release(northup_tree_t t, northup_buf_t b);
 /* ------------------------------------------------------- the GEMM (§IV-A) */
 typedef struct {
   int schedule;         /* NU_SCHED_AUTO / S1 / S2 */
-  int replicate_result; /* 1: after the join, all-gather C to every GPU's HBM (NCCL) */
+  int replicate_result; /* 1: after the join, gather C into every HBM node's replica
+                           buffer (northup_tree_set_replica) — NCCL over NVLink */
   int64_t k_chunk;      /* TMEM accumulation length in K (0 = library default, 2048) */
   int npass;            /* 3 = 3xTF32 (default, 0 means 3); 1 = plain TF32 (tests only) */
   int resident;         /* 1: run the plan with operands already resident (in-HBM timing) */

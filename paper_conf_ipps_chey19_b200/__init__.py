@@ -102,6 +102,7 @@ _SIGS = {
     "northup_tree_add_node": [_vp, _int, _int, _int, _u64, _int, _pint],
     "northup_tree_set_block": [_vp, _int, _i64, _i64, _i64],
     "northup_tree_set_arena": [_vp, _int, _vp, _u64],
+    "northup_tree_set_replica": [_vp, _int, _vp, _u64],
     "northup_tree_finalize": [_vp],
     "northup_tree_destroy": [_vp],
     "northup_fetch_node_type": [_vp, _int, _pint],
@@ -339,6 +340,11 @@ class Tree:
 
     def set_arena(self, node: int, ptr: int, nbytes: int, keepalive=None) -> None:
         check(lib().northup_tree_set_arena(self.handle, node, ptr, nbytes))
+        if keepalive is not None:
+            self._keep.append(keepalive)
+
+    def set_replica(self, node: int, ptr: int, nbytes: int, keepalive=None) -> None:
+        check(lib().northup_tree_set_replica(self.handle, node, ptr, nbytes))
         if keepalive is not None:
             self._keep.append(keepalive)
 

@@ -37,7 +37,7 @@ def build(force: bool = False, verbose: bool = False, out: str = OUT, defines=()
     if out == OUT and not defines and not force and not _stale():
         return OUT
     cmd = [NVCC, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"),
-           "-o", out + ".tmp", *sources(), "-lpthread"]
+           "-o", out + ".tmp", *sources(), "-lpthread", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

@@ -66,8 +66,8 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
   const uint64_t need_a = 4ull * M * K, need_b = 4ull * K * N, need_c = 4ull * M * N;
   if (A->bytes < need_a || B->bytes < need_b || C->bytes < need_c)
     return fail(NU_EINVAL, "buffer smaller than its matrix");
-  if (o && o->replicate_result && t->workers.size() > 1)
-    return fail(NU_ENOTSUP, "replicate_result needs the NCCL gather (not built in this version)");
+  if (o && o->replicate_result && t->nodes[0].storage == NU_FILE)
+    return fail(NU_ENOTSUP, "replicate_result from a FILE root is not supported");
   northup_stats local{};
   northup_stats* st = s ? s : &local;
   *st = northup_stats{};
@@ -89,6 +89,7 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
     int prev = 0;
     cudaGetDevice(&prev);
     rc = execute_plan(t, plan, A, B, C, o, st);
+    if (!rc && o && o->replicate_result) rc = gather_replicas(t, plan, C, st);
     cudaSetDevice(prev);
   }
   t->busy = false;

@@ -39,6 +39,9 @@ struct Node {
   void* arena = nullptr;
   uint64_t arena_bytes = 0;
   bool arena_owned = false;
+  // replicate_result target (caller-owned device buffer of M x N floats)
+  void* replica = nullptr;
+  uint64_t replica_bytes = 0;
 };
 
 }  // namespace nu
@@ -66,6 +69,7 @@ struct northup_tree_s {
   std::string file_dir = "/tmp";
   std::vector<northup_buf_s*> bufs;
   std::vector<WorkerState*> workers;   // one per HBM node (created at finalize)
+  std::vector<void*> nccl_comms;       // ncclComm_t per HBM sibling (replicate_result)
 };
 
 namespace nu {
@@ -118,6 +122,8 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,
                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
 int finalize_workers(northup_tree_s* t);
+int gather_replicas(northup_tree_s* t, const Plan& P, northup_buf_s* C, northup_stats* st);
+void destroy_nccl(northup_tree_s* t);
 void destroy_workers(northup_tree_s* t);
 
 }  // namespace nu

@@ -165,3 +165,22 @@ def test_hbm_capacity_enforced():
         t.alloc(2 << 20, hbm[0])
     assert e.value.code == nu.NU_ENOMEM
     t.destroy()
+
+
+@pytest.mark.parametrize("G", [1, 2, 4])
+def test_replicate_result(G):
+    """S§8(e) replicate_result: every sibling's HBM replica holds the whole C
+    (G = 1; G > 1 as virtual siblings on one device -> device-copy gather)."""
+    M, N, K = 700, 520, 900
+    t, hbm = nu.host_tree(G, devices=[0] * G)
+    t.finalize()
+    p = HostProblem(t, M, N, K, 3, "int")
+    reps = [torch.full((M, N), float("nan"), device="cuda:0") for _ in range(G)]
+    for h, r in zip(hbm, reps):
+        t.set_replica(h, r.data_ptr(), r.numel() * 4)
+    st = t.gemm(p.A, p.B, p.C, M, N, K, nu.make_opts(replicate_result=True))
+    ref = oracle.gemm(p.a, p.b)
+    assert np.array_equal(p.c.astype(np.float64), ref)
+    for r in reps:
+        assert np.array_equal(r.cpu().numpy().astype(np.float64), ref)
+    t.destroy()
