@@ -221,12 +221,24 @@ static int run_worker(RunCtx& c, int wi, double* busy) {
     if (e != cudaSuccess) return cuda_fail(e, "stream synchronize");
   }
   if (c.timing) {
+    // per-op (start, end) relative to this worker's first op, for the timeline
+    int first = -1;
+    for (size_t i = 0; i < nops; ++i)
+      if (P.ops[i].worker == wi) {
+        first = static_cast<int>(i);
+        break;
+      }
     for (size_t i = 0; i < nops; ++i) {
       const northup_op& op = P.ops[i];
       if (op.worker != wi) continue;
-      float ms = 0.f;
+      float ms = 0.f, t0 = 0.f, t1 = 0.f;
       if (cudaEventElapsedTime(&ms, w->tev[2 * i], w->tev[2 * i + 1]) == cudaSuccess)
         busy[op.stream] += ms;
+      cudaEventElapsedTime(&t0, w->tev[2 * first], w->tev[2 * i]);
+      cudaEventElapsedTime(&t1, w->tev[2 * first], w->tev[2 * i + 1]);
+      std::lock_guard<std::mutex> g(c.m);
+      c.t->timeline.push_back({static_cast<float>(i), static_cast<float>(wi),
+                               static_cast<float>(op.stream), t0, t1});
     }
   }
   return 0;
@@ -329,6 +341,7 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   }
   ctx.needs_event = &needs;
   ctx.issued.assign(P.ops.size(), 0);
+  if (ctx.timing) t->timeline.clear();
   ctx.io_done.assign(P.ops.size(), 0);
 
   const int W = P.num_workers;
@@ -373,3 +386,13 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
 }
 
 }  // namespace nu
+
+// Debug (not in northup.h): per-op timeline of the last collect_timing run,
+// rows of (op index, worker, stream, start ms, end ms).  Returns the row count.
+extern "C" int northup_debug_timeline(northup_tree_t t, float* out, int cap_rows) {
+  if (!t) return -1;
+  const int n = static_cast<int>(t->timeline.size());
+  for (int i = 0; i < n && i < cap_rows; ++i)
+    for (int j = 0; j < 5; ++j) out[5 * i + j] = t->timeline[i][j];
+  return n;
+}

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <array>
 #include <string>
 #include <vector>
 
@@ -70,6 +71,7 @@ struct northup_tree_s {
   std::vector<northup_buf_s*> bufs;
   std::vector<WorkerState*> workers;   // one per HBM node (created at finalize)
   std::vector<void*> nccl_comms;       // ncclComm_t per HBM sibling (replicate_result)
+  std::vector<std::array<float, 5>> timeline;   // last collect_timing run (debug)
 };
 
 namespace nu {

@@ -76,9 +76,22 @@ namespace {
 struct Access {
   int op;
   int stream;
-  int64_t lo, hi;
+  int64_t lo, hi;      // bounding element interval
+  int64_t off, ld, rows, cols;
   bool write;
 };
+
+// Do two 2-D regions of one buffer overlap?  Exact rectangle test when both
+// use the same leading dimension and stay inside it, else the bounding
+// intervals (conservative).
+static bool overlaps(const Access& p, int64_t lo, int64_t hi, int64_t off, int64_t ld, int64_t rows,
+                     int64_t cols) {
+  if (p.hi <= lo || hi <= p.lo) return false;
+  if (p.ld != ld || ld <= 0) return true;
+  const int64_t pr = p.off / ld, pc = p.off % ld, r = off / ld, c = off % ld;
+  if (pc + p.cols > ld || c + cols > ld) return true;
+  return pr < r + rows && r < pr + p.rows && pc < c + cols && c < pc + p.cols;
+}
 
 struct Builder {
   Plan* P;
@@ -112,8 +125,8 @@ struct Builder {
       const bool user = P->bufs[a.buf].kind != B_ARENA && P->bufs[a.buf].kind != B_DRAM;
       auto& h = hist[a.buf];
       for (const Access& p : h) {
-        if (p.hi <= lo || hi <= p.lo) continue;
         if (!a.write && !p.write) continue;
+        if (!overlaps(p, lo, hi, a.off, a.ld, a.rows, a.cols)) continue;
         const northup_op& q = P->ops[p.op];
         if (q.worker == op.worker && q.stream == op.stream) continue;
         // root-tier regions of different siblings are disjoint by construction
@@ -128,7 +141,7 @@ struct Builder {
           }
         if (!found) last.emplace_back(key, p.op);
       }
-      h.push_back(Access{idx, op.stream, lo, hi, a.write});
+      h.push_back(Access{idx, op.stream, lo, hi, a.off, a.ld, a.rows, a.cols, a.write});
     }
     op.ndeps = 0;
     for (auto& kv : last) {
@@ -238,7 +251,11 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
   // Prefer whole-region blocks (fewest H2D bytes), then the longest tail.
   for (int64_t bn : bns) {
     for (int64_t bm : bms) {
-      const int64_t tails[] = {std::min(K, want_tail), std::min(K, want_tail / 2),
+      // a tail longer than the break-even 2P/BW lets graded (shrinking) strips
+      // keep D2H behind compute down to a small last strip
+      const int64_t long_tail = rup(want_tail * 8 / 5, x.kc);
+      const int64_t tails[] = {long_tail < K ? long_tail : std::min(K, want_tail),
+                               std::min(K, want_tail), std::min(K, want_tail / 2),
                                std::min(K, x.kc), 0};
       for (int64_t tail : tails) {
         if (tail < 0) continue;
@@ -299,7 +316,11 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
     st->bn = s.bn;
     st->bk = s.bk;
     st->tail_k = s.tail;
-    st->strips = s.tail > 0 ? cdiv(s.bm, s.sr) : 0;
+    st->strips = 0;
+    for (int64_t r = 0, rr = 0; s.tail > 0 && r < s.bm; r += rr, ++st->strips) {
+      const int64_t rem = s.bm - r;
+      rr = rem > 2 * s.sr ? s.sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
+    }
     st->hbm_peak_bytes = s.bytes;
     st->schedule = NU_SCHED_S2;
   }
@@ -324,28 +345,50 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
       for (int64_t p = 0; p < npan; ++p, ++panel_it) {
         const int sl = panel_it % kSlots;
         const int64_t k0 = p * s.bk, kk = std::min(s.bk, kmain - k0);
-        B.emit(make_copy(w, S_H2D, x.A, gr * x.lda + k0, x.lda, arena, offSA[sl], ldA, bm, kk),
-               {{x.A, gr * x.lda + k0, x.lda, bm, kk, false}, {arena, offSA[sl], ldA, bm, kk, true}});
-        B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc, x.ldb, arena, offSB[sl], ldBs, kk, bn),
-               {{x.Bb, k0 * x.ldb + gc, x.ldb, kk, bn, false},
-                {arena, offSB[sl], ldBs, kk, bn, true}});
         st->bytes_h2d += static_cast<uint64_t>(bm) * kk * 4 + static_cast<uint64_t>(kk) * bn * 4;
-        B.emit(make_leaf(w, arena, offSA[sl], ldA, arena, offSB[sl], ldBs, arena, offC, ldC, bm, bn,
-                         kk, p > 0 ? 1 : 0),
-               {{arena, offSA[sl], ldA, bm, kk, false},
-                {arena, offSB[sl], ldBs, kk, bn, false},
-                {arena, offC, ldC, bm, bn, true}});
-        st->leaf_launches++;
-        // interleave the B-tail pieces over the main phase so they overlap compute
-        while (pieces_done < ntail_pieces && (pieces_done + 1) * npan <= (p + 1) * ntail_pieces) {
+        // The first panel is computed in a 4 x 4 grid of sub-blocks so the
+        // leaf starts after 1/4 of A's and B's panel have landed instead of
+        // the whole panel (pipeline fill); per-element arithmetic is unchanged.
+        const int64_t gb = (p == 0 && bm >= 4096 && bn >= 4096) ? 4 : 1;
+        const int64_t sbm = rup(cdiv(bm, gb), 256), sbn = rup(cdiv(bn, gb), 256);
+        for (int64_t jj = 0; jj < bn; jj += sbn) {
+          const int64_t cn = std::min(sbn, bn - jj);
+          B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc + jj, x.ldb, arena, offSB[sl] + jj, ldBs,
+                           kk, cn),
+                 {{x.Bb, k0 * x.ldb + gc + jj, x.ldb, kk, cn, false},
+                  {arena, offSB[sl] + jj, ldBs, kk, cn, true}});
+          for (int64_t ii = 0; ii < bm; ii += sbm) {
+            const int64_t rm = std::min(sbm, bm - ii);
+            if (jj == 0)
+              B.emit(make_copy(w, S_H2D, x.A, (gr + ii) * x.lda + k0, x.lda, arena,
+                               offSA[sl] + ii * ldA, ldA, rm, kk),
+                     {{x.A, (gr + ii) * x.lda + k0, x.lda, rm, kk, false},
+                      {arena, offSA[sl] + ii * ldA, ldA, rm, kk, true}});
+            B.emit(make_leaf(w, arena, offSA[sl] + ii * ldA, ldA, arena, offSB[sl] + jj, ldBs, arena,
+                             offC + ii * ldC + jj, ldC, rm, cn, kk, p > 0 ? 1 : 0),
+                   {{arena, offSA[sl] + ii * ldA, ldA, rm, kk, false},
+                    {arena, offSB[sl] + jj, ldBs, kk, cn, false},
+                    {arena, offC + ii * ldC + jj, ldC, rm, cn, true}});
+            st->leaf_launches++;
+          }
+        }
+        // interleave the B-tail pieces over the main phase so they overlap
+        // compute; none during the first panels, whose copies gate the
+        // pipeline fill (the H2D stream is in-order)
+        const int64_t skip = std::min<int64_t>(2, std::max<int64_t>(0, npan - 1));
+        while (pieces_done < ntail_pieces && p >= skip &&
+               (pieces_done + 1) * (npan - skip) <= (p + 1 - skip) * ntail_pieces) {
           load_tail_piece(pieces_done++);
         }
       }
       while (pieces_done < ntail_pieces) load_tail_piece(pieces_done++);
       if (s.tail > 0) {
         // ---- tail phase: strips of C finish and drain one by one
-        for (int64_t r = 0; r < bm; r += s.sr, ++strip_it) {
-          const int64_t rr = std::min(s.sr, bm - r);
+        // Graded strips: full strips while more than two remain, then halving
+        // sizes, so the last D2H (the exposed drain) is small.
+        for (int64_t r = 0, rr = 0; r < bm; r += rr, ++strip_it) {
+          const int64_t rem = bm - r;
+          rr = rem > 2 * s.sr ? s.sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
           const int sl = strip_it % kSlots;
           B.emit(make_copy(w, S_H2D, x.A, (gr + r) * x.lda + kmain, x.lda, arena, offAT[sl], ldAt, rr,
                            s.tail),
