@@ -9,6 +9,6 @@ A = torch.rand((M, K), device=dev) * 2 - 1
 B = torch.rand((K, N), device=dev) * 2 - 1
 C = torch.empty((M, N), device=dev)
 for _ in range(3):
-    nu.leaf_gemm(A, B, C, k_chunk=1024)
+    nu.leaf_gemm(A, B, C)
 torch.cuda.synchronize()
 print("done")
