@@ -270,16 +270,21 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     peaks = measured_peaks()
     p_tf32 = peaks["bf16_sustained"] * NOMINAL_TF32_OVER_BF16
     p_eff = p_tf32 / 3.0
-    leaf_ms = statistics.mean(per_hbm)
-    achieved = 2.0 * m * n * K / (leaf_ms * 1e-3) / 1e12
+    # dominant kernel: the leaf.  One in-HBM step = ceil(K / k_chunk) K-panel
+    # launches on the torch stream (leaf_host.cu), back to back.
+    kc_eff = kc or 2048
+    launches_per_step = -(-K // kc_eff)
+    leaf_ms = statistics.mean(per_hbm) / launches_per_step
+    flops_per_launch = 2.0 * m * n * min(K, kc_eff)
+    achieved = flops_per_launch / (leaf_ms * 1e-3) / 1e12
     traffic = None
     tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
             tj = json.load(f)
-        if (tj.get("M"), tj.get("N"), tj.get("K")) == (m, n, K):
+        if (tj.get("M"), tj.get("N"), tj.get("launch_K")) == (m, n, min(K, kc_eff)):
             traffic = tj.get("dram_bytes")
-
+    clock_ghz = None
     result = None
     if rank == 0:
         cpu = None
@@ -324,9 +329,13 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                                         f"{peaks['bf16_sustained']} TF/s x nominal tf32/bf16 "
                                         f"{NOMINAL_TF32_OVER_BF16:.3f} / 3 MMAs"),
                          "tensor_pipe_frac_of_tf32_peak": round(3 * achieved / p_tf32, 4),
-                         "kernel": "nu::leaf::sm2::leaf_gemm_2sm_kernel", "launch": [m, n, K],
-                         "ms_per_launch": round(leaf_ms, 3)},
-            "gpu_launches": args.steps + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
+                         "kernel": "nu::leaf::sm2::leaf_gemm_2sm_kernel",
+                         "launch": [m, n, min(K, kc_eff)], "launches_per_step": launches_per_step,
+                         "flops_per_launch": flops_per_launch, "ms_per_launch": round(leaf_ms, 3),
+                         "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "
+                                          "(profiles/leaf_traffic.json); algorithmic bytes per launch "
+                                          f"= A/B panel + C read+write = {4 * (m + n) * min(K, kc_eff) + 8 * m * n:.3e}"},
+            "gpu_launches": args.steps * launches_per_step + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
             "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise_cross_tier,
                        "bitwise_tree_vs_leaf": bitwise_tree_vs_leaf},
             "clocks": clk.summary(),

@@ -658,8 +658,24 @@ int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K, const n
   return build_plan_ex(t, M, N, K, o, true, true, out);
 }
 
+static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
+                           const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out);
+
 int build_plan_ex(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
                   const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out) {
+  int rc = build_plan_impl(t, M, N, K, o, a_aligned, b_aligned, out);
+  if (rc) return rc;
+  // leaf_launches counts kernel launches: the leaf issues one launch per
+  // k_chunk panel of each LEAF op (leaf_host.cu, kPanelChunks).
+  int64_t n = 0;
+  for (const northup_op& op : out->ops)
+    if (op.op == NU_OP_LEAF) n += kPanelChunks > 0 ? cdiv(op.k, kPanelChunks * out->kc) : 1;
+  out->stats.leaf_launches = n;
+  return 0;
+}
+
+static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
+                           const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out) {
   int rc = validate_tree(t);
   if (rc) return rc;
   if (M < 0 || N < 0 || K < 0) return fail(NU_EINVAL, "negative dimension");
