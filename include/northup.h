@@ -179,7 +179,8 @@ typedef struct {
   int replicate_result; /* 1: after the join, gather C into every HBM node's replica
                            buffer (northup_tree_set_replica) — NCCL over NVLink */
   int64_t k_chunk;      /* TMEM accumulation length in K (0 = library default, 2048) */
-  int npass;            /* 3 = 3xTF32 (default, 0 means 3); 1 = plain TF32 (tests only) */
+  int npass;            /* leaf split (R19/R21): 0 = default (2); 2 = tf32 hi.hi +
+                           bf16 cross terms; 3 = 3xTF32; 1 = plain TF32 (negative test) */
   int resident;         /* 1: run the plan with operands already resident (in-HBM timing) */
   int collect_timing;   /* 1: record per-stage CUDA-event timings into the stats */
   int64_t a_panel_k;    /* FILE root only: A is stored K-panel-major (R15 preprocessing,
@@ -221,7 +222,8 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
  * C = A.B (accumulate = 0) or C += A.B (accumulate = 1), row-major, on `stream`
  * (a cudaStream_t, NULL = legacy default) of the CURRENT device. A and B need a
  * 16-byte-aligned base and lda, ldb multiples of 4 (TMA); C any alignment.
- * k_chunk = TMEM accumulation length (0 = 2048); npass 3 = 3xTF32, 1 = TF32.
+ * k_chunk = TMEM accumulation length (0 = 2048); npass 0/2 = tf32 hi.hi + bf16
+ * cross terms, 3 = 3xTF32, 1 = plain TF32 (negative test).
  * Asynchronous: returns after the launch. */
 int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                       int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t k_chunk,

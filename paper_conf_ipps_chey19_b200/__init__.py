@@ -194,14 +194,14 @@ def _stream_ptr(stream) -> int | None:
 
 
 def northup_leaf_gemm(A: int, lda: int, B: int, ldb: int, C: int, ldc: int, M: int, N: int,
-                      K: int, accumulate: int = 0, k_chunk: int = 0, npass: int = 3,
+                      K: int, accumulate: int = 0, k_chunk: int = 0, npass: int = 0,
                       stream=None) -> None:
     """Raw leaf call on device pointers (asynchronous on `stream`)."""
     check(lib().northup_leaf_gemm(A, lda, B, ldb, C, ldc, M, N, K, accumulate, k_chunk, npass,
                                   _stream_ptr(stream)))
 
 
-def leaf_gemm(A, B, C, accumulate: bool = False, k_chunk: int = 0, npass: int = 3,
+def leaf_gemm(A, B, C, accumulate: bool = False, k_chunk: int = 0, npass: int = 0,
               stream=None) -> None:
     """C (+)= A @ B for row-major fp32 CUDA tensors (views with unit column stride)."""
     M, K = A.shape
@@ -236,7 +236,7 @@ def partition_region(G: int, M: int, N: int, K: int, r: int) -> tuple[int, int, 
     return tuple(x.value for x in v)
 
 
-def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 3,
+def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 0,
               collect_timing: bool = False, replicate_result: bool = False,
               a_panel_k: int = 0) -> GemmOpts:
     o = GemmOpts()

@@ -23,6 +23,7 @@
 //   tfull[a]   (each CTA)  leader's commit, multicast          -> own epilogue
 //   tempty[a]  (leader)    both CTAs drained TMEM (count 2)    -> MMA issuer
 #include <cuda.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -51,6 +52,7 @@ constexpr int A_BYTES = BM_CTA * BK * 4;           // 16 KiB
 constexpr int B_BYTES = BN_CTA * BK * 4;           // 16 KiB
 constexpr int TMA_BYTES = A_BYTES + B_BYTES;       // per CTA per stage
 constexpr int STAGE_BYTES = TMA_BYTES;             // one raw or one lo stage
+constexpr int XA_BYTES = BM_CTA * 2 * BK * 2;      // A' (bf16, 2 x BK virtual k): 16 KiB
 #ifndef NU_LEAF_XFORM_WARPS
 #define NU_LEAF_XFORM_WARPS 4
 #endif
@@ -155,6 +157,36 @@ __device__ __forceinline__ void umma_tf32_2sm_alast(uint32_t tmem_d, uint64_t da
       : "memory");
 }
 
+__device__ __forceinline__ void umma_bf16_2sm(uint32_t tmem_d, uint64_t da, uint64_t db,
+                                              uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+// Instruction descriptor, kind::f16 with bf16 operands: D f32 [4,6)=1,
+// A bf16 [7,10)=1, B bf16 [10,13)=1, A K-major, B MN-major, N>>3, M>>4.
+__host__ __device__ constexpr uint32_t idesc_bf16(int m, int n) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) |
+         (static_cast<uint32_t>(n >> 3) << 17) | (static_cast<uint32_t>(m >> 4) << 24);
+}
+
+__device__ __forceinline__ void sts64(uint32_t a, uint32_t x, uint32_t y) {
+  asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(a), "r"(x), "r"(y) : "memory");
+}
+
+__device__ __forceinline__ uint32_t pack_bf16(float lo_elem, float hi_elem) {
+  __nv_bfloat162 v = __floats2bfloat162_rn(lo_elem, hi_elem);   // .x at the lower address
+  return *reinterpret_cast<uint32_t*>(&v);
+}
+
+__device__ __forceinline__ float trunc13(float x) {
+  return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+}
+
 // Arrive on the same barrier offset in both CTAs of the pair once the MMAs
 // issued so far have completed.
 __device__ __forceinline__ void umma_commit_pair(uint32_t bar) {
@@ -249,6 +281,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     // ------------------------------------------------ MMA issuer (leader CTA only)
     if (leader && lane == 0) {
       const uint32_t idesc = idesc_tf32(BM, BN, 1u);
+      const uint32_t idesc_bf = idesc_bf16(BM, BN);
       uint32_t it = 0, chunk_it = 0;
       long long w_xf = 0, w_te = 0, t_beg = clock64();   // profile mode (p.dbg)
       for (int t = cid; t < num_tiles; t += nclusters) {
@@ -279,7 +312,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
               const uint64_t dbh = umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
               const uint64_t dbl = umma_desc(b_lo + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
               const uint32_t first = (kb == kb0 && k == 0) ? 0u : 1u;
-              if (p.npass == 3) {
+              if (p.npass == 2) {
+                // hi.hi in tf32 on the raw tiles, then both cross terms of
+                // this k8 step in ONE bf16 MMA over 16 virtual k (hi_a|lo_a)
+                // x (lo_b;hi_b) from the split's bf16 tiles (R21)
+                umma_tf32_2sm(tmem_d, dah, dbh, idesc, first);
+                const uint64_t da2 = umma_desc(a_lo + k * 32, 16, 1024);
+                const uint64_t db2 = umma_desc(a_lo + XA_BYTES + k * 2048, 8192, 1024);
+                umma_bf16_2sm(tmem_d, da2, db2, idesc_bf, 1u);
+              } else if (p.npass == 3) {
                 umma_tf32_2sm_afill(tmem_d, dah, dbl, idesc, first);
                 umma_tf32_2sm_alast(tmem_d, dah, dbh, idesc, 1u);
                 umma_tf32_2sm(tmem_d, dal, dbh, idesc, 1u);
@@ -319,7 +360,54 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         w_lem += clock64() - c1;
         const uint32_t raw = smem_u32(raw_base + s * STAGE_BYTES);
         const uint32_t lo = smem_u32(lo_base + j * STAGE_BYTES);
-        if (p.npass == 3 && !(p.b_kmajor & 2)) {   // exp. 2: skip the split work
+        if (p.npass == 2 && !(p.b_kmajor & 2)) {
+          // A' (K-major SW128 bf16, 128 rows x 64 virtual k): row r, virtual
+          //   chunk 2g = bf16(hi) of real k 8g..8g+7, chunk 2g+1 = bf16(lo)
+#pragma unroll
+          for (int u = 0; u < 512 / XFORM_THREADS; ++u) {
+            const int item = tid + u * XFORM_THREADS;
+            const int r = item >> 2, g = item & 3, sw = r & 7;
+            const uint32_t rowa = raw + r * 128;
+            const uint4 x0 = lds128(rowa + (((2 * g) ^ sw) << 4));
+            const uint4 x1 = lds128(rowa + (((2 * g + 1) ^ sw) << 4));
+            const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
+                                __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
+                                __uint_as_float(x1.z), __uint_as_float(x1.w)};
+            float h[8], l[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              h[e] = trunc13(f[e]);
+              l[e] = f[e] - h[e];
+            }
+            const uint32_t rowd = lo + r * 128;
+            sts128(rowd + (((2 * g) ^ sw) << 4),
+                   make_uint4(pack_bf16(h[0], h[1]), pack_bf16(h[2], h[3]), pack_bf16(h[4], h[5]),
+                              pack_bf16(h[6], h[7])));
+            sts128(rowd + (((2 * g + 1) ^ sw) << 4),
+                   make_uint4(pack_bf16(l[0], l[1]), pack_bf16(l[2], l[3]), pack_bf16(l[4], l[5]),
+                              pack_bf16(l[6], l[7])));
+          }
+          // B' (MN-major SW128 bf16, 64 virtual k x 128 n): virtual row
+          //   16g+i = bf16(lo) of real k 8g+i, 16g+8+i = bf16(hi)
+#pragma unroll
+          for (int u = 0; u < 1024 / XFORM_THREADS; ++u) {
+            const int item = tid + u * XFORM_THREADS;
+            const int k = item >> 5, n0 = (item & 31) * 4;
+            const int nn = n0 & 31;
+            const uint4 x = lds128(raw + A_BYTES + (n0 >> 5) * B_CHUNK_BYTES + k * 128 +
+                                   ((((nn >> 3) ^ (k & 3)) << 5) | ((nn & 7) << 2)));
+            const float f0 = __uint_as_float(x.x), f1 = __uint_as_float(x.y);
+            const float f2 = __uint_as_float(x.z), f3 = __uint_as_float(x.w);
+            const float h0 = trunc13(f0), h1 = trunc13(f1), h2 = trunc13(f2), h3 = trunc13(f3);
+            const int vlo = 16 * (k >> 3) + (k & 7), vhi = vlo + 8;
+            const int c = (n0 & 63) >> 3;
+            const uint32_t base = lo + XA_BYTES + (n0 >> 6) * 8192 + ((n0 & 7) << 1);
+            sts64(base + (vlo >> 3) * 1024 + (vlo & 7) * 128 + ((c ^ (vlo & 7)) << 4),
+                  pack_bf16(f0 - h0, f1 - h1), pack_bf16(f2 - h2, f3 - h3));
+            sts64(base + (vhi >> 3) * 1024 + (vhi & 7) * 128 + ((c ^ (vhi & 7)) << 4),
+                  pack_bf16(h0, h1), pack_bf16(h2, h3));
+          }
+        } else if (p.npass == 3 && !(p.b_kmajor & 2)) {   // exp. 2: skip the split work
           uint4 x[TMA_BYTES / 16 / XFORM_THREADS];
 #pragma unroll
           for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u)

@@ -90,7 +90,7 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
   p.kb_per_chunk = static_cast<int>(kbpc);
   p.accumulate = accumulate ? 1 : 0;
   p.vec_ok = (reinterpret_cast<uintptr_t>(C) % 16 == 0) && (ldc % 4 == 0);
-  p.npass = npass == 1 ? 1 : 3;
+  p.npass = (npass == 1 || npass == 2) ? npass : (npass == 3 ? 3 : kDefaultNpass);
   p.b_kmajor = b_kmajor;
   p.dbg = dbg;
   p.tiles_m = p.tiles_n = 0;
@@ -120,6 +120,7 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
     }
     variant = env_variant;
   }
+  if (variant == 1 && p.npass == 2) p.npass = 3;   // the 1-CTA v0 kernel has no bf16 path
   // K-panel launches: each launch covers `panel` of K for
   // every tile, so all CTAs stream the same K range and share A/B panels in
   // L2; the grid-wide launch boundary re-synchronises them.  panel is a

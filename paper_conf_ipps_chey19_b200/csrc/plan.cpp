@@ -686,7 +686,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   P.K = K;
   P.kc = (o && o->k_chunk > 0) ? o->k_chunk : kDefaultKChunk;
   if (P.kc % 4) return fail(NU_EINVAL, "k_chunk must be a multiple of 4");
-  P.npass = (o && o->npass == 1) ? 1 : 3;
+  P.npass = o ? o->npass : 0;   // 0 = library default (leaf_host.cu)
   const int sched = o ? o->schedule : NU_SCHED_AUTO;
   if (sched < NU_SCHED_AUTO || sched > NU_SCHED_S2) return fail(NU_EINVAL, "unknown schedule");
   Builder B;

@@ -21,7 +21,7 @@ def _dev():
     return torch.device("cuda:0")
 
 
-def run_leaf(A, B, C0=None, accumulate=False, k_chunk=0, npass=3, lda_pad=0, ldb_pad=0, ldc_pad=0):
+def run_leaf(A, B, C0=None, accumulate=False, k_chunk=0, npass=0, lda_pad=0, ldb_pad=0, ldc_pad=0):
     dev = _dev()
     M, K = A.shape
     N = B.shape[1]
@@ -61,13 +61,41 @@ def test_leaf_integer_inputs_bitwise(M, N, K):
         f"{np.argwhere(C.astype(np.float64) != ref)[:5]}"
 
 
+@pytest.mark.parametrize("npass", [2, 3])
 @pytest.mark.parametrize("M,N,K", SHAPES)
-def test_leaf_uniform_normwise(M, N, K):
+def test_leaf_uniform_normwise(M, N, K, npass):
     A = nugen.fill(M, K, 12, 1)
     B = nugen.fill(K, N, 12, 2)
-    C = run_leaf(A, B)
+    C = run_leaf(A, B, npass=npass)
     e = normwise(C, A, B)
     assert e <= TOL, e
+
+
+@pytest.mark.parametrize("M,N,K", [(257, 300, 65), (512, 256, 1024), (1000, 1000, 999)])
+def test_leaf_3xtf32_integer_bitwise(M, N, K):
+    A = nugen.fill(M, K, 11, 1, "int")
+    B = nugen.fill(K, N, 11, 2, "int")
+    assert np.array_equal(run_leaf(A, B, npass=3).astype(np.float64), oracle.gemm(A, B))
+
+
+def test_leaf_v0_one_cta_kernel():
+    """The 1-CTA v0 kernel (kept for comparison) still meets the bar."""
+    import ctypes
+    f = nu.lib().northup_debug_leaf_gemm
+    f.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                  ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                  ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                  ctypes.c_void_p]
+    M, N, K = 300, 520, 1000
+    A = nugen.fill(M, K, 18, 1)
+    B = nugen.fill(K, N, 18, 2)
+    dev = _dev()
+    Ad, Bd = torch.from_numpy(A).to(dev), torch.from_numpy(B).to(dev)
+    Cd = torch.empty((M, N), device=dev)
+    assert f(Ad.data_ptr(), K, Bd.data_ptr(), N, Cd.data_ptr(), N, M, N, K, 0, 0, 3, 0, None, 1,
+             None) == 0
+    torch.cuda.synchronize()
+    assert normwise(Cd.cpu().numpy(), A, B) <= TOL
 
 
 def test_leaf_closed_forms():
@@ -109,13 +137,15 @@ def test_leaf_strided_operands_and_predicated_stores():
 
 
 def test_leaf_plain_tf32_fails_the_bound():
-    """Reading R9: one TF32 pass (npass=1) must NOT meet 1e-5 — the 3xTF32
-    split is what buys fp32-level accuracy (negative test)."""
+    """Reading R9: one TF32 pass (npass=1) must NOT meet 1e-5 — the split
+    (3xTF32, or tf32 hi.hi + bf16 cross terms) is what buys fp32-level
+    accuracy (negative test)."""
     A = nugen.fill(256, 512, 17, 1)
     B = nugen.fill(512, 256, 17, 2)
     e1 = normwise(run_leaf(A, B, npass=1), A, B)
+    e2 = normwise(run_leaf(A, B, npass=2), A, B)
     e3 = normwise(run_leaf(A, B, npass=3), A, B)
-    assert e1 > 1e-4 > TOL >= e3
+    assert e1 > 1e-4 > TOL >= max(e2, e3)
 
 
 def test_leaf_rejects_tma_illegal_operands():
