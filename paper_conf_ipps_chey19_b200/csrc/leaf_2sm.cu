@@ -54,7 +54,7 @@ constexpr int TMA_BYTES = A_BYTES + B_BYTES;       // per CTA per stage
 constexpr int STAGE_BYTES = TMA_BYTES;             // one raw or one lo stage
 constexpr int XA_BYTES = BM_CTA * 2 * BK * 2;      // A' (bf16, 2 x BK virtual k): 16 KiB
 #ifndef NU_LEAF_XFORM_WARPS
-#define NU_LEAF_XFORM_WARPS 4
+#define NU_LEAF_XFORM_WARPS 8
 #endif
 constexpr int XFORM_WARPS = NU_LEAF_XFORM_WARPS;   // split warps (2 .. 2+XFORM_WARPS-1)
 constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
@@ -364,8 +364,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           // A' (K-major SW128 bf16, 128 rows x 64 virtual k): row r, virtual
           //   chunk 2g = bf16(hi) of real k 8g..8g+7, chunk 2g+1 = bf16(lo)
 #pragma unroll
-          for (int u = 0; u < 512 / XFORM_THREADS; ++u) {
+          for (int u = 0; u < (512 + XFORM_THREADS - 1) / XFORM_THREADS; ++u) {
             const int item = tid + u * XFORM_THREADS;
+            if (item >= 512) break;
             const int r = item >> 2, g = item & 3, sw = r & 7;
             const uint32_t rowa = raw + r * 128;
             const uint4 x0 = lds128(rowa + (((2 * g) ^ sw) << 4));
@@ -388,32 +389,50 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
                               pack_bf16(l[6], l[7])));
           }
           // B' (MN-major SW128 bf16, 64 virtual k x 128 n): virtual row
-          //   16g+i = bf16(lo) of real k 8g+i, 16g+8+i = bf16(hi)
+          //   16g+i = bf16(lo) of real k 8g+i, 16g+8+i = bf16(hi).  One item =
+          //   8 consecutive n of one k: a 32-B granule of the raw tile (the
+          //   BASE32B swizzle keeps granules whole) -> one 16-B chunk of B'.
 #pragma unroll
-          for (int u = 0; u < 1024 / XFORM_THREADS; ++u) {
+          for (int u = 0; u < (512 + XFORM_THREADS - 1) / XFORM_THREADS; ++u) {
             const int item = tid + u * XFORM_THREADS;
-            const int k = item >> 5, n0 = (item & 31) * 4;
+            if (item >= 512) break;
+            const int k = item >> 4, n0 = (item & 15) * 8;
             const int nn = n0 & 31;
-            const uint4 x = lds128(raw + A_BYTES + (n0 >> 5) * B_CHUNK_BYTES + k * 128 +
-                                   ((((nn >> 3) ^ (k & 3)) << 5) | ((nn & 7) << 2)));
-            const float f0 = __uint_as_float(x.x), f1 = __uint_as_float(x.y);
-            const float f2 = __uint_as_float(x.z), f3 = __uint_as_float(x.w);
-            const float h0 = trunc13(f0), h1 = trunc13(f1), h2 = trunc13(f2), h3 = trunc13(f3);
+            const uint32_t src = raw + A_BYTES + (n0 >> 5) * B_CHUNK_BYTES + k * 128 +
+                                 (((nn >> 3) ^ (k & 3)) << 5);
+            // lanes 4..7 of each 8-lane phase read the second 16 B first, so a
+            // phase touches 8 distinct bank groups (no 2-way conflict)
+            const uint32_t h1 = (threadIdx.x >> 2) & 1;
+            const uint4 y0 = lds128(src + 16 * h1), y1 = lds128(src + 16 * (h1 ^ 1));
+            const uint4 x0 = h1 ? y1 : y0, x1 = h1 ? y0 : y1;
+            const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
+                                __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
+                                __uint_as_float(x1.z), __uint_as_float(x1.w)};
+            float h[8], l[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              h[e] = trunc13(f[e]);
+              l[e] = f[e] - h[e];
+            }
             const int vlo = 16 * (k >> 3) + (k & 7), vhi = vlo + 8;
             const int c = (n0 & 63) >> 3;
-            const uint32_t base = lo + XA_BYTES + (n0 >> 6) * 8192 + ((n0 & 7) << 1);
-            sts64(base + (vlo >> 3) * 1024 + (vlo & 7) * 128 + ((c ^ (vlo & 7)) << 4),
-                  pack_bf16(f0 - h0, f1 - h1), pack_bf16(f2 - h2, f3 - h3));
-            sts64(base + (vhi >> 3) * 1024 + (vhi & 7) * 128 + ((c ^ (vhi & 7)) << 4),
-                  pack_bf16(h0, h1), pack_bf16(h2, h3));
+            const uint32_t base = lo + XA_BYTES + (n0 >> 6) * 8192;
+            sts128(base + (vlo >> 3) * 1024 + (vlo & 7) * 128 + ((c ^ (vlo & 7)) << 4),
+                   make_uint4(pack_bf16(l[0], l[1]), pack_bf16(l[2], l[3]), pack_bf16(l[4], l[5]),
+                              pack_bf16(l[6], l[7])));
+            sts128(base + (vhi >> 3) * 1024 + (vhi & 7) * 128 + ((c ^ (vhi & 7)) << 4),
+                   make_uint4(pack_bf16(h[0], h[1]), pack_bf16(h[2], h[3]), pack_bf16(h[4], h[5]),
+                              pack_bf16(h[6], h[7])));
           }
         } else if (p.npass == 3 && !(p.b_kmajor & 2)) {   // exp. 2: skip the split work
-          uint4 x[TMA_BYTES / 16 / XFORM_THREADS];
+          constexpr int NV = (TMA_BYTES / 16 + XFORM_THREADS - 1) / XFORM_THREADS;
+          uint4 x[NV];
 #pragma unroll
-          for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u)
-            x[u] = lds128(raw + (tid + u * XFORM_THREADS) * 16);
+          for (int u = 0; u < NV; ++u)
+            if (tid + u * XFORM_THREADS < TMA_BYTES / 16) x[u] = lds128(raw + (tid + u * XFORM_THREADS) * 16);
 #pragma unroll
-          for (int u = 0; u < TMA_BYTES / 16 / XFORM_THREADS; ++u) {
+          for (int u = 0; u < NV; ++u) {
+            if (tid + u * XFORM_THREADS >= TMA_BYTES / 16) break;
             uint4 l;   // lo = x - trunc13(x): exact in fp32
             l.x = __float_as_uint(__uint_as_float(x[u].x) - __uint_as_float(x[u].x & 0xFFFFE000u));
             l.y = __float_as_uint(__uint_as_float(x[u].y) - __uint_as_float(x[u].y & 0xFFFFE000u));

@@ -3,7 +3,6 @@ mkdir -p gpurun_out
 : > gpurun_out/variants.log
 for so in build/variants/*.so; do
   echo "== $so" >> gpurun_out/variants.log
-  NORTHUP_LIB_PATH=$PWD/$so SZ=32768 KCS=2048 timeout 200 python tools/sweep.py perf >> gpurun_out/variants.log 2>&1
-  NORTHUP_LIB_PATH=$PWD/$so SZ=8192 KCS=2048 timeout 200 python tools/sweep.py perf >> gpurun_out/variants.log 2>&1
+  NORTHUP_LIB_PATH=$PWD/$so timeout 300 python tools/npass2_check.py >> gpurun_out/variants.log 2>&1
   NORTHUP_LIB_PATH=$PWD/$so timeout 200 python tools/mma_prof.py >> gpurun_out/variants.log 2>&1
 done

@@ -22,7 +22,7 @@ for (M, N, K, kind) in [(256, 256, 32, "int"), (512, 768, 1024, "int"), (257, 30
         else:
             res[f"{M}x{N}x{K}_{kind}_np{npass}"] = oracle.normwise_err(C, ref, oracle.row_norms(A), oracle.col_norms(B))[0]
 print(json.dumps(res), flush=True)
-for SZ in (8192, 32768):
+for SZ in [int(x) for x in os.environ.get("SZS", "8192,32768").split(",")]:
     A = torch.rand((SZ, SZ), device=dev) * 2 - 1; B = torch.rand((SZ, SZ), device=dev) * 2 - 1
     C = torch.empty((SZ, SZ), device=dev)
     for npass in (2, 3):
