@@ -254,6 +254,20 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     with ClockSampler(local_rank) as clk:
         t_hbm, per_hbm = timed(step_hbm, args.steps, args.warmup)
         t_ooc, per_ooc = timed(step_ooc, args.steps, args.warmup)
+    replicate_ms = None
+    if world > 1 and args.replicate:
+        from paper_conf_ipps_chey19_b200.dist import gather_regions
+        creg = torch.from_numpy(c).to(dev) if args.dist_backend == "nccl" else torch.from_numpy(c.copy())
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        full = gather_regions(creg, M, N, K, rank, world)
+        e1.record(stream)
+        barrier()
+        replicate_ms = e0.elapsed_time(e1)
+        ok = bool(torch.equal(full[r0:r1, c0:c1].cpu(), torch.from_numpy(c)))
+        del full
+        replicate_ms = (replicate_ms, ok)
     c_hbm = Cd.cpu().numpy()
     c_ooc = c.copy()
     bitwise_cross_tier = bool(np.array_equal(c_hbm, c_ooc))
@@ -304,7 +318,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
             "higher_is_better": True,
             "scaling": "strong" if world > 1 else "weak",
             "vs_baseline": None,
-            "dtype": "f32 (3xTF32 tcgen05, fp32 accumulate)",
+            "dtype": "f32 (tcgen05 split: tf32 hi.hi + bf16 cross terms, fp32 accumulate)",
             "data": "synthetic (counter-hash uniform [-1,1) fp32, seed = config index)",
             "config": {
                 "workload": f"{name}: {cfg['desc']}" + (" [quick: /4 sizes]" if args.quick else ""),
@@ -323,6 +337,10 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                     "ms_per_step": round(ms_ooc, 3),
                     "leaf_launches_per_step": int(ooc_stats.get("leaf_launches", 0))},
             "slowdown_pct_vs_in_hbm": round(100.0 * (ms_ooc / ms_hbm - 1.0), 2),
+            "replicate": None if replicate_ms is None else {
+                "ms": round(replicate_ms[0], 3), "region_roundtrip_ok": replicate_ms[1],
+                "backend": args.dist_backend,
+                "bytes_per_gpu_received": 4 * (M * N - m * n)},
             "paper_context": {"avg_ooc_slowdown_pct": 17, "dmm_ooc_gap_pct": 5,
                               "note": "APU + SSD, OpenCL fp32 (PAPER.md P:10, P:381); context only"},
             "roofline": {"bound": "tensor", "achieved": round(achieved, 3),
@@ -410,12 +428,20 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--ref-step-s", type=float, default=5.0)
+    ap.add_argument("--replicate", action="store_true",
+                    help="N>1: after the timed steps, gather C to every GPU (S8e) and time it")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend (gloo only for multi-rank tests on one GPU)")
+    ap.add_argument("--device-mod", type=int, default=0,
+                    help="map LOCAL_RANK modulo this many GPUs (multi-rank tests on one GPU)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("warning: the timing rules ask for >= 3 warm-up steps")
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.device_mod > 0:          # test mode: several ranks share the visible GPUs
+        local_rank %= args.device_mod
 
     if args.impl == "reference":
         if rank == 0:
@@ -426,7 +452,10 @@ def main():
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(args.dist_backend)
     res = run_ours(args, rank, world, local_rank)
     if rank == 0 and res is not None:
         print(json.dumps(res), flush=True)
