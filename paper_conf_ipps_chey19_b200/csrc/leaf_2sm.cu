@@ -29,6 +29,7 @@
 
 #include <atomic>
 
+#include "leaf_2sm_common.cuh"
 #include "leaf_common.cuh"
 #include "northup_internal.h"
 
@@ -66,137 +67,6 @@ constexpr int BAR_BYTES = 256;
 constexpr int SMEM_BYTES = (RS + LS) * STAGE_BYTES + BAR_BYTES + 1024;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 
-__device__ __forceinline__ uint32_t cluster_ctarank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
-
-__device__ __forceinline__ uint32_t mapa(uint32_t saddr, uint32_t rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
-  return r;
-}
-
-// Arrive on a barrier of another CTA of the cluster (address from mapa).
-__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
-
-__device__ __forceinline__ uint4 lds128(uint32_t a) {
-  uint4 v;
-  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
-               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-               : "r"(a));
-  return v;
-}
-
-__device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
-  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z),
-               "r"(v.w)
-               : "memory");
-}
-
-// Wait with cluster-scope acquire (the phase may be completed by the peer CTA).
-__device__ __forceinline__ void mbar_wait_cluster(uint32_t bar, uint32_t parity) {
-  uint32_t done = 0;
-  uint64_t t0 = 0;
-  for (uint32_t it = 0;; ++it) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(done)
-        : "r"(bar), "r"(parity)
-        : "memory");
-    if (done) return;
-    if ((it & 1023u) == 0) {
-      const uint64_t t = globaltimer();
-      if (it == 0) t0 = t;
-      else if (t - t0 > 4000000000ull) __trap();
-    }
-  }
-}
-
-__device__ __forceinline__ void cluster_sync() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
-                   : "memory");
-}
-
-__device__ __forceinline__ void named_bar(uint32_t id, uint32_t count) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
-}
-
-__device__ __forceinline__ void umma_tf32_2sm(uint32_t tmem_d, uint64_t da, uint64_t db,
-                                              uint32_t idesc, uint32_t accum) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(da), "l"(db), "r"(idesc), "r"(accum)
-      : "memory");
-}
-
-__device__ __forceinline__ void umma_tf32_2sm_afill(uint32_t tmem_d, uint64_t da, uint64_t db,
-                                                    uint32_t idesc, uint32_t accum) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::tf32.collector::a::fill [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(da), "l"(db), "r"(idesc), "r"(accum)
-      : "memory");
-}
-
-__device__ __forceinline__ void umma_tf32_2sm_alast(uint32_t tmem_d, uint64_t da, uint64_t db,
-                                                    uint32_t idesc, uint32_t accum) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::tf32.collector::a::lastuse [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(da), "l"(db), "r"(idesc), "r"(accum)
-      : "memory");
-}
-
-__device__ __forceinline__ void umma_bf16_2sm(uint32_t tmem_d, uint64_t da, uint64_t db,
-                                              uint32_t idesc, uint32_t accum) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(da), "l"(db), "r"(idesc), "r"(accum)
-      : "memory");
-}
-
-// Instruction descriptor, kind::f16 with bf16 operands: D f32 [4,6)=1,
-// A bf16 [7,10)=1, B bf16 [10,13)=1, A K-major, B MN-major, N>>3, M>>4.
-__host__ __device__ constexpr uint32_t idesc_bf16(int m, int n) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) |
-         (static_cast<uint32_t>(n >> 3) << 17) | (static_cast<uint32_t>(m >> 4) << 24);
-}
-
-__device__ __forceinline__ void sts64(uint32_t a, uint32_t x, uint32_t y) {
-  asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(a), "r"(x), "r"(y) : "memory");
-}
-
-__device__ __forceinline__ uint32_t pack_bf16(float lo_elem, float hi_elem) {
-  __nv_bfloat162 v = __floats2bfloat162_rn(lo_elem, hi_elem);   // .x at the lower address
-  return *reinterpret_cast<uint32_t*>(&v);
-}
-
-__device__ __forceinline__ float trunc13(float x) {
-  return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
-}
-
-// Arrive on the same barrier offset in both CTAs of the pair once the MMAs
-// issued so far have completed.
-__device__ __forceinline__ void umma_commit_pair(uint32_t bar) {
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
-      " [%0], %1;" ::"r"(bar),
-      "h"(static_cast<uint16_t>(3))
-      : "memory");
-}
-
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     leaf_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tmA,
                          const __grid_constant__ CUtensorMap tmB, const Params p) {
@@ -212,7 +82,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   const uint32_t bar_lempty = bar_xform + 8 * LS;
   const uint32_t bar_tfull = bar_lempty + 8 * LS;
   const uint32_t bar_tempty = bar_tfull + 16;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (2 * RS + 2 * LS + 4));
+  const uint32_t bar_rawfull = bar_tempty + 16;      // [RS] leader: both CTAs' raw tiles landed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (3 * RS + 2 * LS + 4));
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -225,6 +96,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     for (int s = 0; s < RS; ++s) {
       mbar_init(bar_full + 8 * s, 1);
       mbar_init(bar_rempty + 8 * s, 1);
+      mbar_init(bar_rawfull + 8 * s, 2);   // one forwarded arrive per CTA
     }
     for (int j = 0; j < LS; ++j) {
       mbar_init(bar_xform + 8 * j, 2);   // one elected arrive per CTA
@@ -295,16 +167,41 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           const int kb0 = ch * p.kb_per_chunk;
           const int kb1 = min(nkb, kb0 + p.kb_per_chunk);
           for (int kb = kb0; kb < kb1; ++kb, ++it) {
-            const uint32_t s = it % RS;
+            const uint32_t s = it % RS, suse = it / RS;
             const uint32_t j = it % LS, juse = it / LS;
-            c0 = clock64();
-            if (!(p.b_kmajor & 1)) mbar_wait_cluster(bar_xform + 8 * j, juse & 1);   // exp. 1: no wait
-            w_xf += clock64() - c0;
-            tc_fence_after();
             const uint32_t a_hi = smem_u32(raw_base + s * STAGE_BYTES);
             const uint32_t b_hi = a_hi + A_BYTES;
             const uint32_t a_lo = smem_u32(lo_base + j * STAGE_BYTES);
             const uint32_t b_lo = a_lo + A_BYTES;
+            if (p.npass == 2) {
+              // hi.hi needs only the raw tiles: issue it as soon as both CTAs'
+              // TMA landed, so the tensor core works while the split finishes
+              // (R21); then both cross terms per k8 from the split's bf16 tiles.
+              c0 = clock64();
+              mbar_wait_cluster(bar_rawfull + 8 * s, suse & 1);
+              w_xf += clock64() - c0;
+              tc_fence_after();
+#pragma unroll
+              for (int k = 0; k < BK / UMMA_K; ++k)
+                umma_tf32_2sm(tmem_d, umma_desc(a_hi + k * 32, 16, 1024),
+                              umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B),
+                              idesc, (kb == kb0 && k == 0) ? 0u : 1u);
+              c0 = clock64();
+              mbar_wait_cluster(bar_xform + 8 * j, juse & 1);
+              w_xf += clock64() - c0;
+              tc_fence_after();
+#pragma unroll
+              for (int k = 0; k < BK / UMMA_K; ++k)
+                umma_bf16_2sm(tmem_d, umma_desc(a_lo + k * 32, 16, 1024),
+                              umma_desc(a_lo + XA_BYTES + k * 2048, 8192, 1024), idesc_bf, 1u);
+              umma_commit_pair(bar_rempty + 8 * s);
+              umma_commit_pair(bar_lempty + 8 * j);
+              continue;
+            }
+            c0 = clock64();
+            if (!(p.b_kmajor & 1)) mbar_wait_cluster(bar_xform + 8 * j, juse & 1);   // exp. 1: no wait
+            w_xf += clock64() - c0;
+            tc_fence_after();
 #pragma unroll
             for (int k = 0; k < BK / UMMA_K; ++k) {
               const uint64_t dah = umma_desc(a_hi + k * 32, 16, 1024);
@@ -312,15 +209,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
               const uint64_t dbh = umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
               const uint64_t dbl = umma_desc(b_lo + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B);
               const uint32_t first = (kb == kb0 && k == 0) ? 0u : 1u;
-              if (p.npass == 2) {
-                // hi.hi in tf32 on the raw tiles, then both cross terms of
-                // this k8 step in ONE bf16 MMA over 16 virtual k (hi_a|lo_a)
-                // x (lo_b;hi_b) from the split's bf16 tiles (R21)
-                umma_tf32_2sm(tmem_d, dah, dbh, idesc, first);
-                const uint64_t da2 = umma_desc(a_lo + k * 32, 16, 1024);
-                const uint64_t db2 = umma_desc(a_lo + XA_BYTES + k * 2048, 8192, 1024);
-                umma_bf16_2sm(tmem_d, da2, db2, idesc_bf, 1u);
-              } else if (p.npass == 3) {
+              if (p.npass == 3) {
                 umma_tf32_2sm_afill(tmem_d, dah, dbl, idesc, first);
                 umma_tf32_2sm_alast(tmem_d, dah, dbh, idesc, 1u);
                 umma_tf32_2sm(tmem_d, dal, dbh, idesc, 1u);
@@ -346,6 +235,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     // ---------------------------------------------------- transform (own half)
     const int tid = threadIdx.x - 64;
     const uint32_t xform_leader0 = mapa(bar_xform, 0);
+    const uint32_t rawfull_leader0 = mapa(bar_rawfull, 0);
     uint32_t it = 0;
     long long w_full = 0, w_lem = 0;
     for (int t = cid; t < num_tiles; t += nclusters) {
@@ -354,6 +244,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         const uint32_t j = it % LS, juse = it / LS;
         long long c0 = clock64();
         mbar_wait(bar_full + 8 * s, use & 1);
+        if (p.npass == 2 && tid == 0) mbar_arrive_cluster(rawfull_leader0 + 8 * s);
         long long c1 = clock64();
         mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
         w_full += c1 - c0;
@@ -361,6 +252,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         const uint32_t raw = smem_u32(raw_base + s * STAGE_BYTES);
         const uint32_t lo = smem_u32(lo_base + j * STAGE_BYTES);
         if (p.npass == 2 && !(p.b_kmajor & 2)) {
+          const bool ptr_ = (p.b_kmajor & 4) != 0;
+#define PK(a, b) (ptr_ ? pack_bf16_trunc(a, b) : pack_bf16(a, b))
           // A' (K-major SW128 bf16, 128 rows x 64 virtual k): row r, virtual
           //   chunk 2g = bf16(hi) of real k 8g..8g+7, chunk 2g+1 = bf16(lo)
 #pragma unroll
@@ -382,11 +275,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             }
             const uint32_t rowd = lo + r * 128;
             sts128(rowd + (((2 * g) ^ sw) << 4),
-                   make_uint4(pack_bf16(h[0], h[1]), pack_bf16(h[2], h[3]), pack_bf16(h[4], h[5]),
-                              pack_bf16(h[6], h[7])));
+                   make_uint4(PK(h[0], h[1]), PK(h[2], h[3]), PK(h[4], h[5]),
+                              PK(h[6], h[7])));
             sts128(rowd + (((2 * g + 1) ^ sw) << 4),
-                   make_uint4(pack_bf16(l[0], l[1]), pack_bf16(l[2], l[3]), pack_bf16(l[4], l[5]),
-                              pack_bf16(l[6], l[7])));
+                   make_uint4(PK(l[0], l[1]), PK(l[2], l[3]), PK(l[4], l[5]),
+                              PK(l[6], l[7])));
           }
           // B' (MN-major SW128 bf16, 64 virtual k x 128 n): virtual row
           //   16g+i = bf16(lo) of real k 8g+i, 16g+8+i = bf16(hi).  One item =
@@ -418,12 +311,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             const int c = (n0 & 63) >> 3;
             const uint32_t base = lo + XA_BYTES + (n0 >> 6) * 8192;
             sts128(base + (vlo >> 3) * 1024 + (vlo & 7) * 128 + ((c ^ (vlo & 7)) << 4),
-                   make_uint4(pack_bf16(l[0], l[1]), pack_bf16(l[2], l[3]), pack_bf16(l[4], l[5]),
-                              pack_bf16(l[6], l[7])));
+                   make_uint4(PK(l[0], l[1]), PK(l[2], l[3]), PK(l[4], l[5]),
+                              PK(l[6], l[7])));
             sts128(base + (vhi >> 3) * 1024 + (vhi & 7) * 128 + ((c ^ (vhi & 7)) << 4),
-                   make_uint4(pack_bf16(h[0], h[1]), pack_bf16(h[2], h[3]), pack_bf16(h[4], h[5]),
-                              pack_bf16(h[6], h[7])));
+                   make_uint4(PK(h[0], h[1]), PK(h[2], h[3]), PK(h[4], h[5]),
+                              PK(h[6], h[7])));
           }
+#undef PK
         } else if (p.npass == 3 && !(p.b_kmajor & 2)) {   // exp. 2: skip the split work
           constexpr int NV = (TMA_BYTES / 16 + XFORM_THREADS - 1) / XFORM_THREADS;
           uint4 x[NV];

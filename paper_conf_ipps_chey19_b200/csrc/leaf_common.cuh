@@ -27,6 +27,10 @@ struct Params {
   int npass;          // 3 = 3xTF32 (product path), 1 = plain TF32 (negative test)
   int b_kmajor;       // debug: B given as N x K (K-major) instead of K x N
   float* dbg;         // debug: dump of stage 0 after the split (NULL in production)
+  const float* A;     // operands for the LDG-fed kernel (v2): row-major, 16-B aligned
+  int64_t lda;
+  const float* B;
+  int64_t ldb;
 };
 
 // ---------------------------------------------------------------- PTX helpers
@@ -190,7 +194,8 @@ int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t oute
               uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer,
               CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B);
 int launch_sm1(LaunchArgs& a);   // v0: 1-CTA 128 x 256 tile
-int launch_sm2(LaunchArgs& a);   // v1: CTA pair (cta_group::2) 256 x 256 tile
+int launch_sm2(LaunchArgs& a);   // v1: CTA pair (cta_group::2) 256 x 256 tile, TMA-fed
+int launch_sm3(LaunchArgs& a);   // v2: CTA pair, split warps load global memory directly
 
 }  // namespace leaf
 }  // namespace nu

@@ -116,11 +116,12 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
     static int env_variant = -1;
     if (env_variant < 0) {
       const char* v = getenv("NORTHUP_LEAF");
-      env_variant = (v && v[0] == '1') ? 1 : 2;
+      env_variant = (v && v[0] >= '1' && v[0] <= '3') ? v[0] - '0' : kDefaultLeafVariant;
     }
     variant = env_variant;
   }
   if (variant == 1 && p.npass == 2) p.npass = 3;   // the 1-CTA v0 kernel has no bf16 path
+  if (variant == 3 && (p.npass != 2 || b_kmajor)) variant = 2;   // v2 implements R21 only
   // K-panel launches: each launch covers `panel` of K for
   // every tile, so all CTAs stream the same K range and share A/B panels in
   // L2; the grid-wide launch boundary re-synchronises them.  panel is a
@@ -139,7 +140,11 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
     b.B = B + (b_kmajor ? k0 : k0 * ldb);
     b.p.K = static_cast<int>(kk);
     b.p.accumulate = (k0 > 0 || accumulate) ? 1 : 0;
-    rc = variant == 1 ? launch_sm1(b) : launch_sm2(b);
+    b.p.A = b.A;
+    b.p.lda = lda;
+    b.p.B = b.B;
+    b.p.ldb = ldb;
+    rc = variant == 1 ? launch_sm1(b) : variant == 3 ? launch_sm3(b) : launch_sm2(b);
   }
   return rc;
 }

@@ -169,3 +169,28 @@ def test_leaf_degenerate_sizes():
                  accumulate=True)
     torch.cuda.synchronize()
     assert (C2 == 3).all()            # K = 0 with accumulate: untouched
+
+
+def test_leaf_v2_ldg_variant_parity():
+    """The experimental LDG-fed pair kernel (v2, NORTHUP_LEAF=3) computes the
+    same result as the default TMA-fed kernel, bit for bit."""
+    import ctypes
+    f = nu.lib().northup_debug_leaf_gemm
+    f.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                  ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                  ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                  ctypes.c_void_p]
+    dev = _dev()
+    for (M, N, K) in [(300, 520, 1000), (257, 132, 37 * 4)]:
+        A = nugen.fill(M, K, 19, 1)
+        B = nugen.fill(K, N, 19, 2)
+        Ad, Bd = torch.from_numpy(A).to(dev), torch.from_numpy(B).to(dev)
+        outs = []
+        for variant in (2, 3):
+            Cd = torch.full((M, N), float("nan"), device=dev)
+            assert f(Ad.data_ptr(), K, Bd.data_ptr(), N, Cd.data_ptr(), N, M, N, K, 0, 0, 2, 0, None,
+                     variant, None) == 0
+            torch.cuda.synchronize()
+            outs.append(Cd.cpu().numpy())
+        assert np.array_equal(outs[0], outs[1])
+        assert normwise(outs[0], A, B) <= TOL
