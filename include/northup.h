@@ -185,7 +185,10 @@ typedef struct {
   int collect_timing;   /* 1: record per-stage CUDA-event timings into the stats */
   int64_t a_panel_k;    /* FILE root only: A is stored K-panel-major (R15 preprocessing,
                            see northup_file_tile_kpanels) with this panel width; 0 = row-major */
-  int reserved[6];
+  int graph;            /* 1: capture each GPU's op list into a CUDA graph and replay it when the
+                           same GEMM (sizes, buffers, options) is called again — the recursion
+                           unfolded into a dependency graph (P:230 future work); HOST/HBM roots */
+  int reserved[5];
 } northup_gemm_opts;
 
 typedef struct {
@@ -204,6 +207,8 @@ typedef struct {
   int schedule;          /* schedule used */
   int num_gpus;          /* HBM siblings used */
   uint64_t hbm_peak_bytes; /* planned footprint at the HBM node of GPU 0 */
+  int graph_replayed;    /* 1 when the call replayed CUDA graphs captured by an earlier call */
+  int reserved_stat;
 } northup_stats;
 
 /* C = A.B (no alpha/beta; C overwritten — reading R3), A (M x K), B (K x N),

@@ -49,7 +49,7 @@ class GemmOpts(ctypes.Structure):
     _fields_ = [("schedule", ctypes.c_int), ("replicate_result", ctypes.c_int),
                 ("k_chunk", ctypes.c_int64), ("npass", ctypes.c_int), ("resident", ctypes.c_int),
                 ("collect_timing", ctypes.c_int), ("a_panel_k", ctypes.c_int64),
-                ("reserved", ctypes.c_int * 6)]
+                ("graph", ctypes.c_int), ("reserved", ctypes.c_int * 5)]
 
 
 class Stats(ctypes.Structure):
@@ -62,7 +62,8 @@ class Stats(ctypes.Structure):
                 ("copies", ctypes.c_int64), ("ops", ctypes.c_int64), ("bm", ctypes.c_int64),
                 ("bn", ctypes.c_int64), ("bk", ctypes.c_int64), ("tail_k", ctypes.c_int64),
                 ("strips", ctypes.c_int64), ("schedule", ctypes.c_int), ("num_gpus", ctypes.c_int),
-                ("hbm_peak_bytes", ctypes.c_uint64)]
+                ("hbm_peak_bytes", ctypes.c_uint64), ("graph_replayed", ctypes.c_int),
+                ("reserved_stat", ctypes.c_int)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -238,9 +239,10 @@ def partition_region(G: int, M: int, N: int, K: int, r: int) -> tuple[int, int, 
 
 def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 0,
               collect_timing: bool = False, replicate_result: bool = False,
-              a_panel_k: int = 0) -> GemmOpts:
+              a_panel_k: int = 0, graph: bool = False) -> GemmOpts:
     o = GemmOpts()
     o.a_panel_k = a_panel_k
+    o.graph = int(graph)
     o.schedule = schedule
     o.k_chunk = k_chunk
     o.npass = npass

@@ -153,12 +153,23 @@ static bool wait_flag(RunCtx& c, std::vector<char>& v, size_t i) {
   return v[i] != 0;
 }
 
-static int run_worker(RunCtx& c, int wi, double* busy) {
+static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_out = nullptr) {
   const Plan& P = *c.plan;
   WorkerState* w = worker_for_node(c.t, P.worker_node[wi]);
   if (!w) return fail(NU_ESTATE, "no worker state for node %d", P.worker_node[wi]);
   cudaError_t e = cudaSetDevice(w->device);
   if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+  cudaEvent_t fork = nullptr;
+  if (capture_out) {
+    // Stream capture: stream 0 starts the capture, the other streams join it
+    // through a fork event and are joined back at the end, so the graph holds
+    // every op with its cross-stream dependencies.
+    e = cudaStreamBeginCapture(w->streams[0], cudaStreamCaptureModeThreadLocal);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamBeginCapture");
+    cudaEventCreateWithFlags(&fork, cudaEventDisableTiming);
+    cudaEventRecord(fork, w->streams[0]);
+    for (int s = 1; s < S_NUM; ++s) cudaStreamWaitEvent(w->streams[s], fork, 0);
+  }
   const size_t nops = P.ops.size();
   while (w->events.size() < nops) {
     cudaEvent_t ev;
@@ -215,6 +226,26 @@ static int run_worker(RunCtx& c, int wi, double* busy) {
       if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
       mark(c, c.issued, i);
     }
+  }
+  if (capture_out) {
+    std::vector<cudaEvent_t> joins;
+    for (int s = 1; s < S_NUM; ++s) {
+      cudaEvent_t j;
+      cudaEventCreateWithFlags(&j, cudaEventDisableTiming);
+      cudaEventRecord(j, w->streams[s]);
+      cudaStreamWaitEvent(w->streams[0], j, 0);
+      joins.push_back(j);
+    }
+    cudaGraph_t g = nullptr;
+    e = cudaStreamEndCapture(w->streams[0], &g);
+    for (cudaEvent_t j : joins) cudaEventDestroy(j);
+    cudaEventDestroy(fork);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamEndCapture");
+    e = cudaGraphInstantiate(capture_out, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+    e = cudaGraphLaunch(*capture_out, w->streams[0]);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
   }
   for (cudaStream_t s : w->streams) {
     e = cudaStreamSynchronize(s);
@@ -311,6 +342,22 @@ static int run_io(RunCtx& c) {
   return 0;
 }
 
+// Key of a captured GEMM: everything the op list and its pointers depend on.
+static std::vector<int64_t> graph_key(const Plan& P, const std::vector<char*>& base,
+                                      const northup_gemm_opts* o) {
+  std::vector<int64_t> k = {P.M, P.N, P.K, P.kc, P.npass, o ? o->schedule : 0,
+                            static_cast<int64_t>(P.ops.size())};
+  for (char* b : base) k.push_back(reinterpret_cast<int64_t>(b));
+  return k;
+}
+
+void destroy_graphs(northup_tree_s* t) {
+  for (auto& g : t->graph_execs)
+    if (g) cudaGraphExecDestroy(static_cast<cudaGraphExec_t>(g));
+  t->graph_execs.clear();
+  t->graph_key.clear();
+}
+
 int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf_s* b,
                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st) {
   RunCtx ctx;
@@ -345,11 +392,37 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   ctx.io_done.assign(P.ops.size(), 0);
 
   const int W = P.num_workers;
+  // CUDA-graph mode: replay the captured op lists of an identical earlier call
+  const bool use_graph = o && o->graph && !has_io && !ctx.timing;
+  std::vector<int64_t> key;
+  if (use_graph) {
+    key = graph_key(P, ctx.base, o);
+    if (key == t->graph_key && static_cast<int>(t->graph_execs.size()) == W) {
+      for (int wi = 0; wi < W; ++wi) {
+        WorkerState* w = worker_for_node(t, P.worker_node[wi]);
+        cudaSetDevice(w->device);
+        cudaError_t e = cudaGraphLaunch(static_cast<cudaGraphExec_t>(t->graph_execs[wi]), w->streams[0]);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
+      }
+      for (int wi = 0; wi < W; ++wi) {
+        WorkerState* w = worker_for_node(t, P.worker_node[wi]);
+        cudaSetDevice(w->device);
+        cudaError_t e = cudaStreamSynchronize(w->streams[0]);
+        if (e != cudaSuccess) return cuda_fail(e, "graph synchronize");
+      }
+      if (st) st->graph_replayed = 1;
+      return 0;
+    }
+    destroy_graphs(t);
+    t->graph_execs.assign(W, nullptr);
+  }
   std::vector<int> rcs(W + 1, 0);
   std::vector<std::string> errs(W + 1);
   std::vector<std::vector<double>> busy(W, std::vector<double>(S_NUM, 0.0));
   auto worker_body = [&](int wi) {
-    rcs[wi] = run_worker(ctx, wi, busy[wi].data());
+    cudaGraphExec_t ge = nullptr;
+    rcs[wi] = run_worker(ctx, wi, busy[wi].data(), use_graph ? &ge : nullptr);
+    if (use_graph) t->graph_execs[wi] = ge;
     if (rcs[wi]) {
       errs[wi] = northup_last_error();
       ctx.abort = true;
@@ -373,7 +446,11 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     for (auto& x : th) x.join();
   }
   for (int wi = 0; wi <= W; ++wi)
-    if (rcs[wi]) return fail(rcs[wi], "%s %d: %s", wi < W ? "worker" : "I/O thread", wi, errs[wi].c_str());
+    if (rcs[wi]) {
+      if (use_graph) destroy_graphs(t);
+      return fail(rcs[wi], "%s %d: %s", wi < W ? "worker" : "I/O thread", wi, errs[wi].c_str());
+    }
+  if (use_graph) t->graph_key = key;
   if (st) {
     for (int wi = 0; wi < W; ++wi) {
       st->t_h2d_ms += busy[wi][S_H2D];

@@ -74,6 +74,8 @@ struct northup_tree_s {
   std::vector<WorkerState*> workers;   // one per HBM node (created at finalize)
   std::vector<void*> nccl_comms;       // ncclComm_t per HBM sibling (replicate_result)
   std::vector<std::array<float, 5>> timeline;   // last collect_timing run (debug)
+  std::vector<void*> graph_execs;      // cudaGraphExec_t per worker (opts->graph)
+  std::vector<int64_t> graph_key;      // the GEMM they were captured for
 };
 
 namespace nu {
@@ -128,6 +130,7 @@ int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_
 int finalize_workers(northup_tree_s* t);
 int gather_replicas(northup_tree_s* t, const Plan& P, northup_buf_s* C, northup_stats* st);
 void destroy_nccl(northup_tree_s* t);
+void destroy_graphs(northup_tree_s* t);
 void destroy_workers(northup_tree_s* t);
 
 }  // namespace nu

@@ -248,35 +248,47 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
     bns.push_back(v);
     if (v <= 256) break;
   }
-  // Prefer whole-region blocks (fewest H2D bytes), then the longest tail.
+  // Among the C-block shapes that fit (each with its longest fitting drain
+  // tail), pick the fewest H2D bytes: every block streams its A row strip and
+  // B column strip once, 4K(bm + bn) per block.  Ties: longer tail, then
+  // taller blocks (contiguous C rows in the root).
+  const int64_t long_tail = rup(want_tail * 8 / 5, x.kc);
+  const int64_t tails[] = {long_tail < K ? long_tail : std::min(K, want_tail), std::min(K, want_tail),
+                           std::min(K, want_tail / 2), std::min(K, x.kc), 0};
+  bool found = false;
+  S2Shape best{};
+  uint64_t best_h2d = 0;
+  int best_rank = 0;
   for (int64_t bn : bns) {
     for (int64_t bm : bms) {
-      // a tail longer than the break-even 2P/BW lets graded (shrinking) strips
-      // keep D2H behind compute down to a small last strip
-      const int64_t long_tail = rup(want_tail * 8 / 5, x.kc);
-      const int64_t tails[] = {long_tail < K ? long_tail : std::min(K, want_tail),
-                               std::min(K, want_tail), std::min(K, want_tail / 2),
-                               std::min(K, x.kc), 0};
+      const uint64_t h2d = static_cast<uint64_t>(cdiv(m, bm) * cdiv(n, bn)) * (bm + bn);
+      int rank = 0;
       for (int64_t tail : tails) {
-        if (tail < 0) continue;
+        ++rank;
         int64_t strips = std::max<int64_t>(1, std::min<int64_t>(16, cdiv(bm, 1024)));
-        int64_t sr = rup(cdiv(bm, strips), 128);
-        sr = std::min(sr, bm);
-        const uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr);
-        if (bytes <= cap) {
-          *out = S2Shape{bm, bn, bk, tail, sr, bytes};
-          return 0;
+        int64_t sr = std::min(rup(cdiv(bm, strips), 128), bm);
+        uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr);
+        int64_t use_bk = bk;
+        if (bytes > cap && tail == 0 && bk > x.kc && x.obk <= 0) {   // the minimum panel
+          use_bk = x.kc;
+          bytes = s2_bytes(bm, bn, use_bk, K, 0, 0);
         }
-      }
-      // also try the minimum panel
-      if (bk > x.kc && x.obk <= 0) {
-        const uint64_t bytes = s2_bytes(bm, bn, x.kc, K, 0, 0);
-        if (bytes <= cap) {
-          *out = S2Shape{bm, bn, x.kc, 0, 0, bytes};
-          return 0;
+        if (bytes > cap) continue;
+        const bool better = !found || h2d < best_h2d || (h2d == best_h2d && rank < best_rank) ||
+                            (h2d == best_h2d && rank == best_rank && bm > best.bm);
+        if (better) {
+          best = S2Shape{bm, bn, use_bk, tail, tail > 0 ? sr : 0, bytes};
+          best_h2d = h2d;
+          best_rank = rank;
+          found = true;
         }
+        break;   // longest fitting tail for this shape
       }
     }
+  }
+  if (found) {
+    *out = best;
+    return 0;
   }
   return fail(NU_ENOMEM, "HBM node %d capacity %llu B is below the minimum block", x.hbm_node,
               (unsigned long long)x.cap);

@@ -177,6 +177,7 @@ int northup_tree_destroy(northup_tree_t t) {
   if (!t) return fail(NU_EINVAL, "tree is NULL");
   while (!t->bufs.empty()) northup_release(t, t->bufs.back());
   destroy_nccl(t);
+  destroy_graphs(t);
   destroy_workers(t);
   for (Node& n : t->nodes) {
     if (n.arena_owned && n.arena) {
