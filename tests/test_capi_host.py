@@ -275,3 +275,39 @@ def test_file_tile_kpanels_round_trip(tmp_path):
     A.tofile(src)
     nu.file_tile_kpanels(str(src), str(dst), M, K, P)
     assert np.array_equal(np.fromfile(dst, dtype=np.float32), kpanels(A, P).astype(np.float32))
+
+
+# ----------------------------------------------------- randomised planner check
+from hypothesis import HealthCheck, given, settings, strategies as st
+
+
+@settings(max_examples=40, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(M=st.integers(1, 300), N=st.integers(1, 300), K=st.integers(1, 300),
+       G=st.sampled_from([1, 2, 3, 4]), cap_kib=st.sampled_from([0, 300, 800, 2000]),
+       kc=st.sampled_from([32, 64, 128]), sched=st.sampled_from([0, 1, 2]),
+       file_root=st.booleans(), panel=st.sampled_from([0, 32, 64]), seed=st.integers(0, 3))
+def test_random_plans_replay_exactly(M, N, K, G, cap_kib, kc, sched, file_root, panel, seed):
+    """Any tree shape / capacity / schedule the planner accepts yields an op
+    list whose dependency-respecting replay computes A.B exactly; capacity
+    errors are NU_ENOMEM, nothing else."""
+    cap = cap_kib * 1024
+    if file_root:
+        t = file_tree(G, cap)
+        opts = nu.make_opts(k_chunk=kc, a_panel_k=panel)
+    else:
+        t, _ = nu.host_tree(G, cap)
+        opts = nu.make_opts(schedule=sched, k_chunk=kc)
+    try:
+        p = t.plan(M, N, K, opts)
+    except nu.NorthupError as e:
+        assert e.code == nu.NU_ENOMEM
+        t.destroy()
+        return
+    A = nugen.fill(M, K, seed, 1, "int")
+    B = nugen.fill(K, N, seed, 2, "int")
+    lay = kpanels(A, panel) if (file_root and panel) else None
+    C = simulate(p, A, B, M, N, K, rng=random.Random(seed), a_layout=lay)
+    assert np.array_equal(C, A.astype(np.float64) @ B.astype(np.float64))
+    if cap:
+        assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
+    t.destroy()
