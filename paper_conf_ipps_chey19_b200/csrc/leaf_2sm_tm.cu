@@ -1,0 +1,457 @@
+// Leaf kernel v3: the v1.2 CTA pair (leaf_2sm.cu, R21 arithmetic: one tf32
+// MMA for hi.hi on the raw tile, one bf16 MMA per k8 step for both cross
+// terms), with the shared-memory traffic of the bf16 A' operand moved into
+// tensor memory.
+//
+// v1.2 is bound by shared memory (~160 KiB per CTA per stage
+// against ~128 B/clk).  Here the split warps write A' = [bf16(hi_a) |
+// bf16(lo_a)] straight into TMEM with tcgen05.st and the cross-term MMA reads
+// A from TMEM ("TS" form), which removes the A' store and the A' operand
+// fetch (32 KiB per stage) from shared memory.  TMEM then holds one 256-column
+// accumulator plus an LS-deep A' ring (32 columns per stage), so the
+// accumulator is no longer double-buffered: the epilogue drains it quickly
+// (tcgen05.ld -> swizzled staging box -> TMA store, or TMA reduce-add into C
+// when accumulating) and releases TMEM before its global writes land.
+//
+// Numerics: the same products in the same MMA order as v1.2 and the same
+// per-chunk fp32 C += acc (an RN add, done by TMA's reduce in L2), so results
+// are bitwise those of v1.2 (tests/test_gpu_leaf.py).
+//
+// TMEM map (512 columns per CTA): acc [0, 256); A' slot j [256 + 32 j, +32).
+//   A' row r (lane r of this CTA's half), column 256 + 32 j + c holds the
+//   virtual-k pair (2c, 2c+1): virtual chunk 2g = bf16(hi) of real k 8g..8g+7,
+//   2g+1 = bf16(lo); B' in shared memory pairs them with lo_b / hi_b.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "leaf_2sm_common.cuh"
+#include "leaf_common.cuh"
+#include "northup_internal.h"
+
+namespace nu {
+namespace leaf {
+namespace sm4 {
+
+using sm2::cluster_ctarank;
+using sm2::cluster_sync;
+using sm2::idesc_bf16;
+using sm2::lds128;
+using sm2::mapa;
+using sm2::mbar_arrive_cluster;
+using sm2::mbar_wait_cluster;
+using sm2::named_bar;
+using sm2::pack_bf16;
+using sm2::sts128;
+using sm2::trunc13;
+using sm2::umma_commit_pair;
+using sm2::umma_tf32_2sm;
+
+constexpr int BM = 256;
+constexpr int BN = 256;
+constexpr int BM_CTA = 128;
+constexpr int BN_CTA = 128;
+#ifndef NU_LEAF3_RS
+#define NU_LEAF3_RS 4
+#endif
+#ifndef NU_LEAF3_LS
+#define NU_LEAF3_LS 3
+#endif
+constexpr int RS = NU_LEAF3_RS;                    // raw (TMA) ring depth
+constexpr int LS = NU_LEAF3_LS;                    // split ring depth (B' smem + A' TMEM)
+static_assert(LS <= 8, "A' ring must fit in TMEM columns [256, 512)");
+constexpr int A_BYTES = BM_CTA * BK * 4;           // 16 KiB
+constexpr int B_BYTES = BN_CTA * BK * 4;           // 16 KiB
+constexpr int TMA_BYTES = A_BYTES + B_BYTES;
+constexpr int XB_BYTES = 2 * BK * BN_CTA * 2;      // B' bf16: 64 virtual k x 128 n = 16 KiB
+constexpr int XFORM_WARPS = 8;                     // warps 2..9: two per TMEM lane quarter
+constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
+constexpr int EPI_WARP0 = 2 + XFORM_WARPS;         // warps 10..13
+constexpr int EPI_THREADS = 128;
+constexpr int NUM_THREADS = 32 * (EPI_WARP0 + 4);
+constexpr int EPI_BUFS = 2;                        // staging boxes per epilogue warp
+constexpr int BOX_BYTES = 32 * 32 * 4;             // 32 rows x 32 cols fp32, SW128
+constexpr int EPI_BYTES = 4 * EPI_BUFS * BOX_BYTES;
+constexpr int TMEM_COLS = 512;
+constexpr int TM_XA = 256;                         // first A' column
+constexpr int BAR_BYTES = 256;
+constexpr int SMEM_BYTES = RS * TMA_BYTES + LS * XB_BYTES + EPI_BYTES + BAR_BYTES + 1024;
+static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
+
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+      "{%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, %16};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
+      "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+
+__device__ __forceinline__ void tmem_wait_st() {
+  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+
+// D[tmem] (+)= A[tmem] . B[smem], kind::f16 (bf16 in, fp32 accumulate), pair MMA.
+__device__ __forceinline__ void umma_bf16_2sm_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db,
+                                                 uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(src), "r"(c0), "r"(c1)
+               : "memory");
+}
+
+__device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* map, uint32_t src, int c0,
+                                                  int c1) {
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(map)),
+      "r"(src), "r"(c0), "r"(c1)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
+    leaf_gemm_2sm_tm_kernel(const __grid_constant__ CUtensorMap tmA,
+                            const __grid_constant__ CUtensorMap tmB,
+                            const __grid_constant__ CUtensorMap tmC, const Params p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint8_t* raw_base = smem;                                  // RS x (A 16 KiB | B 16 KiB)
+  uint8_t* xb_base = smem + RS * TMA_BYTES;                  // LS x B' 16 KiB
+  uint8_t* epi_base = xb_base + LS * XB_BYTES;               // 4 warps x EPI_BUFS boxes
+  uint8_t* bars = epi_base + EPI_BYTES;
+  const uint32_t bar_full = smem_u32(bars);
+  const uint32_t bar_rempty = bar_full + 8 * RS;
+  const uint32_t bar_rawfull = bar_rempty + 8 * RS;
+  const uint32_t bar_xform = bar_rawfull + 8 * RS;
+  const uint32_t bar_lempty = bar_xform + 8 * LS;
+  const uint32_t bar_tfull = bar_lempty + 8 * LS;
+  const uint32_t bar_tempty = bar_tfull + 8;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (3 * RS + 2 * LS + 2));
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+
+  if (threadIdx.x == 0) {
+    prefetch_tmap(&tmA);
+    prefetch_tmap(&tmB);
+    prefetch_tmap(&tmC);
+    for (int s = 0; s < RS; ++s) {
+      mbar_init(bar_full + 8 * s, 1);
+      mbar_init(bar_rempty + 8 * s, 1);
+      mbar_init(bar_rawfull + 8 * s, 2);
+    }
+    for (int j = 0; j < LS; ++j) {
+      mbar_init(bar_xform + 8 * j, 2);
+      mbar_init(bar_lempty + 8 * j, 1);
+    }
+    mbar_init(bar_tfull, 1);
+    mbar_init(bar_tempty, 2 * EPI_THREADS);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  const int cid = blockIdx.x >> 1;
+  const int nclusters = gridDim.x >> 1;
+  const int num_tiles = p.tiles_m * p.tiles_n;
+  const int nkb = (p.K + BK - 1) / BK;
+  const int nchunks = (nkb + p.kb_per_chunk - 1) / p.kb_per_chunk;
+
+  if (warp == 0) {
+    // ------------------------------------------------------ TMA producer (own half)
+    if (lane == 0) {
+      uint32_t it = 0;
+      for (int t = cid; t < num_tiles; t += nclusters) {
+        int mb, nb;
+        tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
+        const int row0 = mb * BM + rank * BM_CTA;
+        const int col0 = nb * BN + rank * BN_CTA;
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const uint32_t s = it % RS, use = it / RS;
+          mbar_wait(bar_rempty + 8 * s, (use & 1) ^ 1);
+          const uint32_t full = bar_full + 8 * s;
+          mbar_arrive_expect_tx(full, TMA_BYTES);
+          const uint32_t sa = smem_u32(raw_base + s * TMA_BYTES);
+          const uint32_t sb = sa + A_BYTES;
+          tma_load_2d(sa, &tmA, full, kb * BK, row0);
+#pragma unroll
+          for (int c = 0; c < BN_CTA / B_CHUNK; ++c)
+            tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------ MMA issuer (leader CTA only)
+    if (leader && lane == 0) {
+      const uint32_t idesc = idesc_tf32(BM, BN, 1u);
+      const uint32_t idesc_bf = idesc_bf16(BM, BN);
+      uint32_t it = 0, chunk_it = 0;
+      long long w_xf = 0, w_te = 0, t_beg = clock64();   // profile mode (p.dbg)
+      for (int t = cid; t < num_tiles; t += nclusters) {
+        for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
+          long long c0 = clock64();
+          mbar_wait_cluster(bar_tempty, (chunk_it & 1) ^ 1);
+          w_te += clock64() - c0;
+          tc_fence_after();
+          const int kb0 = ch * p.kb_per_chunk;
+          const int kb1 = min(nkb, kb0 + p.kb_per_chunk);
+          for (int kb = kb0; kb < kb1; ++kb, ++it) {
+            const uint32_t s = it % RS, suse = it / RS;
+            const uint32_t j = it % LS, juse = it / LS;
+            const uint32_t a_hi = smem_u32(raw_base + s * TMA_BYTES);
+            const uint32_t b_hi = a_hi + A_BYTES;
+            const uint32_t b_x = smem_u32(xb_base + j * XB_BYTES);
+            const uint32_t a_x = tmem_base + TM_XA + 32 * j;
+            c0 = clock64();
+            mbar_wait_cluster(bar_rawfull + 8 * s, suse & 1);
+            w_xf += clock64() - c0;
+            tc_fence_after();
+#pragma unroll
+            for (int k = 0; k < BK / UMMA_K; ++k)
+              umma_tf32_2sm(tmem_base, umma_desc(a_hi + k * 32, 16, 1024),
+                            umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B),
+                            idesc, (kb == kb0 && k == 0) ? 0u : 1u);
+            c0 = clock64();
+            mbar_wait_cluster(bar_xform + 8 * j, juse & 1);
+            w_xf += clock64() - c0;
+            tc_fence_after();
+#pragma unroll
+            for (int k = 0; k < BK / UMMA_K; ++k)
+              umma_bf16_2sm_ts(tmem_base, a_x + 8 * k, umma_desc(b_x + k * 2048, 8192, 1024),
+                               idesc_bf, 1u);
+            umma_commit_pair(bar_rempty + 8 * s);
+            umma_commit_pair(bar_lempty + 8 * j);
+          }
+          umma_commit_pair(bar_tfull);
+        }
+      }
+      if (p.dbg) {
+        float* d = p.dbg + 8 * cid;
+        d[0] = static_cast<float>(clock64() - t_beg);
+        d[1] = static_cast<float>(w_xf);
+        d[2] = static_cast<float>(w_te);
+        d[3] = static_cast<float>(it);
+      }
+    }
+  } else if (warp < EPI_WARP0) {
+    // ---------------------------------------------------- split (own half)
+    const int tid = threadIdx.x - 64;
+    const int q = warp & 3;                 // TMEM lane quarter this warp may access
+    const int h = (warp - 2) >> 2;          // which 16 of the stage's 32 k
+    const int r = 32 * q + lane;            // A row of this CTA's half
+    const uint32_t xform_leader0 = mapa(bar_xform, 0);
+    const uint32_t rawfull_leader0 = mapa(bar_rawfull, 0);
+    const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + TM_XA + 16 * h;
+    uint32_t it = 0;
+    long long w_full = 0, w_lem = 0;
+    for (int t = cid; t < num_tiles; t += nclusters) {
+      for (int kb = 0; kb < nkb; ++kb, ++it) {
+        const uint32_t s = it % RS, use = it / RS;
+        const uint32_t j = it % LS, juse = it / LS;
+        long long c0 = clock64();
+        mbar_wait(bar_full + 8 * s, use & 1);
+        if (tid == 0) mbar_arrive_cluster(rawfull_leader0 + 8 * s);
+        long long c1 = clock64();
+        mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
+        tc_fence_after();
+        w_full += c1 - c0;
+        w_lem += clock64() - c1;
+        const uint32_t raw = smem_u32(raw_base + s * TMA_BYTES);
+        // A' row r, real k 16h..16h+15 -> TMEM columns 16h..16h+15 of slot j
+        {
+          const uint32_t rowa = raw + r * 128;
+          const int sw = r & 7;
+          uint32_t v[16];
+#pragma unroll
+          for (int g = 0; g < 2; ++g) {
+            const uint4 x0 = lds128(rowa + (((4 * h + 2 * g) ^ sw) << 4));
+            const uint4 x1 = lds128(rowa + (((4 * h + 2 * g + 1) ^ sw) << 4));
+            const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
+                                __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
+                                __uint_as_float(x1.z), __uint_as_float(x1.w)};
+            float hi[8], lo[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              hi[e] = trunc13(f[e]);
+              lo[e] = f[e] - hi[e];
+            }
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              v[8 * g + e] = pack_bf16(hi[2 * e], hi[2 * e + 1]);
+              v[8 * g + 4 + e] = pack_bf16(lo[2 * e], lo[2 * e + 1]);
+            }
+          }
+          tmem_st16(t_row + 32 * j, v);
+        }
+        // B' (MN-major SW128 bf16, 64 virtual k x 128 n): as leaf_2sm.cu
+        const uint32_t xb = smem_u32(xb_base + j * XB_BYTES);
+#pragma unroll
+        for (int u = 0; u < 512 / XFORM_THREADS; ++u) {
+          const int item = tid + u * XFORM_THREADS;
+          const int k = item >> 4, n0 = (item & 15) * 8;
+          const int nn = n0 & 31;
+          const uint32_t src = raw + A_BYTES + (n0 >> 5) * B_CHUNK_BYTES + k * 128 +
+                               (((nn >> 3) ^ (k & 3)) << 5);
+          const uint32_t h1 = (threadIdx.x >> 2) & 1;
+          const uint4 y0 = lds128(src + 16 * h1), y1 = lds128(src + 16 * (h1 ^ 1));
+          const uint4 x0 = h1 ? y1 : y0, x1 = h1 ? y0 : y1;
+          const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
+                              __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
+                              __uint_as_float(x1.z), __uint_as_float(x1.w)};
+          float hi[8], lo[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            hi[e] = trunc13(f[e]);
+            lo[e] = f[e] - hi[e];
+          }
+          const int vlo = 16 * (k >> 3) + (k & 7), vhi = vlo + 8;
+          const int c = (n0 & 63) >> 3;
+          const uint32_t base = xb + (n0 >> 6) * 8192;
+          sts128(base + (vlo >> 3) * 1024 + (vlo & 7) * 128 + ((c ^ (vlo & 7)) << 4),
+                 make_uint4(pack_bf16(lo[0], lo[1]), pack_bf16(lo[2], lo[3]),
+                            pack_bf16(lo[4], lo[5]), pack_bf16(lo[6], lo[7])));
+          sts128(base + (vhi >> 3) * 1024 + (vhi & 7) * 128 + ((c ^ (vhi & 7)) << 4),
+                 make_uint4(pack_bf16(hi[0], hi[1]), pack_bf16(hi[2], hi[3]),
+                            pack_bf16(hi[4], hi[5]), pack_bf16(hi[6], hi[7])));
+        }
+        tmem_wait_st();
+        fence_proxy_async_smem();
+        tc_fence_before();
+        named_bar(1, XFORM_THREADS);
+        if (tid == 0) mbar_arrive_cluster(xform_leader0 + 8 * j);
+      }
+    }
+    if (p.dbg && tid == 0) {
+      float* d = p.dbg + 8 * cid + 4 + 2 * rank;
+      d[0] = static_cast<float>(w_full);
+      d[1] = static_cast<float>(w_lem);
+    }
+  } else {
+    // ------------------------------------------------------ epilogue (own rows)
+    const int q = warp & 3;
+    const uint32_t tempty_leader0 = mapa(bar_tempty, 0);
+    const uint32_t stage0 = smem_u32(epi_base + (warp - EPI_WARP0) * EPI_BUFS * BOX_BYTES);
+    const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16);
+    uint32_t chunk_it = 0, box_it = 0;
+    for (int t = cid; t < num_tiles; t += nclusters) {
+      int mb, nb;
+      tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
+      const int row0 = mb * BM + rank * BM_CTA + 32 * q;
+      for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
+        mbar_wait(bar_tfull, chunk_it & 1);
+        tc_fence_after();
+        const bool add = (ch > 0) || p.accumulate;
+#pragma unroll 1
+        for (int c = 0; c < BN / 32; ++c, ++box_it) {
+          uint32_t v[32];
+          __syncwarp();
+          tmem_ld32(t_row + c * 32, v);
+          if (c == BN / 32 - 1) {
+            // the accumulator is in registers: hand TMEM back to the MMA issuer
+            tc_fence_before();
+            mbar_arrive_cluster(tempty_leader0);
+          }
+          const uint32_t box = stage0 + (box_it % EPI_BUFS) * BOX_BYTES;
+          if (lane == 0) bulk_wait_read<EPI_BUFS - 1>();   // the box's last store has read it
+          __syncwarp();
+          const uint32_t rowp = box + lane * 128;
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            sts128(rowp + ((i ^ (lane & 7)) << 4),
+                   make_uint4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]));
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) {
+            const int col = nb * BN + c * 32;
+            if (add) tma_reduce_add_2d(&tmC, box, col, row0);
+            else tma_store_2d(&tmC, box, col, row0);
+            bulk_commit();
+          }
+        }
+      }
+    }
+    if (lane == 0) bulk_wait_all();
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "n"(TMEM_COLS)
+                 : "memory");
+  }
+}
+
+}  // namespace sm4
+
+// v3 implements the R21 (npass 2) arithmetic with B row-major and a C that
+// TMA can address (16-B aligned, ldc % 4 == 0); other calls go to v1.2.
+bool launch_sm4_ok(const LaunchArgs& a) {
+  return a.p.npass == 2 && !a.p.b_kmajor && a.p.vec_ok;
+}
+
+int launch_sm4(LaunchArgs& a) {
+  using namespace sm4;
+  int rc;
+  CUtensorMap tmA, tmB, tmC;
+  Params& p = a.p;
+  if ((rc = encode_2d(&tmA, a.A, p.K, p.M, a.lda, BK, BM_CTA))) return rc;
+  if ((rc = encode_2d(&tmB, a.B, p.N, p.K, a.ldb, B_CHUNK, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)))
+    return rc;
+  if ((rc = encode_2d(&tmC, p.C, p.N, p.M, p.ldc, 32, 32))) return rc;
+  p.tiles_m = (p.M + BM - 1) / BM;
+  p.tiles_n = (p.N + BN - 1) / BN;
+  static std::atomic<int> configured[kMaxDevices];
+  if (!configured[a.dev].load()) {
+    cudaError_t e = cudaFuncSetAttribute(leaf_gemm_2sm_tm_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    if (e != cudaSuccess) return fail(NU_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+    configured[a.dev].store(1);
+  }
+  const int tiles = p.tiles_m * p.tiles_n;
+  const int pairs = a.sms / 2;
+  const int grid = 2 * (tiles < pairs ? tiles : pairs);
+  leaf_gemm_2sm_tm_kernel<<<grid, NUM_THREADS, SMEM_BYTES, a.stream>>>(tmA, tmB, tmC, p);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : fail(NU_ECUDA, "leaf (2sm tmem) launch: %s", cudaGetErrorString(e));
+}
+
+}  // namespace leaf
+}  // namespace nu

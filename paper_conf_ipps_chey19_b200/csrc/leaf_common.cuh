@@ -196,6 +196,8 @@ int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t oute
 int launch_sm1(LaunchArgs& a);   // v0: 1-CTA 128 x 256 tile
 int launch_sm2(LaunchArgs& a);   // v1: CTA pair (cta_group::2) 256 x 256 tile, TMA-fed
 int launch_sm3(LaunchArgs& a);   // v2: CTA pair, split warps load global memory directly
+int launch_sm4(LaunchArgs& a);   // v3: CTA pair, A' operand in TMEM, TMA-store epilogue
+bool launch_sm4_ok(const LaunchArgs& a);
 
 }  // namespace leaf
 }  // namespace nu

@@ -52,7 +52,8 @@ bool leaf_tma_legal(const void* p, int64_t ld) {
   return (reinterpret_cast<uintptr_t>(p) % 16 == 0) && (ld % 4 == 0) && ld > 0;
 }
 
-// variant: 0 = default (NORTHUP_LEAF env may override: "1sm" / "2sm"), 1 = 1sm, 2 = 2sm.
+// variant: 0 = default (env NORTHUP_LEAF=1..4 may override), 1 = v0 (1 CTA), 2 = v1.2 (pair),
+// 3 = v2 (pair, LDG-fed), 4 = v3 (pair, A' in TMEM).
 int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                          int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                          int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream) {
@@ -116,7 +117,7 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
     static int env_variant = -1;
     if (env_variant < 0) {
       const char* v = getenv("NORTHUP_LEAF");
-      env_variant = (v && v[0] >= '1' && v[0] <= '3') ? v[0] - '0' : kDefaultLeafVariant;
+      env_variant = (v && v[0] >= '1' && v[0] <= '4') ? v[0] - '0' : kDefaultLeafVariant;
     }
     variant = env_variant;
   }
@@ -144,7 +145,8 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
     b.p.lda = lda;
     b.p.B = b.B;
     b.p.ldb = ldb;
-    rc = variant == 1 ? launch_sm1(b) : variant == 3 ? launch_sm3(b) : launch_sm2(b);
+    if (variant == 4 && !launch_sm4_ok(b)) variant = 2;
+    rc = variant == 1 ? launch_sm1(b) : variant == 3 ? launch_sm3(b) : variant == 4 ? launch_sm4(b) : launch_sm2(b);
   }
   return rc;
 }

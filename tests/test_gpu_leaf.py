@@ -194,3 +194,55 @@ def test_leaf_v2_ldg_variant_parity():
             outs.append(Cd.cpu().numpy())
         assert np.array_equal(outs[0], outs[1])
         assert normwise(outs[0], A, B) <= TOL
+
+
+def _debug_leaf(Ad, Bd, Cd, M, N, K, variant, accumulate=0, kc=0, npass=2):
+    import ctypes
+    f = nu.lib().northup_debug_leaf_gemm
+    f.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                  ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                  ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                  ctypes.c_void_p]
+    rc = f(Ad.data_ptr(), Ad.stride(0), Bd.data_ptr(), Bd.stride(0), Cd.data_ptr(), Cd.stride(0),
+           M, N, K, accumulate, kc, npass, 0, None, variant, None)
+    assert rc == 0
+    torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("M,N,K,kc", [(300, 520, 1000, 0), (257, 132, 148, 0), (512, 512, 4096, 1024),
+                                      (1, 4, 8, 0), (1000, 1000, 999, 256), (2048, 2304, 2048, 0)])
+def test_leaf_v3_tmem_variant_parity(M, N, K, kc):
+    """v3 (A' operand in TMEM, TMA store / reduce-add epilogue, NORTHUP_LEAF=4)
+    computes the same products in the same order as v1.2: bitwise equal, on
+    C = A.B and on C += A.B over several K panels."""
+    dev = _dev()
+    A = nugen.fill(M, K, 20, 1)
+    B = nugen.fill(K, N, 20, 2)
+    C0 = torch.from_numpy(nugen.fill(M, N, 20, 3)).to(dev)
+    Ad, Bd = torch.from_numpy(A).to(dev), torch.from_numpy(B).to(dev)
+    for acc in (0, 1):
+        outs = []
+        for variant in (2, 4):
+            Cd = C0.clone() if acc else torch.full((M, N), float("nan"), device=dev)
+            _debug_leaf(Ad, Bd, Cd, M, N, K, variant, accumulate=acc, kc=kc)
+            outs.append(Cd.cpu().numpy())
+        assert np.array_equal(outs[0], outs[1]), (acc, np.argwhere(outs[0] != outs[1])[:5])
+    ref = oracle.gemm(A, B) + C0.cpu().numpy().astype(np.float64)
+    assert normwise(outs[1], A, B, ref=ref) <= TOL
+
+
+def test_leaf_v3_integer_exact_and_clipped_edges():
+    """Integer inputs: exact vs the oracle; C columns beyond N (ldc > N) and
+    rows beyond M stay untouched by the TMA-store epilogue."""
+    dev = _dev()
+    M, N, K = 261, 300, 2100
+    A = nugen.fill(M, K, 21, 1, "int")
+    B = nugen.fill(K, N, 21, 2, "int")
+    Ad = torch.zeros((M, 2104), device=dev)
+    Ad[:, :K] = torch.from_numpy(A)
+    Bd = torch.from_numpy(B).to(dev)
+    big = torch.full((M + 3, 308), float("nan"), device=dev)
+    _debug_leaf(Ad[:, :K], Bd, big[:M, :N], M, N, K, 4)
+    out = big.cpu().numpy()
+    assert np.array_equal(out[:M, :N].astype(np.float64), oracle.gemm(A, B))
+    assert np.isnan(out[:M, N:]).all() and np.isnan(out[M:]).all()
