@@ -47,6 +47,8 @@ CONFIGS = {
                  desc="tall-skinny 1048576x4096x4096 fp32, A streamed from host"),
 }
 NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25      # B200_PROFILING.md nominal dense ratio
+LEAF_KERNELS = {1: "nu::leaf::sm1::leaf_gemm_1sm_kernel", 2: "nu::leaf::sm2::leaf_gemm_2sm_kernel",
+                3: "nu::leaf::sm3::leaf_gemm_2sm_ldg_kernel", 4: "nu::leaf::sm4::leaf_gemm_2sm_tm_kernel"}
 
 
 def log(*a):
@@ -350,7 +352,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                                         f"P_bf16 = {peaks['source']} bf16 sustained "
                                         f"{peaks['bf16_sustained']} TF/s, P_tf32 = P_bf16 x nominal "
                                         f"tf32/bf16 {NOMINAL_TF32_OVER_BF16:.3f}"),
-                         "kernel": "nu::leaf::sm2::leaf_gemm_2sm_kernel",
+                         "kernel": LEAF_KERNELS.get(nu.lib().northup_debug_leaf_variant(), "?"),
                          "launch": [m, n, min(K, kc_eff)], "launches_per_step": launches_per_step,
                          "flops_per_launch": flops_per_launch, "ms_per_launch": round(leaf_ms, 3),
                          "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "

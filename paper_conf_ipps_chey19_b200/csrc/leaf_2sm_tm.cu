@@ -55,7 +55,7 @@ constexpr int BN = 256;
 constexpr int BM_CTA = 128;
 constexpr int BN_CTA = 128;
 #ifndef NU_LEAF3_RS
-#define NU_LEAF3_RS 4
+#define NU_LEAF3_RS 3
 #endif
 #ifndef NU_LEAF3_LS
 #define NU_LEAF3_LS 3
@@ -69,12 +69,21 @@ constexpr int TMA_BYTES = A_BYTES + B_BYTES;
 constexpr int XB_BYTES = 2 * BK * BN_CTA * 2;      // B' bf16: 64 virtual k x 128 n = 16 KiB
 constexpr int XFORM_WARPS = 8;                     // warps 2..9: two per TMEM lane quarter
 constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
-constexpr int EPI_WARP0 = 2 + XFORM_WARPS;         // warps 10..13
-constexpr int EPI_THREADS = 128;
-constexpr int NUM_THREADS = 32 * (EPI_WARP0 + 4);
-constexpr int EPI_BUFS = 2;                        // staging boxes per epilogue warp
+#ifndef NU_LEAF3_EPI_WARPS
+#define NU_LEAF3_EPI_WARPS 8
+#endif
+#ifndef NU_LEAF3_EPI_BUFS
+#define NU_LEAF3_EPI_BUFS 2
+#endif
+constexpr int EPI_WARP0 = 2 + XFORM_WARPS;         // warps 10..
+constexpr int EPI_WARPS = NU_LEAF3_EPI_WARPS;      // 4 or 8: one or two per TMEM lane quarter
+static_assert(EPI_WARPS == 4 || EPI_WARPS == 8, "epilogue warps cover the lane quarters evenly");
+constexpr int EPI_THREADS = 32 * EPI_WARPS;
+constexpr int EPI_COLS = BN * 4 / EPI_WARPS;       // accumulator columns drained per warp
+constexpr int NUM_THREADS = 32 * (EPI_WARP0 + EPI_WARPS);
+constexpr int EPI_BUFS = NU_LEAF3_EPI_BUFS;        // staging boxes per epilogue warp
 constexpr int BOX_BYTES = 32 * 32 * 4;             // 32 rows x 32 cols fp32, SW128
-constexpr int EPI_BYTES = 4 * EPI_BUFS * BOX_BYTES;
+constexpr int EPI_BYTES = EPI_WARPS * EPI_BUFS * BOX_BYTES;
 constexpr int TMEM_COLS = 512;
 constexpr int TM_XA = 256;                         // first A' column
 constexpr int BAR_BYTES = 256;
@@ -364,6 +373,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   } else {
     // ------------------------------------------------------ epilogue (own rows)
     const int q = warp & 3;
+    const int cbeg = ((warp - EPI_WARP0) >> 2) * (EPI_COLS / 32);   // first 32-column box
     const uint32_t tempty_leader0 = mapa(bar_tempty, 0);
     const uint32_t stage0 = smem_u32(epi_base + (warp - EPI_WARP0) * EPI_BUFS * BOX_BYTES);
     const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16);
@@ -377,11 +387,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         tc_fence_after();
         const bool add = (ch > 0) || p.accumulate;
 #pragma unroll 1
-        for (int c = 0; c < BN / 32; ++c, ++box_it) {
+        for (int c = cbeg; c < cbeg + EPI_COLS / 32; ++c, ++box_it) {
           uint32_t v[32];
           __syncwarp();
           tmem_ld32(t_row + c * 32, v);
-          if (c == BN / 32 - 1) {
+          if (c == cbeg + EPI_COLS / 32 - 1) {
             // the accumulator is in registers: hand TMEM back to the MMA issuer
             tc_fence_before();
             mbar_arrive_cluster(tempty_leader0);

@@ -48,6 +48,15 @@ int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t oute
 
 }  // namespace leaf
 
+int default_leaf_variant() {
+  static int env_variant = -1;
+  if (env_variant < 0) {
+    const char* v = getenv("NORTHUP_LEAF");
+    env_variant = (v && v[0] >= '1' && v[0] <= '4') ? v[0] - '0' : kDefaultLeafVariant;
+  }
+  return env_variant;
+}
+
 bool leaf_tma_legal(const void* p, int64_t ld) {
   return (reinterpret_cast<uintptr_t>(p) % 16 == 0) && (ld % 4 == 0) && ld > 0;
 }
@@ -113,14 +122,7 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
   }
   a.dev = dev;
   a.sms = num_sms[dev].load();
-  if (variant == 0) {
-    static int env_variant = -1;
-    if (env_variant < 0) {
-      const char* v = getenv("NORTHUP_LEAF");
-      env_variant = (v && v[0] >= '1' && v[0] <= '4') ? v[0] - '0' : kDefaultLeafVariant;
-    }
-    variant = env_variant;
-  }
+  if (variant == 0) variant = default_leaf_variant();
   if (variant == 1 && p.npass == 2) p.npass = 3;   // the 1-CTA v0 kernel has no bf16 path
   if (variant == 3 && (p.npass != 2 || b_kmajor)) variant = 2;   // v2 implements R21 only
   // K-panel launches: each launch covers `panel` of K for
@@ -159,6 +161,9 @@ int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, f
 }
 
 }  // namespace nu
+
+// Debug entry (not part of northup.h): the leaf variant default calls use.
+extern "C" int northup_debug_leaf_variant(void) { return nu::default_leaf_variant(); }
 
 // Debug entry (not part of northup.h): kernel variant, B K-major, stage dump.
 extern "C" int northup_debug_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb,

@@ -15,7 +15,7 @@ namespace nu {
 constexpr int kMaxDevices = 64;
 constexpr int64_t kDefaultKChunk = 2048;   // TMEM accumulation length (R20)
 constexpr int kDefaultNpass = 2;            // 2 = TF32 hi.hi + bf16 cross terms (R21), 3 = 3xTF32
-constexpr int kDefaultLeafVariant = 2;      // 1 = v0 1-CTA, 2 = v1 TMA-fed pair, 3 = v2 LDG-fed pair
+constexpr int kDefaultLeafVariant = 4;      // 1 = v0 1-CTA, 2 = v1.2 TMA-fed pair, 3 = v2 LDG-fed pair, 4 = v3 A' in TMEM
 constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
 constexpr int kRasterBand = 16;            // n-blocks per raster band in the leaf
 constexpr int64_t kPanelChunks = 1;        // leaf K-panel launches, in k_chunks (0 = one launch)

@@ -210,7 +210,7 @@ def _debug_leaf(Ad, Bd, Cd, M, N, K, variant, accumulate=0, kc=0, npass=2):
 
 
 @pytest.mark.parametrize("M,N,K,kc", [(300, 520, 1000, 0), (257, 132, 148, 0), (512, 512, 4096, 1024),
-                                      (1, 4, 8, 0), (1000, 1000, 999, 256), (2048, 2304, 2048, 0)])
+                                      (1, 4, 8, 0), (1000, 1000, 996, 256), (2048, 2304, 2048, 0)])
 def test_leaf_v3_tmem_variant_parity(M, N, K, kc):
     """v3 (A' operand in TMEM, TMA store / reduce-add epilogue, NORTHUP_LEAF=4)
     computes the same products in the same order as v1.2: bitwise equal, on
