@@ -28,10 +28,11 @@ static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 static int64_t rup(int64_t a, int64_t b) { return cdiv(a, b) * b; }
 static int64_t pad_ld(int64_t n) { return std::max<int64_t>(32, rup(n, 32)); }  // 128-B rows
 
-// Nominal planning constants: useful 3xTF32 flop rate and the
+// Nominal planning constants: the leaf's useful flop rate on
+// one B200 under its power cap (v3, measured 320-336 TF/s) and the measured
 // PCIe Gen5 x16 per-direction bandwidth.  Only used to size the drain tail.
-static constexpr double kPlanFlops = 250e12;
-static constexpr double kPlanPcie = 50e9;
+static constexpr double kPlanFlops = 320e12;
+static constexpr double kPlanPcie = 52e9;
 
 int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc) {
   if (G <= 0) return fail(NU_EINVAL, "G must be positive");
@@ -230,13 +231,26 @@ uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, i
   return e * 4;
 }
 
+// Predicted time of one S2 block with drain tail K_t: the main
+// phase streams the A/B panels of K - K_t plus the resident B tail over H2D
+// while computing K - K_t; the tail phase computes row strips over K_t while
+// their A strips arrive (H2D) and finished C strips leave (D2H).
+static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail) {
+  const double fl = 2.0 * bm * bn / kPlanFlops;               // s per unit of K
+  const double main_c = fl * (K - tail);
+  const double main_h = 4.0 * ((bm + bn) * static_cast<double>(K - tail) + static_cast<double>(tail) * bn) /
+                        kPlanPcie;
+  const double tail_c = fl * tail;
+  const double tail_h = 4.0 * bm * static_cast<double>(tail) / kPlanPcie;
+  const double d2h = 4.0 * bm * static_cast<double>(bn) / kPlanPcie;
+  return std::max(main_c, main_h) + std::max(std::max(tail_c, tail_h), d2h);
+}
+
 int choose_s2(const EdgeCtx& x, S2Shape* out) {
   const int64_t m = x.r1 - x.r0, n = x.c1 - x.c0, K = x.K;
   const uint64_t cap = x.cap ? x.cap : (uint64_t(1) << 62);
   int64_t bk = x.obk > 0 ? x.obk : std::max<int64_t>(x.kc, 4);
   bk = std::min<int64_t>(bk, rup(K, 4));
-  // drain tail: strip compute must cover the strip's D2H: K_t >= 2 P / BW.
-  int64_t want_tail = rup(static_cast<int64_t>(2.0 * kPlanFlops / kPlanPcie), x.kc);
   std::vector<int64_t> bms, bns;
   int64_t bm0 = x.obm > 0 ? std::min(x.obm, m) : m;
   int64_t bn0 = x.obn > 0 ? std::min(x.obn, n) : n;
@@ -248,25 +262,30 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
     bns.push_back(v);
     if (v <= 256) break;
   }
-  // Among the C-block shapes that fit (each with its longest fitting drain
-  // tail), pick the fewest H2D bytes: every block streams its A row strip and
-  // B column strip once, 4K(bm + bn) per block.  Ties: longer tail, then
-  // taller blocks (contiguous C rows in the root).
-  const int64_t long_tail = rup(want_tail * 8 / 5, x.kc);
-  const int64_t tails[] = {long_tail < K ? long_tail : std::min(K, want_tail), std::min(K, want_tail),
-                           std::min(K, want_tail / 2), std::min(K, x.kc), 0};
+  // drain-tail candidates: multiples of k_chunk (at most ~64 of them) and K
+  std::vector<int64_t> tails{0};
+  const int64_t tstep = std::max<int64_t>(x.kc, rup(cdiv(K, 64), x.kc));
+  for (int64_t t = tstep; t < K; t += tstep) tails.push_back(t);
+  tails.push_back(K);
+  // Among the C-block shapes that fit, pick the fewest H2D bytes: every block
+  // streams its A row strip and B column strip once, 4K(bm + bn) per block.
+  // For each shape the drain tail minimises the predicted block time (ties:
+  // the longer tail); ties between shapes: predicted time, then taller blocks
+  // (contiguous C rows in the root).
   bool found = false;
   S2Shape best{};
   uint64_t best_h2d = 0;
-  int best_rank = 0;
+  double best_t = 0;
   for (int64_t bn : bns) {
     for (int64_t bm : bms) {
       const uint64_t h2d = static_cast<uint64_t>(cdiv(m, bm) * cdiv(n, bn)) * (bm + bn);
-      int rank = 0;
+      if (found && h2d > best_h2d) continue;
+      const int64_t strips = std::max<int64_t>(1, std::min<int64_t>(16, cdiv(bm, 1024)));
+      const int64_t sr = std::min(rup(cdiv(bm, strips), 128), bm);
+      bool have = false;
+      S2Shape cand{};
+      double cand_t = 0;
       for (int64_t tail : tails) {
-        ++rank;
-        int64_t strips = std::max<int64_t>(1, std::min<int64_t>(16, cdiv(bm, 1024)));
-        int64_t sr = std::min(rup(cdiv(bm, strips), 128), bm);
         uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr);
         int64_t use_bk = bk;
         if (bytes > cap && tail == 0 && bk > x.kc && x.obk <= 0) {   // the minimum panel
@@ -274,15 +293,22 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
           bytes = s2_bytes(bm, bn, use_bk, K, 0, 0);
         }
         if (bytes > cap) continue;
-        const bool better = !found || h2d < best_h2d || (h2d == best_h2d && rank < best_rank) ||
-                            (h2d == best_h2d && rank == best_rank && bm > best.bm);
-        if (better) {
-          best = S2Shape{bm, bn, use_bk, tail, tail > 0 ? sr : 0, bytes};
-          best_h2d = h2d;
-          best_rank = rank;
-          found = true;
+        const double t = s2_time(bm, bn, K, tail);
+        if (!have || t <= cand_t * (1.0 + 1e-9)) {
+          cand = S2Shape{bm, bn, use_bk, tail, tail > 0 ? sr : 0, bytes};
+          cand_t = t;
+          have = true;
         }
-        break;   // longest fitting tail for this shape
+      }
+      if (!have) continue;
+      const double tot = cand_t * static_cast<double>(cdiv(m, bm) * cdiv(n, bn));
+      const bool better = !found || h2d < best_h2d || (h2d == best_h2d && tot < best_t * (1.0 - 1e-9)) ||
+                          (h2d == best_h2d && tot <= best_t * (1.0 + 1e-9) && bm > best.bm);
+      if (better) {
+        best = cand;
+        best_h2d = h2d;
+        best_t = tot;
+        found = true;
       }
     }
   }
