@@ -188,7 +188,13 @@ typedef struct {
   int graph;            /* 1: capture each GPU's op list into a CUDA graph and replay it when the
                            same GEMM (sizes, buffers, options) is called again — the recursion
                            unfolded into a dependency graph (P:230 future work); HOST/HBM roots */
-  int reserved[5];
+  int shared_staging;   /* HOST root with G > 1 HBM siblings (S§8(f) NEXT-1): 0 = auto (on
+                           when every sibling has a region of the same shape under S2), -1 = off.
+                           Each sibling loads only 1/Pc of every A panel and 1/Pr of every B panel
+                           over its PCIe link and pulls the rest from its grid-row / grid-column
+                           peers' HBM (NVLink P2P; a local copy between virtual siblings).  C is
+                           bitwise identical with and without it.  Disables `graph`. */
+  int reserved[4];
 } northup_gemm_opts;
 
 typedef struct {
@@ -208,7 +214,9 @@ typedef struct {
   int num_gpus;          /* HBM siblings used */
   uint64_t hbm_peak_bytes; /* planned footprint at the HBM node of GPU 0 */
   int graph_replayed;    /* 1 when the call replayed CUDA graphs captured by an earlier call */
-  int reserved_stat;
+  int shared_staging;    /* 1 when the plan used NVLink-shared staging (opts->shared_staging) */
+  uint64_t bytes_p2p;    /* bytes pulled from sibling HBM (shared staging), all GPUs */
+  double t_p2p_ms;       /* sum over GPUs of busy time of sibling pulls (timing mode) */
 } northup_stats;
 
 /* C = A.B (no alpha/beta; C overwritten — reading R3), A (M x K), B (K x N),
@@ -246,14 +254,15 @@ int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, 
 typedef struct {
   int op;
   int worker;   /* GPU worker index (0 .. num_gpus-1) */
-  int stream;   /* 0 = H2D, 1 = compute, 2 = D2H, 3 = file I/O, 4 = D2D */
+  int stream;   /* 0 = H2D, 1 = compute, 2 = D2H, 3 = file I/O, 4 = D2D (sibling pulls) */
   int accumulate;
   int src_buf, dst_buf; /* COPY */
   int a_buf, b_buf, c_buf; /* LEAF / ZERO(c) */
   int64_t src_off, dst_off, src_ld, dst_ld, rows, cols; /* COPY, element units */
   int64_t a_off, b_off, c_off, lda, ldb, ldc, m, n, k;  /* LEAF, element units */
   int ndeps;
-  int deps[16]; /* indices of earlier ops this op must wait for (pruned per worker and stream) */
+  int deps[16]; /* indices of earlier ops this op must wait for (pruned per worker and stream;
+                   may name another worker's op: shared-staging pulls) */
 } northup_op;
 
 typedef struct {

@@ -49,7 +49,8 @@ class GemmOpts(ctypes.Structure):
     _fields_ = [("schedule", ctypes.c_int), ("replicate_result", ctypes.c_int),
                 ("k_chunk", ctypes.c_int64), ("npass", ctypes.c_int), ("resident", ctypes.c_int),
                 ("collect_timing", ctypes.c_int), ("a_panel_k", ctypes.c_int64),
-                ("graph", ctypes.c_int), ("reserved", ctypes.c_int * 5)]
+                ("graph", ctypes.c_int), ("shared_staging", ctypes.c_int),
+                ("reserved", ctypes.c_int * 4)]
 
 
 class Stats(ctypes.Structure):
@@ -63,7 +64,8 @@ class Stats(ctypes.Structure):
                 ("bn", ctypes.c_int64), ("bk", ctypes.c_int64), ("tail_k", ctypes.c_int64),
                 ("strips", ctypes.c_int64), ("schedule", ctypes.c_int), ("num_gpus", ctypes.c_int),
                 ("hbm_peak_bytes", ctypes.c_uint64), ("graph_replayed", ctypes.c_int),
-                ("reserved_stat", ctypes.c_int)]
+                ("shared_staging", ctypes.c_int), ("bytes_p2p", ctypes.c_uint64),
+                ("t_p2p_ms", ctypes.c_double)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -239,8 +241,10 @@ def partition_region(G: int, M: int, N: int, K: int, r: int) -> tuple[int, int, 
 
 def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 0,
               collect_timing: bool = False, replicate_result: bool = False,
-              a_panel_k: int = 0, graph: bool = False) -> GemmOpts:
+              a_panel_k: int = 0, graph: bool = False, shared_staging: int = 0) -> GemmOpts:
+    """northup_gemm_opts; shared_staging: 0 = auto (on for G > 1 uniform regions), -1 = off."""
     o = GemmOpts()
+    o.shared_staging = shared_staging
     o.a_panel_k = a_panel_k
     o.graph = int(graph)
     o.schedule = schedule

@@ -53,6 +53,20 @@ int finalize_workers(northup_tree_s* t) {
     t->workers.push_back(w);
     if (e != cudaSuccess) return cuda_fail(e, "stream creation");
   }
+  // Shared staging pulls panels from sibling HBM: enable NVLink P2P between
+  // every pair of distinct devices (without it the copies still work, staged
+  // by the driver).
+  for (WorkerState* a : t->workers)
+    for (WorkerState* b : t->workers) {
+      if (a->device == b->device) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, a->device, b->device);
+      if (!can) continue;
+      cudaSetDevice(a->device);
+      cudaError_t e = cudaDeviceEnablePeerAccess(b->device, 0);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+      else if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+    }
   return 0;
 }
 
@@ -195,7 +209,16 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
         if (!wait_flag(c, c.io_done, op.deps[d])) return fail(NU_EIO, "aborted: file I/O failed");
         continue;
       }
-      e = cudaStreamWaitEvent(s, w->events[op.deps[d]], 0);
+      cudaEvent_t ev = w->events[op.deps[d]];
+      if (q.worker != wi) {
+        // another sibling's op (shared-staging pull, NEXT-1): wait until that
+        // worker has recorded its event in this call, then wait on it on the
+        // device (cross-device event waits are legal).  Dependencies point
+        // backwards in plan order, so this cannot deadlock.
+        if (!wait_flag(c, c.issued, op.deps[d])) return fail(NU_ECUDA, "aborted: a sibling worker failed");
+        ev = worker_for_node(c.t, P.worker_node[q.worker])->events[op.deps[d]];
+      }
+      e = cudaStreamWaitEvent(s, ev, 0);
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent");
     }
     if (c.timing) cudaEventRecord(w->tev[2 * i], s);
@@ -381,9 +404,13 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   }
   // Only record an event where some later op on another stream waits for it.
   std::vector<char> needs(P.ops.size(), 0);
-  bool has_io = false;
+  bool has_io = false, cross = false;
   for (const northup_op& op : P.ops) {
-    for (int d = 0; d < op.ndeps; ++d) needs[op.deps[d]] = 1;
+    for (int d = 0; d < op.ndeps; ++d) {
+      needs[op.deps[d]] = 1;
+      cross |= P.ops[op.deps[d]].worker != op.worker && P.ops[op.deps[d]].stream != S_IO &&
+               op.stream != S_IO;
+    }
     has_io |= op.stream == S_IO;
   }
   ctx.needs_event = &needs;
@@ -393,7 +420,9 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
 
   const int W = P.num_workers;
   // CUDA-graph mode: replay the captured op lists of an identical earlier call
-  const bool use_graph = o && o->graph && !has_io && !ctx.timing;
+  // (per-worker graphs cannot hold another worker's events: no graphs with
+  // shared staging)
+  const bool use_graph = o && o->graph && !has_io && !cross && !ctx.timing;
   std::vector<int64_t> key;
   if (use_graph) {
     key = graph_key(P, ctx.base, o);
@@ -455,7 +484,8 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     for (int wi = 0; wi < W; ++wi) {
       st->t_h2d_ms += busy[wi][S_H2D];
       st->t_compute_ms += busy[wi][S_COMP];
-      st->t_d2h_ms += busy[wi][S_D2H] + busy[wi][S_D2D];
+      st->t_d2h_ms += busy[wi][S_D2H];
+      st->t_p2p_ms += busy[wi][S_D2D];
     }
     st->t_io_ms = ctx.io_ms;
   }

@@ -211,6 +211,10 @@ struct EdgeCtx {
   int64_t kc;
   int64_t obm, obn, obk;   // block override at the parent node
   int sched;
+  // NVLink-shared staging (S§8(f) NEXT-1): this worker loads 1/a_share of each
+  // A panel and 1/b_share of each B panel over PCIe, its row / column peers
+  // the rest, and pulls the other pieces from them over NVLink.
+  int a_share = 1, b_share = 1;
 };
 
 // ---------------------------------------------------------------- S2
@@ -235,13 +239,17 @@ uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, i
 // phase streams the A/B panels of K - K_t plus the resident B tail over H2D
 // while computing K - K_t; the tail phase computes row strips over K_t while
 // their A strips arrive (H2D) and finished C strips leave (D2H).
-static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail) {
+// With shared staging only this worker's pieces (1/a_share of A, 1/b_share of
+// B) cross its PCIe link; NVLink pulls are ~20x faster and not modelled.
+static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail, int a_share = 1,
+                      int b_share = 1) {
   const double fl = 2.0 * bm * bn / kPlanFlops;               // s per unit of K
+  const double ea = static_cast<double>(bm) / a_share, eb = static_cast<double>(bn) / b_share;
   const double main_c = fl * (K - tail);
-  const double main_h = 4.0 * ((bm + bn) * static_cast<double>(K - tail) + static_cast<double>(tail) * bn) /
+  const double main_h = 4.0 * ((ea + eb) * static_cast<double>(K - tail) + static_cast<double>(tail) * eb) /
                         kPlanPcie;
   const double tail_c = fl * tail;
-  const double tail_h = 4.0 * bm * static_cast<double>(tail) / kPlanPcie;
+  const double tail_h = 4.0 * ea * static_cast<double>(tail) / kPlanPcie;
   const double d2h = 4.0 * bm * static_cast<double>(bn) / kPlanPcie;
   return std::max(main_c, main_h) + std::max(std::max(tail_c, tail_h), d2h);
 }
@@ -278,7 +286,10 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
   double best_t = 0;
   for (int64_t bn : bns) {
     for (int64_t bm : bms) {
-      const uint64_t h2d = static_cast<uint64_t>(cdiv(m, bm) * cdiv(n, bn)) * (bm + bn);
+      // per-GPU PCIe bytes per unit of K, scaled by a_share * b_share (shared
+      // staging divides A by a_share and B by b_share)
+      const uint64_t h2d = static_cast<uint64_t>(cdiv(m, bm) * cdiv(n, bn)) *
+                           static_cast<uint64_t>(bm * x.b_share + bn * x.a_share);
       if (found && h2d > best_h2d) continue;
       const int64_t strips = std::max<int64_t>(1, std::min<int64_t>(16, cdiv(bm, 1024)));
       const int64_t sr = std::min(rup(cdiv(bm, strips), 128), bm);
@@ -293,7 +304,7 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
           bytes = s2_bytes(bm, bn, use_bk, K, 0, 0);
         }
         if (bytes > cap) continue;
-        const double t = s2_time(bm, bn, K, tail);
+        const double t = s2_time(bm, bn, K, tail, x.a_share, x.b_share);
         if (!have || t <= cand_t * (1.0 + 1e-9)) {
           cand = S2Shape{bm, bn, use_bk, tail, tail > 0 ? sr : 0, bytes};
           cand_t = t;
@@ -320,6 +331,63 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
               (unsigned long long)x.cap);
 }
 
+// Arena layout of one S2 worker (elements):
+//   [C block bm x pad(bn)] [kSlots x (A slot bm x pad(bk), B slot bk x pad(bn))]
+//   [B tail tail x pad(bn)] [kSlots x A strip sr x pad(tail)]
+struct S2Layout {
+  int arena = -1;
+  int64_t ldC = 0, ldA = 0, ldBs = 0, ldAt = 0;
+  int64_t offC = 0, offBT = 0;
+  int64_t offSA[kSlots] = {}, offSB[kSlots] = {}, offAT[kSlots] = {};
+};
+
+S2Layout layout_s2(Builder& B, const S2Shape& s, int hbm_node, int w, int64_t K) {
+  S2Layout L;
+  L.arena = B.add_buf(B_ARENA, hbm_node, w, s.bytes);
+  L.ldC = pad_ld(s.bn);
+  L.ldA = pad_ld(s.bk);
+  L.ldBs = pad_ld(s.bn);
+  L.ldAt = pad_ld(s.tail);
+  int64_t off = 0;
+  L.offC = off;
+  off += s.bm * L.ldC;
+  const int64_t kmain = K - s.tail;
+  for (int i = 0; i < kSlots; ++i) {
+    L.offSA[i] = off;
+    off += kmain > 0 ? s.bm * L.ldA : 0;
+    L.offSB[i] = off;
+    off += kmain > 0 ? s.bk * L.ldBs : 0;
+  }
+  if (s.tail > 0) {
+    L.offBT = off;
+    off += s.tail * L.ldBs;
+    for (int i = 0; i < kSlots; ++i) {
+      L.offAT[i] = off;
+      off += s.sr * L.ldAt;
+    }
+  }
+  return L;
+}
+
+// Rows of the graded drain strips (full strips while more than two remain,
+// then halving sizes, so the last D2H is small).
+static int64_t next_strip(int64_t bm, int64_t r, int64_t sr) {
+  const int64_t rem = bm - r;
+  return rem > 2 * sr ? sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
+}
+
+void s2_stats(const S2Shape& s, northup_stats* st) {
+  st->bm = s.bm;
+  st->bn = s.bn;
+  st->bk = s.bk;
+  st->tail_k = s.tail;
+  st->strips = 0;
+  for (int64_t r = 0; s.tail > 0 && r < s.bm; r += next_strip(s.bm, r, s.sr), ++st->strips) {
+  }
+  st->hbm_peak_bytes = s.bytes;
+  st->schedule = NU_SCHED_S2;
+}
+
 int build_s2(const EdgeCtx& x, northup_stats* st) {
   S2Shape s{};
   int rc = choose_s2(x, &s);
@@ -327,41 +395,14 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
   Builder& B = *x.B;
   const int w = x.worker;
   const int64_t m = x.r1 - x.r0, n = x.c1 - x.c0, K = x.K;
-  const int arena = B.add_buf(B_ARENA, x.hbm_node, w, s.bytes);
-  // arena layout (elements)
-  const int64_t ldC = pad_ld(s.bn), ldA = pad_ld(s.bk), ldBs = pad_ld(s.bn), ldAt = pad_ld(s.tail);
-  int64_t off = 0;
-  const int64_t offC = off;
-  off += s.bm * ldC;
+  const S2Layout L = layout_s2(B, s, x.hbm_node, w, K);
+  const int arena = L.arena;
+  const int64_t ldC = L.ldC, ldA = L.ldA, ldBs = L.ldBs, ldAt = L.ldAt, offC = L.offC, offBT = L.offBT;
+  const int64_t* offSA = L.offSA;
+  const int64_t* offSB = L.offSB;
+  const int64_t* offAT = L.offAT;
   const int64_t kmain = K - s.tail;
-  int64_t offSA[kSlots], offSB[kSlots], offAT[kSlots], offBT = 0;
-  for (int i = 0; i < kSlots; ++i) {
-    offSA[i] = off;
-    off += kmain > 0 ? s.bm * ldA : 0;
-    offSB[i] = off;
-    off += kmain > 0 ? s.bk * ldBs : 0;
-  }
-  if (s.tail > 0) {
-    offBT = off;
-    off += s.tail * ldBs;
-    for (int i = 0; i < kSlots; ++i) {
-      offAT[i] = off;
-      off += s.sr * ldAt;
-    }
-  }
-  if (w == 0) {
-    st->bm = s.bm;
-    st->bn = s.bn;
-    st->bk = s.bk;
-    st->tail_k = s.tail;
-    st->strips = 0;
-    for (int64_t r = 0, rr = 0; s.tail > 0 && r < s.bm; r += rr, ++st->strips) {
-      const int64_t rem = s.bm - r;
-      rr = rem > 2 * s.sr ? s.sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
-    }
-    st->hbm_peak_bytes = s.bytes;
-    st->schedule = NU_SCHED_S2;
-  }
+  if (w == 0) s2_stats(s, st);
   int panel_it = 0, strip_it = 0;
   for (int64_t i0 = 0; i0 < m; i0 += s.bm) {
     const int64_t bm = std::min(s.bm, m - i0);
@@ -425,8 +466,7 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
         // Graded strips: full strips while more than two remain, then halving
         // sizes, so the last D2H (the exposed drain) is small.
         for (int64_t r = 0, rr = 0; r < bm; r += rr, ++strip_it) {
-          const int64_t rem = bm - r;
-          rr = rem > 2 * s.sr ? s.sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
+          rr = next_strip(bm, r, s.sr);
           const int sl = strip_it % kSlots;
           B.emit(make_copy(w, S_H2D, x.A, (gr + r) * x.lda + kmain, x.lda, arena, offAT[sl], ldAt, rr,
                            s.tail),
@@ -453,6 +493,185 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
     }
   }
   return 0;
+}
+
+// ------------------------------------------- S2 with NVLink-shared staging
+// S§8(f) NEXT-1 (P:230 siblings; "streaming over networks").  The G
+// siblings form the partition grid Pr x Pc: the Pc siblings of a grid row need
+// the same A panels, the Pr siblings of a grid column the same B panels.  Per
+// K panel every sibling loads only its piece over its own PCIe link (rows
+// piece j of the A panel, j = its index in the grid row; columns piece i of the
+// B panel, i = its index in the grid column) and pulls the other pieces from
+// its peers' HBM slots with a copy on its own D2D stream (NVLink P2P between
+// devices, a local copy between virtual siblings of one device).  All workers
+// use the same S2 shape and arena layout; the plan is emitted in lock step
+// (loads, then pulls, then leaves of a panel, for all workers) so every pull's
+// cross-worker dependency points backwards in plan order.  The leaf ops and
+// their K-panel sequence are those of build_s2, so C is bitwise identical.
+static void piece_range(int64_t n, int parts, int q, int64_t* lo, int64_t* hi) {
+  const int64_t step = rup(cdiv(n, parts), 32);   // 128-B aligned piece edges
+  *lo = std::min(n, step * q);
+  *hi = std::min(n, *lo + step);
+}
+
+int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northup_stats* st) {
+  const int G = static_cast<int>(xs.size());
+  for (EdgeCtx& x : xs) {
+    x.a_share = Pc;
+    x.b_share = Pr;
+  }
+  S2Shape s{};
+  int rc = choose_s2(xs[0], &s);
+  if (rc) return rc;
+  for (const EdgeCtx& x : xs)
+    if (x.cap && s.bytes > x.cap)
+      return fail(NU_ENOMEM, "HBM node %d capacity %llu B below the shared S2 block", x.hbm_node,
+                  (unsigned long long)x.cap);
+  const EdgeCtx& x0 = xs[0];
+  const int64_t m = x0.r1 - x0.r0, n = x0.c1 - x0.c0, K = x0.K;
+  const int64_t lda = x0.lda, ldb = x0.ldb, ldc = x0.ldc;
+  std::vector<S2Layout> L(G);
+  for (int w = 0; w < G; ++w) L[w] = layout_s2(B, s, xs[w].hbm_node, w, K);
+  const S2Layout& Y = L[0];   // offsets are the same in every worker's arena
+  s2_stats(s, st);
+  st->shared_staging = 1;
+  const int64_t kmain = K - s.tail;
+
+  // One shared slot region (rows x cols at offset `off`, leading dim `ld`):
+  // A side pieces split rows among the Pc row peers, B side pieces split
+  // columns among the Pr column peers.
+  struct Side {
+    bool a;
+    int hb;                      // user buffer (root tier)
+    int64_t hld;                 // its leading dimension
+    std::vector<int64_t> src;    // per worker: root offset of the region's origin
+    int64_t off, ld, rows, cols;
+  };
+  auto idx = [&](const Side& sd, int w) { return sd.a ? w % Pc : w / Pc; };
+  auto peer = [&](const Side& sd, int w, int q) { return sd.a ? (w / Pc) * Pc + q : q * Pc + w % Pc; };
+  auto sub = [&](const Side& sd, int q, int64_t* r0, int64_t* nr, int64_t* c0, int64_t* nc) {
+    int64_t lo, hi;
+    piece_range(sd.a ? sd.rows : sd.cols, sd.a ? Pc : Pr, q, &lo, &hi);
+    *r0 = sd.a ? lo : 0;
+    *nr = sd.a ? hi - lo : sd.rows;
+    *c0 = sd.a ? 0 : lo;
+    *nc = sd.a ? sd.cols : hi - lo;
+  };
+  auto load = [&](const Side& sd) {        // own piece over PCIe (data_down)
+    for (int w = 0; w < G; ++w) {
+      int64_t r0, nr, c0, nc;
+      sub(sd, idx(sd, w), &r0, &nr, &c0, &nc);
+      if (nr <= 0 || nc <= 0) continue;
+      const int64_t so = sd.src[w] + r0 * sd.hld + c0, d = sd.off + r0 * sd.ld + c0;
+      B.emit(make_copy(w, S_H2D, sd.hb, so, sd.hld, L[w].arena, d, sd.ld, nr, nc),
+             {{sd.hb, so, sd.hld, nr, nc, false}, {L[w].arena, d, sd.ld, nr, nc, true}});
+      st->bytes_h2d += 4ull * nr * nc;
+    }
+  };
+  auto pull = [&](const Side& sd) {        // the peers' pieces over NVLink
+    const int parts = sd.a ? Pc : Pr;
+    for (int w = 0; w < G; ++w)
+      for (int q = 0; q < parts; ++q) {
+        if (q == idx(sd, w)) continue;
+        int64_t r0, nr, c0, nc;
+        sub(sd, q, &r0, &nr, &c0, &nc);
+        if (nr <= 0 || nc <= 0) continue;
+        const int src = L[peer(sd, w, q)].arena;
+        const int64_t d = sd.off + r0 * sd.ld + c0;
+        B.emit(make_copy(w, S_D2D, src, d, sd.ld, L[w].arena, d, sd.ld, nr, nc),
+               {{src, d, sd.ld, nr, nc, false}, {L[w].arena, d, sd.ld, nr, nc, true}});
+        st->bytes_p2p += 4ull * nr * nc;
+      }
+  };
+  auto side = [&](bool a, int64_t off, int64_t ld, int64_t rows, int64_t cols, auto src_of) {
+    Side sd{a, a ? x0.A : x0.Bb, a ? lda : ldb, std::vector<int64_t>(G), off, ld, rows, cols};
+    for (int w = 0; w < G; ++w) sd.src[w] = src_of(xs[w]);
+    return sd;
+  };
+
+  int panel_it = 0, strip_it = 0;
+  for (int64_t i0 = 0; i0 < m; i0 += s.bm) {
+    const int64_t bm = std::min(s.bm, m - i0);
+    for (int64_t j0 = 0; j0 < n; j0 += s.bn) {
+      const int64_t bn = std::min(s.bn, n - j0);
+      const int64_t npan = kmain > 0 ? cdiv(kmain, s.bk) : 0;
+      const int64_t ntail_pieces = s.tail > 0 ? cdiv(s.tail, s.bk) : 0;
+      int64_t pieces_done = 0;
+      auto load_tail_piece = [&](int64_t pc) {
+        const int64_t k0 = kmain + pc * s.bk, kk = std::min(s.bk, K - k0);
+        Side sb = side(false, Y.offBT + (k0 - kmain) * Y.ldBs, Y.ldBs, kk, bn,
+                       [&](const EdgeCtx& x) { return k0 * ldb + x.c0 + j0; });
+        load(sb);
+        pull(sb);
+      };
+      for (int64_t p = 0; p < npan; ++p, ++panel_it) {
+        const int sl = panel_it % kSlots;
+        const int64_t k0 = p * s.bk, kk = std::min(s.bk, kmain - k0);
+        Side sa = side(true, Y.offSA[sl], Y.ldA, bm, kk,
+                       [&](const EdgeCtx& x) { return (x.r0 + i0) * lda + k0; });
+        Side sb = side(false, Y.offSB[sl], Y.ldBs, kk, bn,
+                       [&](const EdgeCtx& x) { return k0 * ldb + x.c0 + j0; });
+        load(sa);
+        load(sb);
+        pull(sa);
+        pull(sb);
+        // the leaf ops of build_s2 (first panel as a 4 x 4 sub-block grid)
+        const int64_t gb = (p == 0 && bm >= 4096 && bn >= 4096) ? 4 : 1;
+        const int64_t sbm = rup(cdiv(bm, gb), 256), sbn = rup(cdiv(bn, gb), 256);
+        for (int w = 0; w < G; ++w) {
+          const int ar = L[w].arena;
+          for (int64_t jj = 0; jj < bn; jj += sbn) {
+            const int64_t cn = std::min(sbn, bn - jj);
+            for (int64_t ii = 0; ii < bm; ii += sbm) {
+              const int64_t rm = std::min(sbm, bm - ii);
+              const int64_t ao = Y.offSA[sl] + ii * Y.ldA, bo = Y.offSB[sl] + jj,
+                            co = Y.offC + ii * Y.ldC + jj;
+              B.emit(make_leaf(w, ar, ao, Y.ldA, ar, bo, Y.ldBs, ar, co, Y.ldC, rm, cn, kk, p > 0 ? 1 : 0),
+                     {{ar, ao, Y.ldA, rm, kk, false}, {ar, bo, Y.ldBs, kk, cn, false},
+                      {ar, co, Y.ldC, rm, cn, true}});
+              st->leaf_launches++;
+            }
+          }
+        }
+        const int64_t skip = std::min<int64_t>(2, std::max<int64_t>(0, npan - 1));
+        while (pieces_done < ntail_pieces && p >= skip &&
+               (pieces_done + 1) * (npan - skip) <= (p + 1 - skip) * ntail_pieces)
+          load_tail_piece(pieces_done++);
+      }
+      while (pieces_done < ntail_pieces) load_tail_piece(pieces_done++);
+      if (s.tail > 0) {
+        for (int64_t r = 0, rr = 0; r < bm; r += rr, ++strip_it) {
+          rr = next_strip(bm, r, s.sr);
+          const int sl = strip_it % kSlots;
+          Side sa = side(true, Y.offAT[sl], Y.ldAt, rr, s.tail,
+                         [&](const EdgeCtx& x) { return (x.r0 + i0 + r) * lda + kmain; });
+          load(sa);
+          pull(sa);
+          for (int w = 0; w < G; ++w) {
+            const int ar = L[w].arena;
+            const int64_t co = Y.offC + r * Y.ldC;
+            B.emit(make_leaf(w, ar, Y.offAT[sl], Y.ldAt, ar, Y.offBT, Y.ldBs, ar, co, Y.ldC, rr, bn, s.tail,
+                             kmain > 0 ? 1 : 0),
+                   {{ar, Y.offAT[sl], Y.ldAt, rr, s.tail, false}, {ar, Y.offBT, Y.ldBs, s.tail, bn, false},
+                    {ar, co, Y.ldC, rr, bn, true}});
+            st->leaf_launches++;
+            const int64_t dst = (xs[w].r0 + i0 + r) * ldc + xs[w].c0 + j0;
+            B.emit(make_copy(w, S_D2H, ar, co, Y.ldC, x0.C, dst, ldc, rr, bn),
+                   {{ar, co, Y.ldC, rr, bn, false}, {x0.C, dst, ldc, rr, bn, true}});
+            st->bytes_d2h += 4ull * rr * bn;
+          }
+        }
+      } else {
+        for (int w = 0; w < G; ++w) {
+          const int64_t dst = (xs[w].r0 + i0) * ldc + xs[w].c0 + j0;
+          B.emit(make_copy(w, S_D2H, L[w].arena, Y.offC, Y.ldC, x0.C, dst, ldc, bm, bn),
+                 {{L[w].arena, Y.offC, Y.ldC, bm, bn, false}, {x0.C, dst, ldc, bm, bn, true}});
+          st->bytes_d2h += 4ull * bm * bn;
+        }
+      }
+    }
+  }
+  return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
 }
 
 // ---------------------------------------------------------------- S1
@@ -788,8 +1007,10 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   P.worker_node = hbm;
   st.num_gpus = G;
   if (M == 0 || N == 0 || K == 0) return 0;
+  std::vector<EdgeCtx> xs;
+  std::vector<int> uses;
   for (int w = 0; w < G; ++w) {
-    EdgeCtx x;
+    EdgeCtx x{};
     x.B = &B;
     x.worker = w;
     x.hbm_node = hbm[w];
@@ -801,7 +1022,6 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     x.ldc = N;
     rc = region_of(G, M, N, w, &x.r0, &x.r1, &x.c0, &x.c1);
     if (rc) return rc;
-    if (x.r1 <= x.r0 || x.c1 <= x.c0) continue;   // more GPUs than rows/cols
     x.K = K;
     x.cap = t->nodes[hbm[w]].capacity;
     x.kc = P.kc;
@@ -817,8 +1037,27 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
                                 (root.bn > 0 && root.bn < x.c1 - x.c0);
       use = small_blocks ? NU_SCHED_S1 : NU_SCHED_S2;
     }
-    rc = use == NU_SCHED_S1 ? build_s1(x, &st) : build_s2(x, &st);
+    xs.push_back(x);
+    uses.push_back(use);
+  }
+  // NVLink-shared staging (NEXT-1): on by default for G > 1 when every sibling
+  // has a region of the same shape under S2 (opts->shared_staging < 0 disables).
+  int Pr = 1, Pc = 1;
+  partition_grid(G, M, N, &Pr, &Pc);
+  bool share = G > 1 && !(o && o->shared_staging < 0);
+  for (int w = 0; w < G && share; ++w)
+    share = uses[w] == NU_SCHED_S2 && xs[w].r1 - xs[w].r0 == xs[0].r1 - xs[0].r0 &&
+            xs[w].c1 - xs[w].c0 == xs[0].c1 - xs[0].c0 && xs[w].r1 > xs[w].r0 && xs[w].c1 > xs[w].c0;
+  if (share) {
+    rc = build_s2_shared(B, xs, Pr, Pc, &st);
     if (rc) return rc;
+  } else {
+    for (int w = 0; w < G; ++w) {
+      const EdgeCtx& x = xs[w];
+      if (x.r1 <= x.r0 || x.c1 <= x.c0) continue;   // more GPUs than rows/cols
+      rc = uses[w] == NU_SCHED_S1 ? build_s1(x, &st) : build_s2(x, &st);
+      if (rc) return rc;
+    }
   }
   st.ops = static_cast<int64_t>(P.ops.size());
   for (const northup_op& op : P.ops)

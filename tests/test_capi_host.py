@@ -311,3 +311,78 @@ def test_random_plans_replay_exactly(M, N, K, G, cap_kib, kc, sched, file_root, 
     if cap:
         assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
     t.destroy()
+
+
+# ------------------------------------------- NVLink-shared staging (NEXT-1)
+@pytest.mark.parametrize("M,N,K,G,cap,kc", [
+    (512, 512, 640, 2, 0, 64),          # 2 x 1 grid: B shared by the 2 row strips
+    (512, 512, 640, 4, 0, 64),          # 2 x 2: A shared in grid rows, B in grid columns
+    (1024, 512, 1000, 8, 0, 128),       # 4 x 2, ragged last K panel
+    (600, 600, 700, 4, 1_200_000, 64),  # capacity forces several C blocks per region
+    (4096, 8192, 512, 8, 0, 128),       # first-panel sub-block grid (bm, bn >= 4096)
+])
+def test_shared_staging_plan_replays_exactly(M, N, K, G, cap, kc):
+    """Shared staging: every A/B byte crosses PCIe once per grid row / column
+    (each sibling loads 1/Pc of A and 1/Pr of B), the rest is pulled from
+    peers; any dependency-respecting order (cross-worker waits included)
+    computes A.B exactly."""
+    A = nugen.fill(M, K, 6, 1, "int")
+    B = nugen.fill(K, N, 6, 2, "int")
+    ref = A.astype(np.float64) @ B.astype(np.float64)
+    t, _ = nu.host_tree(G, cap)
+    p = t.plan(M, N, K, nu.make_opts(k_chunk=kc))
+    s = p.stats()
+    assert s["shared_staging"] == 1
+    ops = p.ops()
+    cross = [o for o in ops for d in o["deps"] if ops[d]["worker"] != o["worker"]]
+    assert cross and all(o["stream"] in (4, 0) for o in cross)   # pulls (and slot reuse by loads)
+    for seed in range(4):
+        C = simulate(p, A, B, M, N, K, rng=random.Random(seed))
+        assert np.array_equal(C, ref), f"order seed {seed} broke a dependency"
+    Pr, Pc = nu.partition(G, M, N)
+    m, n = M // Pr, N // Pc
+    nbr, nbc = -(-m // s["bm"]), -(-n // s["bn"])
+    # per C block every sibling streams its A strip once (shared by Pc) and
+    # its B strip once (shared by Pr): total PCIe bytes = blocks x (A + B) once
+    assert s["bytes_h2d"] == 4 * K * (M * nbc + N * nbr)
+    assert s["bytes_p2p"] == 4 * K * (M * nbc * (Pc - 1) + N * nbr * (Pr - 1))
+    assert s["bytes_d2h"] == 4 * M * N
+    if cap:
+        assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
+    t.destroy()
+
+
+def test_shared_staging_same_leaf_sequence_and_fewer_pcie_bytes():
+    """On and off give the same leaf ops per worker (so bitwise-identical C on
+    the GPU) while PCIe bytes drop from 4K(M Pc + N Pr) to 4K(M + N)."""
+    M, N, K, G = 2048, 2048, 4096, 8
+    t, _ = nu.host_tree(G)
+    on = t.plan(M, N, K, nu.make_opts(k_chunk=256))
+    off = t.plan(M, N, K, nu.make_opts(k_chunk=256, shared_staging=-1))
+    so, sf = on.stats(), off.stats()
+    assert so["shared_staging"] == 1 and sf["shared_staging"] == 0
+    Pr, Pc = nu.partition(G, M, N)
+    assert sf["bytes_h2d"] == 4 * K * (M * Pc + N * Pr) and so["bytes_h2d"] == 4 * K * (M + N)
+
+    def leaves(p):
+        bufs = p.bufs()
+        out = {}
+        for o in p.ops():
+            if o["op"] == nu.NU_OP_LEAF:
+                out.setdefault(o["worker"], []).append(
+                    (o["m"], o["n"], o["k"], o["accumulate"], o["c_off"], o["ldc"]))
+        return out
+    lo, lf = leaves(on), leaves(off)
+    # the leaf sequence per worker covers the same C elements in the same K order
+    for w in range(G):
+        ko = [(m, n, k, a) for (m, n, k, a, _, _) in lo[w]]
+        kf = [(m, n, k, a) for (m, n, k, a, _, _) in lf[w]]
+        assert sum(m * n * k for m, n, k, _ in ko) == sum(m * n * k for m, n, k, _ in kf)
+    t.destroy()
+
+
+def test_shared_staging_falls_back_for_ragged_regions():
+    t, _ = nu.host_tree(3)
+    p = t.plan(301, 200, 90, nu.make_opts(k_chunk=32))     # 1 x 3 grid, 200 = 67+67+66
+    assert p.stats()["shared_staging"] == 0
+    t.destroy()

@@ -196,7 +196,7 @@ def test_graph_capture_and_replay(G, block):
         t.set_block(0, *block)
     t.finalize()
     p = HostProblem(t, M, N, K, 8, "int")
-    o = nu.make_opts(graph=True)
+    o = nu.make_opts(graph=True, shared_staging=-1)   # shared staging disables graphs
     st1 = t.gemm(p.A, p.B, p.C, M, N, K, o)
     c1 = p.c.copy()
     p.c[...] = np.nan
@@ -205,3 +205,23 @@ def test_graph_capture_and_replay(G, block):
     assert np.array_equal(c1, p.c)
     assert np.array_equal(p.c.astype(np.float64), oracle.gemm(p.a, p.b))
     t.destroy()
+
+
+@pytest.mark.parametrize("G,M,N,K,cap,kind", [
+    (2, 1024, 768, 4096, 0, "uniform"),
+    (4, 1024, 1024, 3000, 0, "int"),
+    (8, 2048, 1024, 2048, 0, "uniform"),
+    (4, 1536, 1536, 2560, 6 << 20, "int"),      # capacity: several C blocks per sibling
+])
+def test_shared_staging_virtual_siblings(G, M, N, K, cap, kind):
+    """NEXT-1 shared staging on G virtual siblings of GPU 0: each sibling loads
+    its piece of every panel over PCIe and pulls the rest from its peers'
+    arenas (cross-worker event waits); C is bitwise identical to the unshared
+    plan and matches the oracle."""
+    kc = 512
+    C1, a, b, s1 = run_host(M, N, K, G=G, cap=cap, kind=kind, seed=4, k_chunk=kc, collect_timing=True)
+    C0, _, _, s0 = run_host(M, N, K, G=G, cap=cap, kind=kind, seed=4, k_chunk=kc, shared_staging=-1)
+    assert s1["shared_staging"] == 1 and s0["shared_staging"] == 0
+    assert s1["bytes_p2p"] > 0 and s1["bytes_h2d"] < s0["bytes_h2d"] and s1["t_p2p_ms"] > 0
+    assert np.array_equal(C1, C0)
+    check(C1, a, b, kind)
