@@ -194,8 +194,15 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     seed = int(name[-1])
     kc = args.k_chunk
 
-    # --- the out-of-core tree: HOST root -> HBM (cap) -> SMEM/TMEM leaf
-    t, hbm = nu.host_tree(1, cfg["cap"], devices=[local_rank])
+    # --- the out-of-core tree: HOST root -> HBM (cap) -> SMEM/TMEM leaf.  N > 1:
+    # the same tree on every rank (one HBM sibling per rank); this rank runs
+    # only its own sibling (multi-process siblings, northup_tree_set_local).
+    if world > 1:
+        devs = [(i % args.device_mod) if args.device_mod > 0 else i for i in range(world)]
+        t, hbm = nu.host_tree(world, cfg["cap"], devices=devs)
+        t.set_local(hbm[rank])
+    else:
+        t, hbm = nu.host_tree(1, cfg["cap"], devices=[local_rank])
     if cfg["block"]:
         t.set_block(0, *cfg["block"])
     t.finalize()
@@ -219,6 +226,18 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     hB = th.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4)
     hC = th.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4)
     opts = nu.make_opts(k_chunk=kc)
+    ooc_opts = nu.make_opts(k_chunk=kc, shared_staging=-1 if args.no_shared_staging else 0)
+    shared_peers = False
+    if world > 1 and not args.no_shared_staging:
+        # NEXT-1: siblings of a grid row / column share A / B panels over
+        # NVLink; exchange the CUDA IPC handles of arenas and flag words
+        blob = t.peer_export(M, N, K, ooc_opts)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, blob)
+        for w, bl in enumerate(blobs):
+            if w != rank:
+                t.peer_import(w, bl)
+        shared_peers = True
     stream = torch.cuda.current_stream(dev)
 
     def barrier():
@@ -250,8 +269,10 @@ def run_ours(args, rank: int, world: int, local_rank: int):
 
     ooc_stats = {}
 
+    GM, GN = (M, N) if world > 1 else (m, n)
+
     def step_ooc():
-        ooc_stats.update(t.gemm(Ab, Bb, Cb, m, n, K, opts))
+        ooc_stats.update(t.gemm(Ab, Bb, Cb, GM, GN, K, ooc_opts))
 
     with ClockSampler(local_rank) as clk:
         t_hbm, per_hbm = timed(step_hbm, args.steps, args.warmup)
@@ -328,6 +349,8 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                 "region_per_gpu": [m, n, K],
                 "parallelism": f"C subtrees {nu.partition(world, M, N)} over {world} GPU(s)" if world > 1 else "1 GPU",
                 "schedule": {1: "S1", 2: "S2"}.get(ooc_stats.get("schedule"), "auto"),
+                "shared_staging": bool(ooc_stats.get("shared_staging")),
+                "shared_staging_peers": "CUDA IPC (multi-process siblings)" if shared_peers else None,
                 "blocks": [ooc_stats.get("bm"), ooc_stats.get("bn"), ooc_stats.get("bk")],
                 "drain_tail_k": ooc_stats.get("tail_k"), "drain_strips": ooc_stats.get("strips"),
                 "hbm_footprint_bytes": ooc_stats.get("hbm_peak_bytes"),
@@ -336,6 +359,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
             "e2e": {"value": round(e2e, 3), "unit": "TFLOP/s",
                     "h2d_bytes_per_step": int(ooc_stats.get("bytes_h2d", 0)),
                     "d2h_bytes_per_step": int(ooc_stats.get("bytes_d2h", 0)),
+                    "p2p_bytes_per_step": int(ooc_stats.get("bytes_p2p", 0)),
                     "ms_per_step": round(ms_ooc, 3),
                     "leaf_launches_per_step": int(ooc_stats.get("leaf_launches", 0))},
             "slowdown_pct_vs_in_hbm": round(100.0 * (ms_ooc / ms_hbm - 1.0), 2),
@@ -358,7 +382,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                          "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "
                                           "(profiles/leaf_traffic.json); algorithmic bytes per launch "
                                           f"= A/B panel + C read+write = {4 * (m + n) * min(K, kc_eff) + 8 * m * n:.3e}"},
-            "gpu_launches": args.steps * launches_per_step + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
+            "gpu_launches": args.steps * launches_per_step * world + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
             "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise_cross_tier,
                        "bitwise_tree_vs_leaf": bitwise_tree_vs_leaf},
             "clocks": clk.summary(),
@@ -434,6 +458,8 @@ def main():
                     help="N>1: after the timed steps, gather C to every GPU (S8e) and time it")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo only for multi-rank tests on one GPU)")
+    ap.add_argument("--no-shared-staging", action="store_true",
+                    help="N>1: every rank loads its whole A/B strips over PCIe (no NVLink sharing)")
     ap.add_argument("--device-mod", type=int, default=0,
                     help="map LOCAL_RANK modulo this many GPUs (multi-rank tests on one GPU)")
     args = ap.parse_args()

@@ -304,6 +304,33 @@ int northup_partition(int G, int64_t M, int64_t N, int64_t K, int* Pr, int* Pc);
 int northup_partition_region(int G, int64_t M, int64_t N, int64_t K, int r, int64_t* r0,
                              int64_t* r1, int64_t* c0, int64_t* c1);
 
+/* ------------------------------------------ multi-process siblings (S§8(e)) */
+/* One process per GPU (torchrun): every process builds the SAME tree (HOST
+ * root -> G HBM children, node i on the GPU of process i) and calls
+ * northup_tree_set_local(t, its HBM node) before finalize.  northup_gemm then
+ * runs only that sibling's share of the plan, and A, B, C passed to it hold
+ * only this sibling's strips: A rows [r0, r1) (ld K), B columns [c0, c1)
+ * (ld c1 - c0), C the (r1 - r0) x (c1 - c0) region (ld c1 - c0), with the region
+ * from northup_partition_region(G, M, N, K, index of the node among the root's
+ * children).  Without shared staging no peer is involved.  With shared staging
+ * (NEXT-1, opts->shared_staging) the pulls read the peers' HBM: before the
+ * first GEMM of a shape every process calls northup_peer_export (plans the GEMM,
+ * allocates its arena and flag words, writes a blob of CUDA IPC handles into
+ * `blob`, `cap` >= *len bytes; *len is set even when cap is too small), the
+ * blobs are exchanged between processes by the caller (e.g. all_gather_object)
+ * and each process imports every other sibling's blob with northup_peer_import
+ * (worker = that sibling's index).  Export/import are collective: every
+ * process does them for the same GEMM, after its previous GEMM returned.
+ * Cross-sibling dependencies are device-side waits on flag words (no host
+ * blocking); each call ends with a device-side join of all siblings.
+ * Errors: NU_ESTATE when called out of order or when northup_gemm runs a
+ * shared plan without a matching export/import; NU_ECUDA for IPC failures
+ * (e.g. a blob from this same process). */
+int northup_tree_set_local(northup_tree_t t, int node);
+int northup_peer_export(northup_tree_t t, int64_t M, int64_t N, int64_t K,
+                        const northup_gemm_opts* opts, void* blob, uint64_t cap, uint64_t* len);
+int northup_peer_import(northup_tree_t t, int worker, const void* blob, uint64_t len);
+
 /* ------------------------------------------------------------ misc */
 const char* northup_last_error(void);
 int northup_version(void);

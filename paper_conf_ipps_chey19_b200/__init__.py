@@ -141,6 +141,10 @@ _SIGS = {
     "northup_partition_region": [_int, _i64, _i64, _i64, _int, ctypes.POINTER(_i64),
                                  ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i64)],
     "northup_file_tile_kpanels": [ctypes.c_char_p, ctypes.c_char_p, _i64, _i64, _i64],
+    "northup_tree_set_local": [_vp, _int],
+    "northup_peer_export": [_vp, _i64, _i64, _i64, ctypes.POINTER(GemmOpts), _vp, _u64,
+                            ctypes.POINTER(_u64)],
+    "northup_peer_import": [_vp, _int, _vp, _u64],
     "northup_version": [],
     "northup_device_count": [],
 }
@@ -359,6 +363,23 @@ class Tree:
 
     def finalize(self) -> None:
         check(lib().northup_tree_finalize(self.handle))
+
+    # -- multi-process siblings (one process per GPU)
+    def set_local(self, node: int) -> None:
+        """This process runs only HBM node `node` (before finalize)."""
+        check(lib().northup_tree_set_local(self.handle, node))
+
+    def peer_export(self, M: int, N: int, K: int, opts: GemmOpts | None = None) -> bytes:
+        """Plan the GEMM, allocate the local arena; CUDA IPC handles for the peers."""
+        n = ctypes.c_uint64()
+        o = ctypes.byref(opts) if opts else None
+        lib().northup_peer_export(self.handle, M, N, K, o, None, 0, ctypes.byref(n))
+        buf = ctypes.create_string_buffer(n.value)
+        check(lib().northup_peer_export(self.handle, M, N, K, o, buf, n.value, ctypes.byref(n)))
+        return buf.raw[: n.value]
+
+    def peer_import(self, worker: int, blob: bytes) -> None:
+        check(lib().northup_peer_import(self.handle, worker, blob, len(blob)))
 
     def destroy(self) -> None:
         if self.handle:

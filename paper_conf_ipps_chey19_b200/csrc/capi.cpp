@@ -63,7 +63,19 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
   if (A->tree != t || B->tree != t || C->tree != t) return fail(NU_EINVAL, "buffer from another tree");
   if (A->node != 0 || B->node != 0 || C->node != 0)
     return fail(NU_EINVAL, "A, B and C must live at the root node (level 0)");
-  const uint64_t need_a = 4ull * M * K, need_b = 4ull * K * N, need_c = 4ull * M * N;
+  // multi-process siblings pass only their own strips (northup_tree_set_local)
+  int64_t m = M, n = N;
+  if (t->local_node >= 0) {
+    const auto& ch = t->nodes[0].children;
+    const int G = static_cast<int>(ch.size());
+    const int idx = static_cast<int>(std::find(ch.begin(), ch.end(), t->local_node) - ch.begin());
+    int64_t r0, r1, c0, c1;
+    int rc = region_of(G, M, N, idx, &r0, &r1, &c0, &c1);
+    if (rc) return rc;
+    m = r1 - r0;
+    n = c1 - c0;
+  }
+  const uint64_t need_a = 4ull * m * K, need_b = 4ull * K * n, need_c = 4ull * m * n;
   if (A->bytes < need_a || B->bytes < need_b || C->bytes < need_c)
     return fail(NU_EINVAL, "buffer smaller than its matrix");
   if (o && o->replicate_result && t->nodes[0].storage == NU_FILE)
@@ -72,7 +84,7 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
   northup_stats* st = s ? s : &local;
   *st = northup_stats{};
   if (M == 0 || N == 0) return 0;
-  if (K == 0) return zero_root_c(t, C, M, N);
+  if (K == 0) return zero_root_c(t, C, m, n);
   if (t->nodes[0].storage == NU_FILE &&
       (A->storage != NU_FILE || B->storage != NU_FILE || C->storage != NU_FILE))
     return fail(NU_EINVAL, "a FILE root needs A, B and C as files (northup_open_file / alloc)");

@@ -41,6 +41,7 @@ int finalize_workers(northup_tree_s* t) {
   int ndev = northup_device_count();
   for (const Node& n : t->nodes) {
     if (n.storage != NU_HBM) continue;
+    if (t->local_node >= 0 && n.id != t->local_node) continue;   // run by a peer process
     if (n.phys >= ndev)
       return fail(NU_ECUDA, "HBM node %d names device %d but %d CUDA device(s) are visible", n.id,
                   n.phys, ndev);
@@ -90,7 +91,7 @@ static WorkerState* worker_for_node(northup_tree_s* t, int node) {
 
 // Make sure the HBM node's arena holds `bytes` (cudaMalloc on first use,
 // grown when a larger plan arrives; counted in the node's `used`).
-static int ensure_arena(northup_tree_s* t, int node, uint64_t bytes) {
+int ensure_arena(northup_tree_s* t, int node, uint64_t bytes) {
   Node& n = t->nodes[node];
   if (bytes == 0 || n.arena_bytes >= bytes) return 0;
   if (n.arena && !n.arena_owned)
@@ -141,8 +142,12 @@ struct RunCtx {
   std::vector<char*> base;             // per plan buffer (host/device pointers)
   std::vector<const northup_buf_s*> file;   // per plan buffer: file handle or NULL
   const std::vector<char>* needs_event;
+  const std::vector<char>* needs_remote;   // local op a peer process waits for
   const northup_gemm_opts* o;
   bool timing;
+  int local = -1;                          // multi-process siblings: the local worker
+  bool cross = false;                      // the plan has cross-sibling dependencies
+  uint32_t gen = 0;
   // cross-thread progress (FILE roots)
   std::mutex m;
   std::condition_variable cv;
@@ -210,6 +215,12 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
         continue;
       }
       cudaEvent_t ev = w->events[op.deps[d]];
+      if (q.worker != wi && c.local >= 0) {
+        // a sibling in another process: device-side wait on its flag word
+        int rc = stream_wait_flag(s, c.t->peers[q.worker].flags + 1 + op.deps[d], c.gen);
+        if (rc) return rc;
+        continue;
+      }
       if (q.worker != wi) {
         // another sibling's op (shared-staging pull, NEXT-1): wait until that
         // worker has recorded its event in this call, then wait on it on the
@@ -249,6 +260,26 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
       mark(c, c.issued, i);
     }
+    if (c.local >= 0 && (*c.needs_remote)[i]) {
+      int rc = stream_write_flag(s, c.t->flags + 1 + i, c.gen);
+      if (rc) return rc;
+    }
+  }
+  if (c.local >= 0 && c.cross) {
+    // device-side join: done word after all local streams, then wait for every
+    // sibling's done word, so no peer still reads this arena when we return
+    for (int k = 1; k < S_NUM; ++k) {
+      cudaEvent_t j = nullptr;
+      e = cudaEventCreateWithFlags(&j, cudaEventDisableTiming);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaEventCreate");
+      cudaEventRecord(j, w->streams[k]);
+      cudaStreamWaitEvent(w->streams[0], j, 0);
+      cudaEventDestroy(j);
+    }
+    int rc = stream_write_flag(w->streams[0], c.t->flags, c.gen);
+    for (int q = 0; q < P.num_workers && !rc; ++q)
+      if (q != wi) rc = stream_wait_flag(w->streams[0], c.t->peers[q].flags, c.gen);
+    if (rc) return rc;
   }
   if (capture_out) {
     std::vector<cudaEvent_t> joins;
@@ -390,12 +421,20 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   ctx.timing = o && o->collect_timing;
   ctx.base.resize(P.bufs.size(), nullptr);
   ctx.file.resize(P.bufs.size(), nullptr);
+  const int lw = local_worker(t, P);
+  if (lw == -2) return fail(NU_ESTATE, "the local node is not a worker of this plan");
+  ctx.local = lw;
   for (size_t i = 0; i < P.bufs.size(); ++i) {
     const PlanBuf& pb = P.bufs[i];
     northup_buf_s* ub = pb.kind == B_USER_A ? a : pb.kind == B_USER_B ? b : pb.kind == B_USER_C ? c : nullptr;
     if (ub) {
       ctx.base[i] = static_cast<char*>(ub->ptr);
       if (ub->storage == NU_FILE) ctx.file[i] = ub;
+      continue;
+    }
+    if (lw >= 0 && pb.worker != lw) {   // a sibling's arena (IPC-mapped, pulls only)
+      ctx.base[i] = pb.worker >= 0 && pb.worker < static_cast<int>(t->peers.size())
+                        ? t->peers[pb.worker].arena : nullptr;
       continue;
     }
     int rc = ensure_arena(t, pb.node, pb.bytes);
@@ -414,6 +453,21 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     has_io |= op.stream == S_IO;
   }
   ctx.needs_event = &needs;
+  ctx.cross = cross;
+  std::vector<char> needs_remote(P.ops.size(), 0);
+  ctx.needs_remote = &needs_remote;
+  if (lw >= 0 && cross) {
+    if (t->peer_key != peer_key_of(P.M, P.N, P.K, o) ||
+        static_cast<int>(t->peers.size()) != P.num_workers)
+      return fail(NU_ESTATE, "multi-process siblings: run northup_peer_export/import for this GEMM first");
+    for (int q = 0; q < P.num_workers; ++q)
+      if (q != lw && !t->peers[q].flags)
+        return fail(NU_ESTATE, "multi-process siblings: worker %d was not imported", q);
+    for (const northup_op& op : P.ops)
+      for (int d = 0; d < op.ndeps; ++d)
+        if (op.worker != lw && P.ops[op.deps[d]].worker == lw) needs_remote[op.deps[d]] = 1;
+    ctx.gen = ++t->gen;
+  }
   ctx.issued.assign(P.ops.size(), 0);
   if (ctx.timing) t->timeline.clear();
   ctx.io_done.assign(P.ops.size(), 0);
@@ -422,7 +476,7 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   // CUDA-graph mode: replay the captured op lists of an identical earlier call
   // (per-worker graphs cannot hold another worker's events: no graphs with
   // shared staging)
-  const bool use_graph = o && o->graph && !has_io && !cross && !ctx.timing;
+  const bool use_graph = o && o->graph && !has_io && !cross && !ctx.timing && lw < 0;
   std::vector<int64_t> key;
   if (use_graph) {
     key = graph_key(P, ctx.base, o);
@@ -466,11 +520,14 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
       ctx.cv.notify_all();
     }
   };
-  if (W == 1 && !has_io) {
-    worker_body(0);
+  std::vector<int> mine;
+  for (int wi = 0; wi < W; ++wi)
+    if (lw < 0 || wi == lw) mine.push_back(wi);
+  if (mine.size() == 1 && !has_io) {
+    worker_body(mine[0]);
   } else {
     std::vector<std::thread> th;
-    for (int wi = 0; wi < W; ++wi) th.emplace_back(worker_body, wi);
+    for (int wi : mine) th.emplace_back(worker_body, wi);
     if (has_io) th.emplace_back(io_body);
     for (auto& x : th) x.join();
   }

@@ -76,6 +76,22 @@ struct northup_tree_s {
   std::vector<std::array<float, 5>> timeline;   // last collect_timing run (debug)
   std::vector<void*> graph_execs;      // cudaGraphExec_t per worker (opts->graph)
   std::vector<int64_t> graph_key;      // the GEMM they were captured for
+  // Multi-process siblings (northup_tree_set_local, peer.cpp): this process
+  // runs only HBM node `local_node`; the other siblings' arenas and flag words
+  // are mapped through CUDA IPC.  Cross-sibling dependencies become device-side
+  // waits on the producer's flag word (cuStreamWaitValue32 >= gen), written
+  // by the producer after the op (cuStreamWriteValue32).
+  int local_node = -1;
+  struct Peer {
+    char* arena = nullptr;       // IPC-mapped arena of that sibling
+    uint32_t* flags = nullptr;   // IPC-mapped flag words of that sibling
+  };
+  std::vector<Peer> peers;             // per plan worker
+  uint32_t* flags = nullptr;           // this process's flag words: [0] = done, [1 + op] = op
+  uint64_t flags_cap = 0;              // words
+  std::vector<void*> flag_graveyard;   // outgrown flag buffers (peers may still map them)
+  uint32_t gen = 0;                    // generation of the current call (monotonic)
+  std::vector<int64_t> peer_key;       // the GEMM the peers were exported/imported for
 };
 
 namespace nu {
@@ -128,6 +144,13 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,
                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
 int finalize_workers(northup_tree_s* t);
+int ensure_arena(northup_tree_s* t, int node, uint64_t bytes);
+// Multi-process siblings (peer.cpp)
+std::vector<int64_t> peer_key_of(int64_t M, int64_t N, int64_t K, const northup_gemm_opts* o);
+int local_worker(const northup_tree_s* t, const Plan& P);   // -1 when every worker is local
+int stream_wait_flag(cudaStream_t s, const uint32_t* addr, uint32_t gen);
+int stream_write_flag(cudaStream_t s, uint32_t* addr, uint32_t gen);
+void destroy_peers(northup_tree_s* t);
 int gather_replicas(northup_tree_s* t, const Plan& P, northup_buf_s* C, northup_stats* st);
 void destroy_nccl(northup_tree_s* t);
 void destroy_graphs(northup_tree_s* t);

@@ -215,6 +215,10 @@ struct EdgeCtx {
   // A panel and 1/b_share of each B panel over PCIe, its row / column peers
   // the rest, and pulls the other pieces from them over NVLink.
   int a_share = 1, b_share = 1;
+  // Origin of the region in the root buffers' addressing: (r0, c0) for a
+  // whole-problem root; (0, 0) with ldb = ldc = region width when the root
+  // buffers hold only this sibling's strips (multi-process siblings).
+  int64_t ar0 = 0, ac0 = 0;
 };
 
 // ---------------------------------------------------------------- S2
@@ -408,7 +412,7 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
     const int64_t bm = std::min(s.bm, m - i0);
     for (int64_t j0 = 0; j0 < n; j0 += s.bn) {
       const int64_t bn = std::min(s.bn, n - j0);
-      const int64_t gr = x.r0 + i0, gc = x.c0 + j0;   // global row/col of the block
+      const int64_t gr = x.ar0 + i0, gc = x.ac0 + j0;   // root row/col of the block
       // ---- main phase: K panels [0, kmain)
       const int64_t npan = kmain > 0 ? cdiv(kmain, s.bk) : 0;
       const int64_t ntail_pieces = s.tail > 0 ? cdiv(s.tail, s.bk) : 0;
@@ -600,7 +604,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
       auto load_tail_piece = [&](int64_t pc) {
         const int64_t k0 = kmain + pc * s.bk, kk = std::min(s.bk, K - k0);
         Side sb = side(false, Y.offBT + (k0 - kmain) * Y.ldBs, Y.ldBs, kk, bn,
-                       [&](const EdgeCtx& x) { return k0 * ldb + x.c0 + j0; });
+                       [&](const EdgeCtx& x) { return k0 * ldb + x.ac0 + j0; });
         load(sb);
         pull(sb);
       };
@@ -608,9 +612,9 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
         const int sl = panel_it % kSlots;
         const int64_t k0 = p * s.bk, kk = std::min(s.bk, kmain - k0);
         Side sa = side(true, Y.offSA[sl], Y.ldA, bm, kk,
-                       [&](const EdgeCtx& x) { return (x.r0 + i0) * lda + k0; });
+                       [&](const EdgeCtx& x) { return (x.ar0 + i0) * lda + k0; });
         Side sb = side(false, Y.offSB[sl], Y.ldBs, kk, bn,
-                       [&](const EdgeCtx& x) { return k0 * ldb + x.c0 + j0; });
+                       [&](const EdgeCtx& x) { return k0 * ldb + x.ac0 + j0; });
         load(sa);
         load(sb);
         pull(sa);
@@ -644,7 +648,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
           rr = next_strip(bm, r, s.sr);
           const int sl = strip_it % kSlots;
           Side sa = side(true, Y.offAT[sl], Y.ldAt, rr, s.tail,
-                         [&](const EdgeCtx& x) { return (x.r0 + i0 + r) * lda + kmain; });
+                         [&](const EdgeCtx& x) { return (x.ar0 + i0 + r) * lda + kmain; });
           load(sa);
           pull(sa);
           for (int w = 0; w < G; ++w) {
@@ -655,7 +659,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
                    {{ar, Y.offAT[sl], Y.ldAt, rr, s.tail, false}, {ar, Y.offBT, Y.ldBs, s.tail, bn, false},
                     {ar, co, Y.ldC, rr, bn, true}});
             st->leaf_launches++;
-            const int64_t dst = (xs[w].r0 + i0 + r) * ldc + xs[w].c0 + j0;
+            const int64_t dst = (xs[w].ar0 + i0 + r) * ldc + xs[w].ac0 + j0;
             B.emit(make_copy(w, S_D2H, ar, co, Y.ldC, x0.C, dst, ldc, rr, bn),
                    {{ar, co, Y.ldC, rr, bn, false}, {x0.C, dst, ldc, rr, bn, true}});
             st->bytes_d2h += 4ull * rr * bn;
@@ -663,7 +667,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
         }
       } else {
         for (int w = 0; w < G; ++w) {
-          const int64_t dst = (xs[w].r0 + i0) * ldc + xs[w].c0 + j0;
+          const int64_t dst = (xs[w].ar0 + i0) * ldc + xs[w].ac0 + j0;
           B.emit(make_copy(w, S_D2H, L[w].arena, Y.offC, Y.ldC, x0.C, dst, ldc, bm, bn),
                  {{L[w].arena, Y.offC, Y.ldC, bm, bn, false}, {x0.C, dst, ldc, bm, bn, true}});
           st->bytes_d2h += 4ull * bm * bn;
@@ -710,7 +714,7 @@ int build_s1(const EdgeCtx& x, northup_stats* st) {
   int shard = 0, cblk = 0, pit = 0;
   for (int64_t i0 = 0; i0 < m; i0 += bm, ++shard) {
     const int64_t rm = std::min(bm, m - i0);
-    const int64_t gr = x.r0 + i0;
+    const int64_t gr = x.ar0 + i0;
     const int as = shard & 1;
     // row shard m moves to level l+1 once and stays
     B.emit(make_copy(w, S_H2D, x.A, gr * x.lda, x.lda, arena, offAs[as], ldAs, rm, K),
@@ -718,7 +722,7 @@ int build_s1(const EdgeCtx& x, northup_stats* st) {
     st->bytes_h2d += static_cast<uint64_t>(rm) * K * 4;
     for (int64_t j0 = 0; j0 < n; j0 += bn, ++cblk) {
       const int64_t cn = std::min(bn, n - j0);
-      const int64_t gc = x.c0 + j0;
+      const int64_t gc = x.ac0 + j0;
       const int cb = cblk & 1;
       for (int64_t k0 = 0; k0 < K; k0 += bk, ++pit) {
         const int64_t kk = std::min(bk, K - k0);
@@ -1022,6 +1026,14 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     x.ldc = N;
     rc = region_of(G, M, N, w, &x.r0, &x.r1, &x.c0, &x.c1);
     if (rc) return rc;
+    x.ar0 = x.r0;
+    x.ac0 = x.c0;
+    if (t->local_node >= 0) {
+      // multi-process siblings: every process passes only its own strips
+      // (A rows [r0, r1) x K, B K x [c0, c1), C region), row-major and dense
+      x.ar0 = x.ac0 = 0;
+      x.ldb = x.ldc = x.c1 - x.c0;
+    }
     x.K = K;
     x.cap = t->nodes[hbm[w]].capacity;
     x.kc = P.kc;

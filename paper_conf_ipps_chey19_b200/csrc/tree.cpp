@@ -160,6 +160,18 @@ int northup_tree_set_arena(northup_tree_t t, int node, void* dev_ptr, uint64_t b
   return 0;
 }
 
+int northup_tree_set_local(northup_tree_t t, int node) {
+  if (!t) return fail(NU_EINVAL, "tree is NULL");
+  if (t->finalized) return fail(NU_ESTATE, "set_local must precede finalize");
+  if (!valid_node(t, node) || t->nodes[node].storage != NU_HBM)
+    return fail(NU_EINVAL, "node %d is not an HBM node", node);
+  const int root = 0;
+  if (t->nodes[root].storage != NU_HOST || t->nodes[node].parent != root)
+    return fail(NU_ENOTSUP, "multi-process siblings need a HOST root with HBM children");
+  t->local_node = node;
+  return 0;
+}
+
 int northup_tree_finalize(northup_tree_t t) {
   if (!t) return fail(NU_EINVAL, "tree is NULL");
   if (t->finalized) return fail(NU_ESTATE, "tree already finalized");
@@ -178,6 +190,7 @@ int northup_tree_destroy(northup_tree_t t) {
   while (!t->bufs.empty()) northup_release(t, t->bufs.back());
   destroy_nccl(t);
   destroy_graphs(t);
+  destroy_peers(t);
   destroy_workers(t);
   for (Node& n : t->nodes) {
     if (n.arena_owned && n.arena) {

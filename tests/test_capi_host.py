@@ -386,3 +386,78 @@ def test_shared_staging_falls_back_for_ragged_regions():
     p = t.plan(301, 200, 90, nu.make_opts(k_chunk=32))     # 1 x 3 grid, 200 = 67+67+66
     assert p.stats()["shared_staging"] == 0
     t.destroy()
+
+
+def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
+    """Replay a multi-process-siblings plan (northup_tree_set_local): worker w's
+    user-buffer ops address only ITS strips (A rows, B columns, C region with
+    region-local leading dimensions); arenas are shared (pulls read peers')."""
+    bufs, ops = plan.bufs(), plan.ops()
+    strips = []
+    for w in range(G):
+        r0, r1, c0, c1 = nu.partition_region(G, M, N, K, w)
+        strips.append({0: A[r0:r1].astype(np.float64).ravel().copy(),
+                       1: B[:, c0:c1].astype(np.float64).ravel().copy(),
+                       2: np.full((r1 - r0) * (c1 - c0), np.nan), "reg": (r0, r1, c0, c1)})
+    arenas = {i: np.full(b["bytes"] // 4, np.nan) for i, b in enumerate(bufs) if b["kind"] >= 3}
+
+    def mem(w, i):
+        return strips[w][bufs[i]["kind"]] if bufs[i]["kind"] < 3 else arenas[i]
+
+    def view(w, buf, off, ld, rows, cols):
+        return np.lib.stride_tricks.as_strided(mem(w, buf)[off:], shape=(rows, cols),
+                                               strides=(ld * 8, 8), writeable=True)
+
+    queues = {}
+    for i, op in enumerate(ops):
+        queues.setdefault((op["worker"], op["stream"]), []).append(i)
+    done = set()
+    while len(done) < len(ops):
+        ready = [q for q in queues.values() if q and all(d in done for d in ops[q[0]]["deps"])]
+        assert ready
+        i = rng.choice(ready).pop(0)
+        op, w = ops[i], ops[i]["worker"]
+        if op["op"] == nu.NU_OP_COPY:
+            view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
+                view(w, op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
+        elif op["op"] == nu.NU_OP_LEAF:
+            a = view(w, op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
+            b = view(w, op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"])
+            c = view(w, op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])
+            c[...] = (c + a @ b) if op["accumulate"] else a @ b
+        done.add(i)
+    C = np.full((M, N), np.nan)
+    for s in strips:
+        r0, r1, c0, c1 = s["reg"]
+        C[r0:r1, c0:c1] = s[2].reshape(r1 - r0, c1 - c0)
+    return C
+
+
+@pytest.mark.parametrize("M,N,K,G,shared", [(512, 512, 640, 2, 0), (512, 512, 640, 4, 0),
+                                             (1024, 512, 1000, 8, 0), (300, 200, 130, 3, -1),
+                                             (512, 256, 384, 4, -1)])
+def test_multiprocess_sibling_plan_uses_local_strips(M, N, K, G, shared):
+    """northup_tree_set_local: the same plan on every process, each sibling's
+    root ops addressing its own strips (region-local leading dimensions);
+    replayed with per-process strips it computes A.B exactly."""
+    A = nugen.fill(M, K, 7, 1, "int")
+    B = nugen.fill(K, N, 7, 2, "int")
+    t, hbm = nu.host_tree(G)
+    t.set_local(hbm[G - 1])
+    p = t.plan(M, N, K, nu.make_opts(k_chunk=64, shared_staging=shared))
+    assert p.stats()["shared_staging"] == (1 if shared == 0 else 0)
+    for seed in range(3):
+        C = simulate_local(p, A, B, M, N, K, G, random.Random(seed))
+        assert np.array_equal(C, A.astype(np.float64) @ B.astype(np.float64))
+    t.destroy()
+
+
+def test_set_local_errors():
+    t, hbm = nu.host_tree(2)
+    with pytest.raises(nu.NorthupError):
+        t.set_local(0)                       # the HOST root is not an HBM node
+    t.set_local(hbm[1])
+    with pytest.raises(nu.NorthupError) as e:
+        t.peer_export(64, 64, 64)            # not finalized
+    assert e.value.code == nu.NU_ESTATE
+    t.destroy()

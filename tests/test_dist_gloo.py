@@ -52,3 +52,43 @@ def test_partitioned_gemm_and_gather_gloo(world, M, N, K):
     ref = A.astype(np.float64) @ B.astype(np.float64)
     for r in range(world):
         assert np.array_equal(outs[r], ref)
+
+
+def _plan_rank(rank, world, port, M, N, K, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import hashlib
+
+        import paper_conf_ipps_chey19_b200 as nu
+        t, hbm = nu.host_tree(world)
+        t.set_local(hbm[rank])          # multi-process siblings: this rank's node
+        p = t.plan(M, N, K, nu.make_opts(k_chunk=64))
+        ops = p.ops()
+        h = hashlib.sha256(repr([sorted(o.items()) for o in ops]).encode()).hexdigest()
+        t.destroy()
+        hs = [None] * world
+        dist.all_gather_object(hs, h)
+        q.put((rank, hs, p.stats()["shared_staging"]))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_multiprocess_siblings_plan_identically_gloo(world):
+    """The cross-process protocol of multi-process siblings (peer flag words
+    indexed by op) needs every rank to build the same op list whatever its
+    local node: checked by all-gathering a hash of each rank's plan."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29500 + random.randint(2001, 4000)
+    procs = [ctx.Process(target=_plan_rank, args=(r, world, port, 512, 512, 640, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    outs = dict((r, (hs, sh)) for r, hs, sh in (q.get(timeout=300) for _ in range(world)))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    hs0 = outs[0][0]
+    assert len(set(hs0)) == 1 and all(outs[r][0] == hs0 for r in range(world))
+    assert all(outs[r][1] == 1 for r in range(world))
