@@ -17,10 +17,11 @@ import subprocess
 
 import numpy as np
 
-UNIFORM, INT, EYE, ONES, RANK1, ZEROS = 0, 1, 2, 3, 4, 5
+UNIFORM, INT, EYE, ONES, RANK1, ZEROS, TEMP, POWER = 0, 1, 2, 3, 4, 5, 6, 7
 KINDS = {"uniform": UNIFORM, "int": INT, "eye": EYE, "ones": ONES,
-         "rank1": RANK1, "zeros": ZEROS}
+         "rank1": RANK1, "zeros": ZEROS, "temp": TEMP, "power": POWER}
 MAT_A, MAT_B = 1, 2
+MAT_T, MAT_P = 3, 4      # HotSpot-2D temperature and power grids (NEXT-3)
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libnugen.so")
@@ -100,11 +101,16 @@ def fill_numpy(rows: int, cols: int, seed: int, mat: int, kind="uniform",
     j = np.arange(j0, j0 + cols, dtype=np.uint64)[None, :]
     with np.errstate(over="ignore"):
         base = np.uint64((seed * _GOLDEN) & _M64) ^ np.uint64((mat << 56) & _M64)
-        if k in (UNIFORM, INT):
+        if k in (UNIFORM, INT, TEMP, POWER):
             h = _splitmix64_np(base ^ (i * np.uint64(ncols) + j))
-            if k == UNIFORM:
+            if k in (UNIFORM, TEMP, POWER):
                 q = (h >> np.uint64(40)).astype(np.int64) - (1 << 23)
-                return (q.astype(np.float64) * 2.0 ** -23).astype(np.float32)
+                u = q.astype(np.float64) * 2.0 ** -23
+                if k == TEMP:
+                    return (330.0 + 10.0 * u).astype(np.float32)
+                if k == POWER:
+                    return (0.25 + 0.25 * u).astype(np.float32)
+                return u.astype(np.float32)
             return ((h % np.uint64(17)).astype(np.int64) - 8).astype(np.float32)
         if k == EYE:
             return (i == j).astype(np.float32)
@@ -131,9 +137,14 @@ def entry_py(seed: int, mat: int, kind, ncols: int, i: int, j: int) -> float:
     """Pure-Python definition of one entry (brute force, for pinning)."""
     k = _kind(kind)
     base = ((seed * _GOLDEN) & _M64) ^ ((mat << 56) & _M64)
-    if k == UNIFORM:
+    if k in (UNIFORM, TEMP, POWER):
         h = _splitmix64_py(base ^ ((i * ncols + j) & _M64))
-        return float(((h >> 40) - (1 << 23)) * 2.0 ** -23)
+        u = float(((h >> 40) - (1 << 23)) * 2.0 ** -23)
+        if k == TEMP:
+            return float(np.float32(330.0 + 10.0 * u))
+        if k == POWER:
+            return float(np.float32(0.25 + 0.25 * u))
+        return u
     if k == INT:
         h = _splitmix64_py(base ^ ((i * ncols + j) & _M64))
         return float(h % 17 - 8)

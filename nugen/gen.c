@@ -16,6 +16,8 @@
  *   rank1   : u(i) * v(j), u(i) = (h(seed,mat,i,0x0F0F..)&7)-3,
  *                          v(j) = (h(seed,mat^0x40,j,0x0F0F..)&7)-3  (small ints)
  *   zeros   : 0
+ *   temp    : (float)(330 + 10 u)   HotSpot-2D temperature grid, K   (u = uniform)
+ *   power   : (float)(0.25 + 0.25 u) HotSpot-2D power grid, in [0, 0.5) (exact fp32)
  *
  * The paper's workload is "16k x 16k and 32k x 32k float matrices" (PAPER.md
  * P:349, §V-A); values are unspecified there, so the distribution is ours.
@@ -29,6 +31,8 @@
 #define NUGEN_ONES 3
 #define NUGEN_RANK1 4
 #define NUGEN_ZEROS 5
+#define NUGEN_TEMP 6
+#define NUGEN_POWER 7
 
 static inline uint64_t splitmix64(uint64_t z) {
   z += 0x9E3779B97F4A7C15ULL;
@@ -48,6 +52,12 @@ static inline float nugen_value(int kind, uint64_t seed, uint64_t mat,
       uint64_t h = nugen_hash(seed, mat, (uint64_t)i * (uint64_t)ncols + (uint64_t)j);
       int64_t q = (int64_t)(h >> 40) - (1LL << 23);
       return (float)q * (1.0f / 8388608.0f);
+    }
+    case NUGEN_TEMP:
+    case NUGEN_POWER: {
+      uint64_t h = nugen_hash(seed, mat, (uint64_t)i * (uint64_t)ncols + (uint64_t)j);
+      double u = (double)((int64_t)(h >> 40) - (1LL << 23)) * (1.0 / 8388608.0);
+      return kind == NUGEN_TEMP ? (float)(330.0 + 10.0 * u) : (float)(0.25 + 0.25 * u);
     }
     case NUGEN_INT: {
       uint64_t h = nugen_hash(seed, mat, (uint64_t)i * (uint64_t)ncols + (uint64_t)j);

@@ -13,6 +13,9 @@ code with the CUDA path (paper_conf_ipps_chey19_b200/) and never imports it.
   * checks           — row/column norms, the normwise error of BASELINE.json
                        (max |C - C_ref| / (||A_i,:||_2 ||B_:,j||_2)), sampled
                        entries and Freivalds' check for full-size configs.
+  * `oracle.hotspot` — HotSpot-2D, the paper's stencil case study (§IV-B,
+                       P:307-325; S§8(f) NEXT-3): the update, [18]'s explicit
+                       edge cases, the blocked recursion, the fp32 bound.
 """
 from __future__ import annotations
 

@@ -6,7 +6,7 @@ import pytest
 import nugen
 
 
-@pytest.mark.parametrize("kind", ["uniform", "int", "eye", "ones", "rank1", "zeros"])
+@pytest.mark.parametrize("kind", ["uniform", "int", "eye", "ones", "rank1", "zeros", "temp", "power"])
 def test_three_implementations_agree(kind):
     rows, cols, ncols, i0, j0 = 13, 37, 101, 5, 17
     c = nugen.fill(rows, cols, seed=3, mat=1, kind=kind, i0=i0, j0=j0, ncols=ncols)
@@ -41,3 +41,12 @@ def test_a_and_b_differ_and_seeds_differ():
     b = nugen.fill(16, 16, seed=1, mat=nugen.MAT_B)
     a2 = nugen.fill(16, 16, seed=2, mat=nugen.MAT_A)
     assert not np.array_equal(a, b) and not np.array_equal(a, a2)
+
+
+def test_hotspot_grid_ranges():
+    t = nugen.fill(128, 256, seed=6, mat=nugen.MAT_T, kind="temp").astype(np.float64)
+    p = nugen.fill(128, 256, seed=6, mat=nugen.MAT_P, kind="power").astype(np.float64)
+    assert t.min() >= 320.0 and t.max() < 340.0 and abs(t.mean() - 330.0) < 0.2
+    assert p.min() >= 0.0 and p.max() < 0.5
+    q = p * 2.0 ** 25
+    assert np.array_equal(q, np.round(q))           # exact fp32, 2^-25 granularity
