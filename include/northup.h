@@ -251,6 +251,9 @@ int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, 
 #define NU_OP_ZERO 2
 #define NU_OP_IO_READ 3  /* file -> DRAM staging (pread), host I/O thread */
 #define NU_OP_IO_WRITE 4 /* DRAM staging -> file (pwrite), host I/O thread */
+#define NU_OP_STENCIL 5  /* HotSpot-2D leaf (northup_hotspot): a_* = temperature in, b_* = power,
+                            c_* = temperature out, all shaped like the m x n window; k = iterations;
+                            src_off / dst_off = the window's grid row / column; rows x cols = grid */
 typedef struct {
   int op;
   int worker;   /* GPU worker index (0 .. num_gpus-1) */
@@ -330,6 +333,56 @@ int northup_tree_set_local(northup_tree_t t, int node);
 int northup_peer_export(northup_tree_t t, int64_t M, int64_t N, int64_t K,
                         const northup_gemm_opts* opts, void* blob, uint64_t cap, uint64_t* len);
 int northup_peer_import(northup_tree_t t, int worker, const void* blob, uint64_t len);
+
+/* ------------------------------------------ HotSpot-2D stencil (S§8(f) NEXT-3) */
+/* The paper's second case study (§IV-B): HotSpot-2D [18] thermal
+ * simulation over the same tree.  One iteration updates every cell (r, c) of
+ * the rows x cols fp32 temperature grid T with power grid P:
+ *   T'[r,c] = T + cap_1 * (P + (T[r+1,c] + T[r-1,c] - 2T) * ry_1
+ *                            + (T[r,c+1] + T[r,c-1] - 2T) * rx_1 + (amb - T) * rz_1)
+ * with out-of-grid neighbours replaced by the cell itself (RH1), in
+ * fp32, evaluated left to right with round-to-nearest and no contraction. */
+typedef struct {
+  float cap_1, rx_1, ry_1, rz_1, amb;
+} northup_hotspot_coeffs;
+
+/* [18]'s chip model with the cell pitch fixed at its 1024-cell value (reading
+ * RH2, so the explicit scheme is stable at any grid size), rounded to fp32. */
+int northup_hotspot_default_coeffs(int64_t rows, int64_t cols, northup_hotspot_coeffs* out);
+
+typedef struct {
+  int64_t block;      /* HBM-level block edge in cells ("8k x 8k blocking"), 0 = planner */
+  int64_t halo;       /* iterations per visit of a block to HBM = its border width, 0 = planner */
+  int leaf_iters;     /* iterations per leaf launch (1..8), 0 = 8 */
+  int collect_timing; /* 1: per-stream busy times into the stats */
+  int reserved[4];
+} northup_hotspot_opts;
+
+/* The leaf on device pointers: `iters` (1..8) iterations on the wm x wn window
+ * whose top-left cell is (gy0, gx0) of a rows x cols grid.  tin/pw/tout are
+ * window-shaped (leading dimensions ldt/ldp/ldo >= wn).  Writes only the valid
+ * region of tout: the window shrunk by `iters` cells on each side that is not
+ * a grid edge.  Asynchronous on `stream` (current device).  NU_EINVAL for a
+ * window outside the grid or iters outside 1..8. */
+int northup_hotspot_leaf(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
+                         int64_t ldo, int64_t wm, int64_t wn, int64_t gy0, int64_t gx0,
+                         int64_t rows, int64_t cols, int iters, const northup_hotspot_coeffs* k,
+                         void* stream);
+
+/* `iters` iterations of HotSpot-2D on the tree: T (input, unchanged), P and
+ * Tout, each rows x cols fp32 row-major, live at the ROOT (pinned host, or
+ * device memory for a single-node HBM tree).  Synchronous.  A HOST root splits
+ * the grid into blocks that move down to the HBM siblings with a border of
+ * `halo` cells (the four borders of P:317, strided rows copied by the DMA
+ * engine), iterate `halo` times there and move back up; passes alternate
+ * between Tout and a library-owned pinned scratch grid.  k NULL = defaults.
+ * iters == 0 copies T to Tout. */
+int northup_hotspot(northup_tree_t t, northup_buf_t T, northup_buf_t P, northup_buf_t Tout,
+                    int64_t rows, int64_t cols, int64_t iters, const northup_hotspot_coeffs* k,
+                    const northup_hotspot_opts* opts, northup_stats* stats);
+/* Build (not run) the HotSpot-2D plan; introspect it with northup_plan_*. */
+int northup_hotspot_plan(northup_tree_t t, int64_t rows, int64_t cols, int64_t iters,
+                         const northup_hotspot_opts* opts, northup_plan_t* out);
 
 /* ------------------------------------------------------------ misc */
 const char* northup_last_error(void);

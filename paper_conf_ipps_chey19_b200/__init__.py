@@ -23,7 +23,7 @@ NU_OK, NU_EINVAL, NU_ENOMEM, NU_EIO, NU_ECUDA, NU_ENCCL, NU_ESTATE, NU_ENOTSUP =
 NU_FILE, NU_HOST, NU_HBM, NU_SMEM = 0, 1, 2, 3
 NU_PROC_NONE, NU_PROC_SM100 = 0, 1
 NU_SCHED_AUTO, NU_SCHED_S1, NU_SCHED_S2 = 0, 1, 2
-NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO, NU_OP_IO_READ, NU_OP_IO_WRITE = 0, 1, 2, 3, 4
+NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO, NU_OP_IO_READ, NU_OP_IO_WRITE, NU_OP_STENCIL = 0, 1, 2, 3, 4, 5
 STREAM_NAMES = {0: "h2d", 1: "compute", 2: "d2h", 3: "io", 4: "d2d"}
 STATUS_NAMES = {0: "NU_OK", -1: "NU_EINVAL", -2: "NU_ENOMEM", -3: "NU_EIO", -4: "NU_ECUDA",
                 -5: "NU_ENCCL", -6: "NU_ESTATE", -7: "NU_ENOTSUP"}
@@ -69,6 +69,16 @@ class Stats(ctypes.Structure):
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class HotspotCoeffs(ctypes.Structure):
+    _fields_ = [("cap_1", ctypes.c_float), ("rx_1", ctypes.c_float), ("ry_1", ctypes.c_float),
+                ("rz_1", ctypes.c_float), ("amb", ctypes.c_float)]
+
+
+class HotspotOpts(ctypes.Structure):
+    _fields_ = [("block", ctypes.c_int64), ("halo", ctypes.c_int64), ("leaf_iters", ctypes.c_int),
+                ("collect_timing", ctypes.c_int), ("reserved", ctypes.c_int * 4)]
 
 
 class Op(ctypes.Structure):
@@ -145,6 +155,12 @@ _SIGS = {
     "northup_peer_export": [_vp, _i64, _i64, _i64, ctypes.POINTER(GemmOpts), _vp, _u64,
                             ctypes.POINTER(_u64)],
     "northup_peer_import": [_vp, _int, _vp, _u64],
+    "northup_hotspot_default_coeffs": [_i64, _i64, ctypes.POINTER(HotspotCoeffs)],
+    "northup_hotspot_leaf": [_vp, _i64, _vp, _i64, _vp, _i64, _i64, _i64, _i64, _i64, _i64, _i64,
+                             _int, ctypes.POINTER(HotspotCoeffs), _vp],
+    "northup_hotspot": [_vp, _vp, _vp, _vp, _i64, _i64, _i64, ctypes.POINTER(HotspotCoeffs),
+                        ctypes.POINTER(HotspotOpts), ctypes.POINTER(Stats)],
+    "northup_hotspot_plan": [_vp, _i64, _i64, _i64, ctypes.POINTER(HotspotOpts), _vp],
     "northup_version": [],
     "northup_device_count": [],
 }
@@ -226,6 +242,38 @@ def leaf_gemm(A, B, C, accumulate: bool = False, k_chunk: int = 0, npass: int = 
                       npass, stream)
 
 
+def hotspot_coeffs(rows: int, cols: int) -> HotspotCoeffs:
+    """northup_hotspot_default_coeffs (RH1/RH2), fp32."""
+    k = HotspotCoeffs()
+    check(lib().northup_hotspot_default_coeffs(rows, cols, ctypes.byref(k)))
+    return k
+
+
+def hotspot_opts(block: int = 0, halo: int = 0, leaf_iters: int = 0,
+                 collect_timing: bool = False) -> HotspotOpts:
+    o = HotspotOpts()
+    o.block, o.halo, o.leaf_iters, o.collect_timing = block, halo, leaf_iters, int(collect_timing)
+    return o
+
+
+def hotspot_leaf(tin, pw, tout, iters: int, gy0: int = 0, gx0: int = 0, rows: int | None = None,
+                 cols: int | None = None, coeffs: HotspotCoeffs | None = None, stream=None) -> None:
+    """The HotSpot-2D leaf on window-shaped fp32 CUDA tensors (row-major views)."""
+    wm, wn = tin.shape
+    rows = wm if rows is None else rows
+    cols = wn if cols is None else cols
+    for x in (tin, pw, tout):
+        if not x.is_cuda or x.dtype.itemsize != 4 or tuple(x.shape) != (wm, wn) or (x.numel() and x.stride(1) != 1):
+            raise NorthupError(NU_EINVAL, "window-shaped row-major fp32 CUDA tensors required")
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream(tin.device)
+    check(lib().northup_hotspot_leaf(tin.data_ptr(), tin.stride(0), pw.data_ptr(), pw.stride(0),
+                                     tout.data_ptr(), tout.stride(0), wm, wn, gy0, gx0, rows, cols,
+                                     iters, ctypes.byref(coeffs) if coeffs else None,
+                                     _stream_ptr(stream)))
+
+
 def file_tile_kpanels(src: str, dst: str, M: int, K: int, panel_k: int) -> None:
     """R15 preprocessing: row-major A file -> K-panel-major file."""
     check(lib().northup_file_tile_kpanels(src.encode(), dst.encode(), M, K, panel_k))
@@ -285,10 +333,10 @@ class Buf:
 class Plan:
     """Host-only plan introspection (northup_plan_*)."""
 
-    def __init__(self, tree: "Tree", M: int, N: int, K: int, opts: GemmOpts | None = None):
+    def __init__(self, tree: "Tree", M: int, N: int, K: int, opts=None, hotspot: bool = False):
         h = ctypes.c_void_p()
-        check(lib().northup_plan_create(tree.handle, M, N, K,
-                                        ctypes.byref(opts) if opts else None, ctypes.byref(h)))
+        create = lib().northup_hotspot_plan if hotspot else lib().northup_plan_create
+        check(create(tree.handle, M, N, K, ctypes.byref(opts) if opts else None, ctypes.byref(h)))
         self.handle = h.value
 
     def ops(self) -> list[dict]:
@@ -491,6 +539,18 @@ class Tree:
 
     def plan(self, M: int, N: int, K: int, opts: GemmOpts | None = None) -> Plan:
         return Plan(self, M, N, K, opts)
+
+    # -- HotSpot-2D (NEXT-3)
+    def hotspot(self, T: Buf, P: Buf, Tout: Buf, rows: int, cols: int, iters: int,
+                opts: HotspotOpts | None = None, coeffs: HotspotCoeffs | None = None) -> dict:
+        st = Stats()
+        check(lib().northup_hotspot(self.handle, T.handle, P.handle, Tout.handle, rows, cols, iters,
+                                    ctypes.byref(coeffs) if coeffs else None,
+                                    ctypes.byref(opts) if opts else None, ctypes.byref(st)))
+        return st.as_dict()
+
+    def hotspot_plan(self, rows: int, cols: int, iters: int, opts: HotspotOpts | None = None) -> "Plan":
+        return Plan(self, rows, cols, iters, opts, hotspot=True)
 
 
 def host_tree(num_gpus: int = 1, hbm_capacity: int = 0, smem_leaf: bool = True,

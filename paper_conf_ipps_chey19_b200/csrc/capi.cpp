@@ -13,9 +13,6 @@
 
 using namespace nu;
 
-struct northup_plan_s {
-  Plan plan;
-};
 
 static double now_ms() {
   using namespace std::chrono;

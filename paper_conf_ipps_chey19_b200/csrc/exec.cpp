@@ -249,6 +249,13 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       int rc = leaf_gemm_launch(a, op.lda, b, op.ldb, cc, op.ldc, op.m, op.n, op.k, op.accumulate,
                                 P.kc, P.npass, s);
       if (rc) return rc;
+    } else if (op.op == NU_OP_STENCIL) {
+      const float* tin = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);
+      const float* pw = reinterpret_cast<const float*>(c.base[op.b_buf] + op.b_off * 4);
+      float* tout = reinterpret_cast<float*>(c.base[op.c_buf] + op.c_off * 4);
+      int rc = hotspot_launch(tin, op.lda, pw, op.ldb, tout, op.ldc, op.m, op.n, op.src_off, op.dst_off,
+                              op.rows, op.cols, static_cast<int>(op.k), P.hs_coef, s);
+      if (rc) return rc;
     } else if (op.op == NU_OP_ZERO) {
       char* cc = c.base[op.c_buf] + op.c_off * 4;
       e = cudaMemset2DAsync(cc, op.ldc * 4, 0, op.n * 4, op.m, s);

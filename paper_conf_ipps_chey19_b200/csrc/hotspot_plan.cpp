@@ -1,0 +1,358 @@
+// HotSpot-2D over the Northup tree (S§8(f) NEXT-3; §IV-B).
+//
+// The paper's recursion: at level l divide the grid into
+// dim(l) x dim(l) sub-blocks; move each block, its power and its four borders
+// to level l+1; recurse; copy the result back.  Unrolled here for the tree
+// HOST root -> HBM siblings -> SMEM leaf:
+//
+//   per pass (h iterations, h = the border width):
+//     per block (b x b, raster order, block rows split over the siblings):
+//       data_down  the window = block + h-wide borders (clipped at the grid
+//                  edge) of the current grid and of P, HOST -> HBM slot
+//                  (strided 2-D copies: the DMA engine gathers the east/west
+//                  borders that P:317 packs by hand)
+//       compute    ceil(h / 8) leaf launches ping-ponging between two window
+//                  buffers of the slot; each launch's window is the previous
+//                  one's valid region (shrunk by its iterations on every side
+//                  that is not a grid edge)
+//       data_up    the block, HBM -> the pass's output grid
+//   passes alternate between Tout and a pinned scratch grid at the root so
+//   the last pass writes Tout.
+//
+// Dependencies come from the rectangle tracker (plan_builder.h): a window of
+// pass q+1 waits for the pass-q blocks it overlaps (RAW on the host grid) and
+// a pass-q+1 block write waits for the pass-q windows that read that grid
+// (WAR) — across siblings too (user_disjoint = false).  Three slots per
+// sibling overlap H2D, compute and D2H.
+#include <math.h>
+
+#include <chrono>
+
+#include "northup_internal.h"
+#include "plan_builder.h"
+
+namespace nu {
+
+namespace {
+
+inline northup_op make_stencil(int worker, int tin, int64_t tin_off, int64_t ldt, int pw,
+                               int64_t pw_off, int64_t ldp, int tout, int64_t tout_off, int64_t ldo,
+                               int64_t wm, int64_t wn, int64_t gy0, int64_t gx0, int64_t R,
+                               int64_t C, int iters) {
+  northup_op o{};
+  o.op = NU_OP_STENCIL;
+  o.worker = worker;
+  o.stream = S_COMP;
+  o.a_buf = tin;
+  o.a_off = tin_off;
+  o.lda = ldt;
+  o.b_buf = pw;
+  o.b_off = pw_off;
+  o.ldb = ldp;
+  o.c_buf = tout;
+  o.c_off = tout_off;
+  o.ldc = ldo;
+  o.m = wm;
+  o.n = wn;
+  o.k = iters;
+  o.src_off = gy0;
+  o.dst_off = gx0;
+  o.rows = R;
+  o.cols = C;
+  o.src_buf = o.dst_buf = -1;
+  return o;
+}
+
+struct Win {
+  int64_t y0, y1, x0, x1;   // grid coordinates, half open
+};
+
+// Valid region after `it` iterations on window w.
+Win shrink(const Win& w, int it, int64_t R, int64_t C) {
+  return Win{w.y0 == 0 ? 0 : w.y0 + it, w.y1 == R ? R : w.y1 - it, w.x0 == 0 ? 0 : w.x0 + it,
+             w.x1 == C ? C : w.x1 - it};
+}
+
+// Emit the leaf launches of `iters` iterations on window `w`, whose cells sit
+// in buffers buf[0] / buf[1] (origin (oy, ox), leading dimension ld) with
+// power in `pb`; returns the buffer index holding the final values.
+int emit_iterations(Builder& B, int worker, Win w, int64_t iters, int hl, const int buf[2],
+                    const int64_t off[2], int pb, int64_t poff, int64_t ld, int64_t oy, int64_t ox,
+                    int64_t R, int64_t C, northup_stats* st) {
+  int cur = 0;
+  for (int64_t done = 0; done < iters;) {
+    const int it = static_cast<int>(std::min<int64_t>(hl, iters - done));
+    const Win v = shrink(w, it, R, C);
+    const int64_t wo = (w.y0 - oy) * ld + (w.x0 - ox), vo = (v.y0 - oy) * ld + (v.x0 - ox);
+    const int64_t wm = w.y1 - w.y0, wn = w.x1 - w.x0;
+    B.emit(make_stencil(worker, buf[cur], off[cur] + wo, ld, pb, poff + wo, ld, buf[cur ^ 1],
+                        off[cur ^ 1] + wo, ld, wm, wn, w.y0, w.x0, R, C, it),
+           {{buf[cur], off[cur] + wo, ld, wm, wn, false},
+            {pb, poff + wo, ld, wm, wn, false},
+            {buf[cur ^ 1], off[cur ^ 1] + vo, ld, v.y1 - v.y0, v.x1 - v.x0, true}});
+    st->leaf_launches++;
+    cur ^= 1;
+    w = v;
+    done += it;
+  }
+  return cur;
+}
+
+}  // namespace
+
+int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t iters,
+                       const northup_hotspot_opts* o, const northup_hotspot_coeffs* k, Plan* out) {
+  int rc = validate_tree(t);
+  if (rc) return rc;
+  if (R < 0 || C < 0 || iters < 0) return fail(NU_EINVAL, "negative grid size or iteration count");
+  const int hl = o && o->leaf_iters ? o->leaf_iters : kHotspotMaxIters;
+  if (hl < 1 || hl > kHotspotMaxIters)
+    return fail(NU_EINVAL, "leaf_iters must be in [1, %d]", kHotspotMaxIters);
+  Plan& P = *out;
+  P = Plan();
+  P.M = R;
+  P.N = C;
+  P.K = iters;
+  northup_hotspot_coeffs kk{};
+  if (k) kk = *k;
+  else northup_hotspot_default_coeffs(R, C, &kk);
+  P.hs_coef[0] = kk.cap_1;
+  P.hs_coef[1] = kk.rx_1;
+  P.hs_coef[2] = kk.ry_1;
+  P.hs_coef[3] = kk.rz_1;
+  P.hs_coef[4] = kk.amb;
+  Builder B;
+  B.P = &P;
+  B.user_disjoint = false;
+  const int T = B.add_buf(B_USER_A, 0, -1, 4ull * R * C);
+  const int PW = B.add_buf(B_USER_B, 0, -1, 4ull * R * C);
+  const int OUT = B.add_buf(B_USER_C, 0, -1, 4ull * R * C);
+  northup_stats& st = P.stats;
+  st = northup_stats{};
+  const Node& root = t->nodes[0];
+
+  if (root.storage == NU_HBM) {
+    // in-HBM reference: whole-grid launches ping-ponging between Tout and an
+    // arena scratch grid; the last launch writes Tout
+    P.root_is_device = true;
+    P.num_workers = 1;
+    P.worker_node.push_back(0);
+    st.num_gpus = 1;
+    if (R == 0 || C == 0) return 0;
+    if (iters == 0) {
+      B.emit(make_copy(0, S_COMP, T, 0, C, OUT, 0, C, R, C), {{T, 0, C, R, C, false}, {OUT, 0, C, R, C, true}});
+      st.bytes_d2d += 4ull * R * C;
+      st.ops = static_cast<int64_t>(P.ops.size());
+      return 0;
+    }
+    const int64_t L = (iters + hl - 1) / hl;
+    const int S = L > 1 ? B.add_buf(B_ARENA, 0, 0, 4ull * R * C) : -1;
+    int src = T;
+    for (int64_t j = 0; j < L; ++j) {
+      const int it = static_cast<int>(std::min<int64_t>(hl, iters - j * hl));
+      const int dst = ((L - 1 - j) % 2 == 0) ? OUT : S;
+      B.emit(make_stencil(0, src, 0, C, PW, 0, C, dst, 0, C, R, C, 0, 0, R, C, it),
+             {{src, 0, C, R, C, false}, {PW, 0, C, R, C, false}, {dst, 0, C, R, C, true}});
+      st.leaf_launches++;
+      src = dst;
+    }
+    st.bm = R;
+    st.bn = C;
+    st.bk = hl;
+    st.hbm_peak_bytes = S >= 0 ? 4ull * R * C : 0;
+    st.ops = static_cast<int64_t>(P.ops.size());
+    return 0;
+  }
+  if (root.storage != NU_HOST) return fail(NU_ENOTSUP, "HotSpot-2D needs a HOST or HBM root");
+  std::vector<int> hbm;
+  for (int c : root.children) {
+    if (t->nodes[c].storage != NU_HBM)
+      return fail(NU_ENOTSUP, "HOST root children must be HBM nodes (node %d is not)", c);
+    hbm.push_back(c);
+  }
+  if (hbm.empty()) return fail(NU_EINVAL, "HOST root has no HBM child");
+  if (t->local_node >= 0) return fail(NU_ENOTSUP, "HotSpot-2D runs in one process (no set_local)");
+  const int G = static_cast<int>(hbm.size());
+  P.num_workers = G;
+  P.worker_node = hbm;
+  st.num_gpus = G;
+  if (R == 0 || C == 0) return 0;
+  if (iters == 0) {
+    B.emit(make_copy(0, S_D2H, T, 0, C, OUT, 0, C, R, C), {{T, 0, C, R, C, false}, {OUT, 0, C, R, C, true}});
+    st.ops = static_cast<int64_t>(P.ops.size());
+    return 0;
+  }
+  uint64_t cap = 0;
+  for (int h : hbm)
+    if (t->nodes[h].capacity) cap = cap ? std::min(cap, t->nodes[h].capacity) : t->nodes[h].capacity;
+  constexpr int kS = kSlots;
+  // slot footprint: three windows (temperature ping, pong, power), (b + 2h) square
+  auto arena_bytes = [&](int64_t b, int64_t h) {
+    const int64_t W = std::min(b + 2 * h, std::max(R, C));
+    return 4ull * kS * 3 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(std::min(W, C));
+  };
+  const int64_t edge = std::max(R, C);
+  int64_t b = o && o->block > 0 ? o->block : std::min<int64_t>(edge, 8192);   // P:325 8k blocking
+  int64_t h = o && o->halo > 0 ? o->halo : 0;
+  if (h <= 0) {
+    // iterations per visit: all of them when the border overhead stays small,
+    // else a multiple of the leaf's iterations with <= ~15% extra window area
+    const int64_t hmax = std::max<int64_t>(hl, (static_cast<int64_t>(0.035 * b) / hl) * hl);
+    h = std::min(iters, hmax);
+  }
+  h = std::min(h, iters);
+  if (!(o && o->block > 0)) {
+    while (cap && arena_bytes(b, h) > cap && b > 8) b = b > 64 ? rup(b / 2, 64) : std::max<int64_t>(8, b / 2);
+    // equal blocks: the fewest blocks of at most b cells per side
+    const int64_t g = b >= 64 ? 64 : 8;
+    const int64_t nby = cdiv(R, b), nbx = cdiv(C, b);
+    const int64_t be = std::max(rup(cdiv(R, nby), g), rup(cdiv(C, nbx), g));
+    if (!cap || arena_bytes(std::min(be, edge), h) <= cap) b = std::min(be, edge);
+  }
+  if (cap && arena_bytes(b, h) > cap)
+    return fail(NU_ENOMEM, "HBM capacity %llu B below the HotSpot block %lld + border %lld",
+                (unsigned long long)cap, (long long)b, (long long)h);
+  const int64_t W = std::min(b + 2 * h, edge);
+  const int64_t WR = std::min(W, R), LD = pad_ld(std::min(W, C));
+  const int64_t win = WR * LD;   // elements per window buffer
+  std::vector<int> arena(G);
+  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, arena_bytes(b, h));
+  const int64_t Q = cdiv(iters, h);
+  const int S = Q > 1 ? B.add_buf(B_DRAM, 0, -1, 4ull * R * C) : -1;   // pinned scratch grid
+  const int64_t nby = cdiv(R, b), nbx = cdiv(C, b);
+  st.bm = st.bn = b;
+  st.bk = h;
+  st.hbm_peak_bytes = arena_bytes(b, h);
+  std::vector<int64_t> slot_ctr(G, 0);
+  int src = T;
+  for (int64_t q = 0; q < Q; ++q) {
+    const int64_t itq = std::min(h, iters - q * h);
+    const int dst = ((Q - 1 - q) % 2 == 0) ? OUT : S;
+    const int ldg_src = C, ldg_dst = C;
+    for (int64_t by = 0; by < nby; ++by) {
+      const int w = static_cast<int>(by * G / nby);   // block rows split over the siblings
+      for (int64_t bx = 0; bx < nbx; ++bx) {
+        const Win blk{by * b, std::min(R, (by + 1) * b), bx * b, std::min(C, (bx + 1) * b)};
+        const Win win_g{std::max<int64_t>(0, blk.y0 - itq), std::min(R, blk.y1 + itq),
+                        std::max<int64_t>(0, blk.x0 - itq), std::min(C, blk.x1 + itq)};
+        const int64_t wm = win_g.y1 - win_g.y0, wn = win_g.x1 - win_g.x0;
+        const int sl = static_cast<int>(slot_ctr[w]++ % kS);
+        const int64_t base = static_cast<int64_t>(sl) * 3 * win;
+        const int64_t off[2] = {base, base + win};
+        const int64_t poff = base + 2 * win;
+        const int bufs[2] = {arena[w], arena[w]};
+        // data_down: window of the current grid and of P (block + borders)
+        const int64_t go = win_g.y0 * C + win_g.x0;
+        B.emit(make_copy(w, S_H2D, src, go, ldg_src, arena[w], off[0], LD, wm, wn),
+               {{src, go, ldg_src, wm, wn, false}, {arena[w], off[0], LD, wm, wn, true}});
+        B.emit(make_copy(w, S_H2D, PW, go, C, arena[w], poff, LD, wm, wn),
+               {{PW, go, C, wm, wn, false}, {arena[w], poff, LD, wm, wn, true}});
+        st.bytes_h2d += 8ull * wm * wn;
+        const int fin = emit_iterations(B, w, win_g, itq, hl, bufs, off, arena[w], poff, LD, win_g.y0,
+                                        win_g.x0, R, C, &st);
+        // data_up: the block
+        const int64_t bo = off[fin] + (blk.y0 - win_g.y0) * LD + (blk.x0 - win_g.x0);
+        const int64_t bm = blk.y1 - blk.y0, bn = blk.x1 - blk.x0;
+        const int64_t dgo = blk.y0 * C + blk.x0;
+        B.emit(make_copy(w, S_D2H, arena[w], bo, LD, dst, dgo, ldg_dst, bm, bn),
+               {{arena[w], bo, LD, bm, bn, false}, {dst, dgo, ldg_dst, bm, bn, true}});
+        st.bytes_d2h += 4ull * bm * bn;
+      }
+    }
+    src = dst;
+  }
+  st.ops = static_cast<int64_t>(P.ops.size());
+  for (const northup_op& op : P.ops)
+    if (op.op == NU_OP_COPY) st.copies++;
+  return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
+}
+
+}  // namespace nu
+
+using namespace nu;
+
+extern "C" {
+
+int northup_hotspot_default_coeffs(int64_t rows, int64_t cols, northup_hotspot_coeffs* out) {
+  if (!out) return fail(NU_EINVAL, "NULL argument");
+  (void)rows;
+  (void)cols;
+  // [18]'s chip model (RH1) at its 1024-cell pitch (RH2): 16 mm / 1024
+  const double t_chip = 0.0005, k_si = 100.0, spec_heat = 1.75e6, factor = 0.5;
+  const double max_pd = 3.0e6, precision = 0.001, pitch = 0.016 / 1024.0;
+  const double cap = factor * spec_heat * t_chip * pitch * pitch;
+  const double rx = pitch / (2.0 * k_si * t_chip * pitch);
+  const double ry = pitch / (2.0 * k_si * t_chip * pitch);
+  const double rz = t_chip / (k_si * pitch * pitch);
+  const double step = precision / (max_pd / (factor * t_chip * spec_heat));
+  out->cap_1 = static_cast<float>(step / cap);
+  out->rx_1 = static_cast<float>(1.0 / rx);
+  out->ry_1 = static_cast<float>(1.0 / ry);
+  out->rz_1 = static_cast<float>(1.0 / rz);
+  out->amb = 80.0f;
+  return 0;
+}
+
+int northup_hotspot_leaf(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
+                         int64_t ldo, int64_t wm, int64_t wn, int64_t gy0, int64_t gx0,
+                         int64_t rows, int64_t cols, int iters, const northup_hotspot_coeffs* k,
+                         void* stream) {
+  northup_hotspot_coeffs kk{};
+  if (k) kk = *k;
+  else northup_hotspot_default_coeffs(rows, cols, &kk);
+  const float coef[5] = {kk.cap_1, kk.rx_1, kk.ry_1, kk.rz_1, kk.amb};
+  return hotspot_launch(tin, ldt, pw, ldp, tout, ldo, wm, wn, gy0, gx0, rows, cols, iters, coef,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int northup_hotspot_plan(northup_tree_t t, int64_t rows, int64_t cols, int64_t iters,
+                         const northup_hotspot_opts* opts, northup_plan_t* out) {
+  if (!t || !out) return fail(NU_EINVAL, "NULL argument");
+  northup_plan_s* p = new northup_plan_s();
+  int rc = build_hotspot_plan(t, rows, cols, iters, opts, nullptr, &p->plan);
+  if (rc) {
+    delete p;
+    return rc;
+  }
+  *out = p;
+  return 0;
+}
+
+int northup_hotspot(northup_tree_t t, northup_buf_t T, northup_buf_t P, northup_buf_t Tout,
+                    int64_t rows, int64_t cols, int64_t iters, const northup_hotspot_coeffs* k,
+                    const northup_hotspot_opts* opts, northup_stats* s) {
+  const auto t0 = std::chrono::steady_clock::now();
+  if (!t || !T || !P || !Tout) return fail(NU_EINVAL, "NULL argument");
+  if (!t->finalized) return fail(NU_ESTATE, "tree not finalized");
+  if (t->busy) return fail(NU_ESTATE, "a call is already in flight on this tree");
+  if (T->tree != t || P->tree != t || Tout->tree != t) return fail(NU_EINVAL, "buffer from another tree");
+  if (T->node != 0 || P->node != 0 || Tout->node != 0)
+    return fail(NU_EINVAL, "T, P and Tout must live at the root node");
+  if (rows < 0 || cols < 0 || iters < 0) return fail(NU_EINVAL, "negative argument");
+  const uint64_t need = 4ull * rows * cols;
+  if (T->bytes < need || P->bytes < need || Tout->bytes < need)
+    return fail(NU_EINVAL, "buffer smaller than the grid");
+  if (T == Tout || T->ptr == Tout->ptr) return fail(NU_EINVAL, "T and Tout must differ");
+  northup_stats local{};
+  northup_stats* st = s ? s : &local;
+  *st = northup_stats{};
+  t->busy = true;
+  Plan plan;
+  int rc = build_hotspot_plan(t, rows, cols, iters, opts, k, &plan);
+  if (!rc) {
+    *st = plan.stats;
+    st->t_plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    northup_gemm_opts go{};
+    go.collect_timing = opts ? opts->collect_timing : 0;
+    go.shared_staging = -1;
+    int prev = 0;
+    cudaGetDevice(&prev);
+    rc = execute_plan(t, plan, T, P, Tout, &go, st);
+    cudaSetDevice(prev);
+  }
+  t->busy = false;
+  st->t_total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return rc;
+}
+
+}  // extern "C"

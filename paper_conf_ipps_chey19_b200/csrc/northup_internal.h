@@ -19,6 +19,7 @@ constexpr int kDefaultLeafVariant = 4;      // 1 = v0 1-CTA, 2 = v1.2 TMA-fed pa
 constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
 constexpr int kRasterBand = 16;            // n-blocks per raster band in the leaf
 constexpr int64_t kPanelChunks = 1;        // leaf K-panel launches, in k_chunks (0 = one launch)
+constexpr int kHotspotMaxIters = 8;        // HotSpot-2D iterations per leaf launch (shared-memory border)
 
 // Thread-local error message (northup_last_error).  Returns its argument so
 // call sites can write `return fail(NU_EINVAL, "...")`.
@@ -118,6 +119,7 @@ struct Plan {
   int npass = 3;
   bool root_is_device = false;
   bool file_root = false;
+  float hs_coef[5] = {};                // HotSpot-2D plans: cap_1, rx_1, ry_1, rz_1, amb
 };
 
 int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
@@ -140,6 +142,17 @@ int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ld
                          int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                          int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream);
 
+// --------------------------------------------------------------- HotSpot-2D
+// The leaf (hotspot.cu): `iters` (<= kHotspotMaxIters) iterations on a window
+// wm x wn at grid origin (gy0, gx0) of an R x C grid; writes the window's valid
+// region (shrunk by `iters` on every side that is not a grid edge) into tout,
+// which has the window's shape.
+int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
+                   int64_t ldo, int64_t wm, int64_t wn, int64_t gy0, int64_t gx0, int64_t R,
+                   int64_t C, int iters, const float coef[5], cudaStream_t stream);
+int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t iters,
+                       const northup_hotspot_opts* o, const northup_hotspot_coeffs* k, Plan* out);
+
 // --------------------------------------------------------------- executor
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,
                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
@@ -157,3 +170,7 @@ void destroy_graphs(northup_tree_s* t);
 void destroy_workers(northup_tree_s* t);
 
 }  // namespace nu
+
+struct northup_plan_s {
+  nu::Plan plan;
+};

@@ -1,0 +1,134 @@
+"""HotSpot-2D on the B200 (NEXT-3): the sm_100a leaf and the tree runtime
+(in-HBM and HOST -> HBM out-of-core, virtual siblings) against the fp64
+oracle (oracle/hotspot.py) within the RH3 bound, and bit for bit against an
+fp32 emulation of the update in the kernel's evaluation order; in-HBM and
+out-of-core runs agree bit for bit whatever the blocks, borders and
+iterations per launch."""
+import ctypes
+
+import numpy as np
+import pytest
+import torch
+
+import nugen
+import paper_conf_ipps_chey19_b200 as nu
+from oracle import hotspot as hs
+
+pytestmark = pytest.mark.gpu
+K = hs.coeffs(1024, 1024)
+
+
+def grids(R, C, seed):
+    return (nugen.fill(R, C, seed, nugen.MAT_T, "temp"), nugen.fill(R, C, seed, nugen.MAT_P, "power"))
+
+
+def emulate_fp32(T, P, iters):
+    """The update in fp32, evaluated in the kernel's order (test-side check,
+    independent of the CUDA code): t + cap*(((p + ((s+n) - 2t)*ry) + ((e+w) - 2t)*rx) + (amb - t)*rz)."""
+    k = nu.hotspot_coeffs(*T.shape)
+    f = np.float32
+    cap, rx, ry, rz, amb = f(k.cap_1), f(k.rx_1), f(k.ry_1), f(k.rz_1), f(k.amb)
+    t = T.astype(np.float32).copy()
+    p = P.astype(np.float32)
+    for _ in range(iters):
+        g = np.pad(t, 1, mode="edge")
+        n, s, e, w = g[:-2, 1:-1], g[2:, 1:-1], g[1:-1, 2:], g[1:-1, :-2]
+        two_t = f(2) * t
+        d = ((p + ((s + n) - two_t) * ry) + ((e + w) - two_t) * rx) + (amb - t) * rz
+        t = (t + cap * d).astype(np.float32)
+    return t
+
+
+def check(out, T, P, iters):
+    ref = hs.run(T, P, iters, K)
+    err = np.abs(out.astype(np.float64) - ref).max()
+    assert err <= hs.tolerance(iters, np.abs(ref).max()), err
+
+
+@pytest.mark.parametrize("R,C,iters", [(1, 1, 3), (7, 300, 8), (200, 257, 1), (333, 129, 5), (130, 70, 8)])
+def test_leaf_whole_grid(R, C, iters):
+    T, P = grids(R, C, seed=R * 7 + C)
+    dev = torch.device("cuda", 0)
+    t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+    o = torch.full_like(t, float("nan"))
+    nu.hotspot_leaf(t, p, o, iters)
+    out = o.cpu().numpy()
+    check(out, T, P, iters)
+    assert np.array_equal(out, emulate_fp32(T, P, iters))
+
+
+def test_leaf_sub_window_valid_region():
+    """A window inside the grid: only the valid region (shrunk by `iters` on
+    non-edge sides) is written, and it equals the full-grid evolution."""
+    R, C, iters = 300, 400, 6
+    T, P = grids(R, C, seed=11)
+    full = emulate_fp32(T, P, iters)
+    dev = torch.device("cuda", 0)
+    for (y0, y1, x0, x1) in [(50, 200, 60, 300), (0, 120, 100, 400), (250, 300, 0, 77)]:
+        t = torch.from_numpy(np.ascontiguousarray(T[y0:y1, x0:x1])).to(dev)
+        p = torch.from_numpy(np.ascontiguousarray(P[y0:y1, x0:x1])).to(dev)
+        o = torch.full_like(t, float("nan"))
+        nu.hotspot_leaf(t, p, o, iters, gy0=y0, gx0=x0, rows=R, cols=C)
+        out = o.cpu().numpy()
+        vy0 = 0 if y0 == 0 else iters
+        vy1 = (y1 - y0) - (0 if y1 == R else iters)
+        vx0 = 0 if x0 == 0 else iters
+        vx1 = (x1 - x0) - (0 if x1 == C else iters)
+        assert np.array_equal(out[vy0:vy1, vx0:vx1], full[y0 + vy0:y0 + vy1, x0 + vx0:x0 + vx1])
+        mask = np.ones(out.shape, bool)
+        mask[vy0:vy1, vx0:vx1] = False
+        assert np.isnan(out[mask]).all()            # nothing outside the valid region
+
+
+def host_view(buf, rows, cols):
+    return np.ctypeslib.as_array((ctypes.c_float * (rows * cols)).from_address(buf.ptr)).reshape(rows, cols)
+
+
+def run_tree(R, C, iters, G=1, cap=0, **opt):
+    t, _ = nu.host_tree(G, cap, devices=[0] * G)
+    t.finalize()
+    Tb, Pb, Ob = t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0)
+    T, P = host_view(Tb, R, C), host_view(Pb, R, C)
+    T[...], P[...] = grids(R, C, seed=R + C)
+    host_view(Ob, R, C)[...] = np.nan
+    st = t.hotspot(Tb, Pb, Ob, R, C, iters, nu.hotspot_opts(**opt))
+    out, Tc, Pc = host_view(Ob, R, C).copy(), T.copy(), P.copy()
+    assert np.array_equal(T, grids(R, C, seed=R + C)[0])      # T is not modified
+    t.destroy()
+    return out, Tc, Pc, st
+
+
+def run_in_hbm(R, C, iters, leaf_iters=0):
+    T, P = grids(R, C, seed=R + C)
+    dev = torch.device("cuda", 0)
+    t = nu.hbm_tree(0)
+    t.finalize()
+    Td, Pd = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+    Od = torch.full_like(Td, float("nan"))
+    st = t.hotspot(t.wrap_device(0, Td.data_ptr(), Td.numel() * 4), t.wrap_device(0, Pd.data_ptr(), Pd.numel() * 4),
+                   t.wrap_device(0, Od.data_ptr(), Od.numel() * 4), R, C, iters, nu.hotspot_opts(leaf_iters=leaf_iters))
+    out = Od.cpu().numpy()
+    t.destroy()
+    return out, T, P, st
+
+
+@pytest.mark.parametrize("R,C,iters,G,cap,opt", [
+    (1000, 1200, 20, 1, 0, dict(block=256, halo=8)),
+    (1000, 1200, 20, 2, 0, dict(block=320, halo=6, leaf_iters=3)),
+    (777, 515, 13, 1, 6 << 20, dict()),
+    (2048, 2048, 40, 4, 0, dict(block=512, halo=20)),
+])
+def test_tree_out_of_core_matches_in_hbm_and_oracle(R, C, iters, G, cap, opt):
+    out, T, P, st = run_tree(R, C, iters, G, cap, **opt)
+    ref_hbm, _, _, _ = run_in_hbm(R, C, iters)
+    assert np.array_equal(out, ref_hbm)                  # bitwise, any blocking
+    assert np.array_equal(out, emulate_fp32(T, P, iters))
+    check(out, T, P, iters)
+    assert st["leaf_launches"] > 0 and st["bytes_h2d"] >= 8 * R * C
+
+
+def test_in_hbm_leaf_iters_invariance():
+    a = run_in_hbm(513, 640, 17, leaf_iters=8)[0]
+    b = run_in_hbm(513, 640, 17, leaf_iters=1)[0]
+    c = run_in_hbm(513, 640, 17, leaf_iters=5)[0]
+    assert np.array_equal(a, b) and np.array_equal(a, c)
