@@ -17,6 +17,7 @@
 // runs agree bit for bit, and so does an fp32 numpy emulation of the update.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "northup_internal.h"
 
@@ -50,6 +51,16 @@ __device__ __forceinline__ float update(float t, float p, float n, float s, floa
   return __fadd_rn(t, __fmul_rn(a.cap_1, d));
 }
 
+// 4-byte asynchronous global -> shared copies (LDGSTS): every element of the
+// tile is in flight at once instead of one load per thread per loop trip.
+__device__ __forceinline__ void cp_async4(float* smem, const float* gmem) {
+  const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+
 __global__ void __launch_bounds__(kThreads) hotspot_kernel(Args a) {
   extern __shared__ float sm[];
   const int it = a.iters;
@@ -66,15 +77,16 @@ __global__ void __launch_bounds__(kThreads) hotspot_kernel(Args a) {
   const int64_t sx0 = max(tx0 - it, int64_t(0)), sx1 = min(tx1 + it, a.wn);
   const int hy = static_cast<int>(sy1 - sy0), hx = static_cast<int>(sx1 - sx0);
 
-  // data_down HBM -> SMEM: the tile with its borders (coalesced rows)
+  // data_down HBM -> SMEM: the tile with its borders (coalesced rows, async)
   for (int y = ty; y < hy; y += kWY) {
     const float* trow = a.tin + (sy0 + y) * a.ldt + sx0;
     const float* prow = a.pw + (sy0 + y) * a.ldp + sx0;
     for (int x = tx; x < hx; x += kWX) {
-      cur[y * SX + x] = __ldg(trow + x);
-      pwr[y * SX + x] = __ldg(prow + x);
+      cp_async4(&cur[y * SX + x], trow + x);
+      cp_async4(&pwr[y * SX + x], prow + x);
     }
   }
+  cp_async_wait_all();
   __syncthreads();
 
   // sides of the shared-memory region that are grid edges (clamped, never shrink)
@@ -108,9 +120,219 @@ __global__ void __launch_bounds__(kThreads) hotspot_kernel(Args a) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// v2: register-blocked.  A CTA owns a region of RH = NWY*RPT rows x RW = NWX*32
+// columns; thread (lane, warp) keeps RPT consecutive cells of one column (and
+// their power) in registers for all iterations.  Per iteration:
+//   * N/S inside the segment come from registers; across segments each thread
+//     publishes its top and bottom cell in shared memory;
+//   * E/W come from warp shuffles; lanes 0 / 31 take the neighbouring warp's
+//     edge column from shared memory;
+//   * one __syncthreads (the exchange arrays are double-buffered by parity).
+// Grid-edge neighbours are clamped per cell, exactly as in v1, and the update
+// is the same function, so v2 is bitwise equal to v1 (tested).
+template <int RPT, int NWX, int NWY>
+__global__ void __launch_bounds__(NWX * NWY * 32, 1) hotspot_kernel_v2(Args a) {
+  constexpr int RW = NWX * 32, RH = NWY * RPT;
+  __shared__ float tops[2][NWY][RW], bots[2][NWY][RW];
+  __shared__ float colL[2][NWX][RH], colR[2][NWX][RH];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int sx = warp % NWX, gyi = warp / NWX;
+  const int h = a.iters;
+  const int OTY = RH - 2 * h, OTX = RW - 2 * h;
+  const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
+  const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
+  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
+  const int x = sx * 32 + lane;                    // column inside the region
+  const int64_t wx = rx + x;                       // window column
+  const int64_t gcol = a.gx0 + wx;                 // grid column
+  const int r0 = gyi * RPT;                        // first row of this segment
+  const bool xin = wx >= 0 && wx < a.wn;
+
+  float v[RPT], p[RPT];
+#pragma unroll
+  for (int r = 0; r < RPT; ++r) {
+    const int64_t wy = ry + r0 + r;
+    const bool in = xin && wy >= 0 && wy < a.wm;
+    v[r] = in ? __ldg(a.tin + wy * a.ldt + wx) : 0.0f;
+    p[r] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
+  }
+  // segment rows r with grid row 0 / R - 1 (clamped neighbours); else out of range
+  const int rtop = static_cast<int>(-(a.gy0 + ry + r0));
+  const int rbot = static_cast<int>(a.R - 1 - (a.gy0 + ry + r0));
+  const bool wclamp = gcol == 0, eclamp = gcol == a.C - 1;
+
+  for (int k = 0; k < h; ++k) {
+    const int b = k & 1;
+    tops[b][gyi][x] = v[0];
+    bots[b][gyi][x] = v[RPT - 1];
+    if (lane == 0) {
+#pragma unroll
+      for (int r = 0; r < RPT; ++r) colL[b][sx][r0 + r] = v[r];
+    }
+    if (lane == 31) {
+#pragma unroll
+      for (int r = 0; r < RPT; ++r) colR[b][sx][r0 + r] = v[r];
+    }
+    __syncthreads();
+    const float n0 = gyi > 0 ? bots[b][gyi - 1][x] : v[0];
+    const float sL = gyi < NWY - 1 ? tops[b][gyi + 1][x] : v[RPT - 1];
+    // in place, top to bottom: `above` keeps the old value of the row above
+    float above = n0;
+#pragma unroll
+    for (int r = 0; r < RPT; ++r) {
+      const float c = v[r];
+      float w = __shfl_up_sync(0xffffffffu, c, 1);
+      float e = __shfl_down_sync(0xffffffffu, c, 1);
+      if (lane == 0) w = sx > 0 ? colR[b][sx - 1][r0 + r] : c;
+      if (lane == 31) e = sx < NWX - 1 ? colL[b][sx + 1][r0 + r] : c;
+      float n = above;
+      float s = r < RPT - 1 ? v[r + 1] : sL;
+      if (r == rtop) n = c;                        // grid-edge clamps (as v1)
+      if (r == rbot) s = c;
+      if (wclamp) w = c;
+      if (eclamp) e = c;
+      v[r] = update(c, p[r], n, s, e, w, a);
+      above = c;
+    }
+  }
+
+  // the output tile: rows [oy0, oy0 + OTY) x cols [ox0, ox0 + OTX) within the valid region
+  if (wx < ox0 || wx >= min(ox0 + OTX, a.vx1)) return;
+  const int64_t ylo = oy0, yhi = min(oy0 + OTY, a.vy1);
+#pragma unroll
+  for (int r = 0; r < RPT; ++r) {
+    const int64_t wy = ry + r0 + r;
+    if (wy >= ylo && wy < yhi) a.tout[wy * a.ldo + wx] = v[r];
+  }
+}
+
+// ---------------------------------------------------------------------------
+// v3: register runs + shared-memory plane.  A CTA owns a region of
+// RH = NWY*V rows x RW = NWX*32 columns (plus a one-cell apron in shared
+// memory).  Thread (lane, warp) keeps V consecutive cells of column
+// x = 32*(warp % NWX) + lane, and their power, in registers for all the
+// launch's iterations.  Per iteration it reads the W/E neighbours of its V
+// cells and the cells above / below its run from the current plane, computes
+// V updates, writes them to the next plane, and the CTA synchronises once
+// (two planes alternate).  CTAs whose region touches no grid edge run the
+// clamp-free body; edge CTAs clamp per cell exactly as v1, so v3 is bitwise
+// equal to v1 (tested).
+template <int V, int NWX, int NWY, bool EDGE>
+__device__ __forceinline__ void v3_iterate(const Args& a, float* __restrict__ pl0, float* __restrict__ pl1,
+                                           float (&v)[V], const float (&p)[V], int x, int r0, int rtop,
+                                           int rbot, bool wclamp, bool eclamp) {
+  constexpr int SW = NWX * 32 + 2;   // plane row stride (apron columns 0 and SW - 1)
+  float* cur = pl0;
+  float* nxt = pl1;
+  for (int k = 0; k < a.iters; ++k) {
+    const float* crow = cur + (r0 + 1) * SW + (x + 1);   // this thread's first cell
+    float above = crow[-SW];
+    const float below = crow[V * SW];
+#pragma unroll
+    for (int r = 0; r < V; ++r) {
+      const float c = v[r];
+      float n = above;
+      float s = r < V - 1 ? v[r + 1] : below;
+      float w = crow[r * SW - 1];
+      float e = crow[r * SW + 1];
+      if (EDGE) {
+        if (r == rtop) n = c;
+        if (r == rbot) s = c;
+        if (wclamp) w = c;
+        if (eclamp) e = c;
+      }
+      v[r] = update(c, p[r], n, s, e, w, a);
+      nxt[(r0 + 1 + r) * SW + x + 1] = v[r];
+      above = c;
+    }
+    __syncthreads();
+    float* t = cur;
+    cur = nxt;
+    nxt = t;
+  }
+}
+
+#ifndef NU_HS_V3_MINB
+#define NU_HS_V3_MINB 1
+#endif
+template <int V, int NWX, int NWY>
+__global__ void __launch_bounds__(NWX * NWY * 32, NU_HS_V3_MINB) hotspot_kernel_v3(Args a) {
+  constexpr int RW = NWX * 32, RH = NWY * V, SW = RW + 2, SH = RH + 2;
+  extern __shared__ float sm3[];
+  float* pl0 = sm3;
+  float* pl1 = sm3 + SH * SW;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int x = (warp % NWX) * 32 + lane, r0 = (warp / NWX) * V;
+  const int h = a.iters;
+  const int OTY = RH - 2 * h, OTX = RW - 2 * h;
+  const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
+  const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
+  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
+  const int64_t wx = rx + x;
+  const bool xin = wx >= 0 && wx < a.wn;
+  float v[V], p[V];
+#pragma unroll
+  for (int r = 0; r < V; ++r) {
+    const int64_t wy = ry + r0 + r;
+    const bool in = xin && wy >= 0 && wy < a.wm;
+    v[r] = in ? __ldg(a.tin + wy * a.ldt + wx) : 0.0f;
+    p[r] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
+  }
+#pragma unroll
+  for (int r = 0; r < V; ++r) pl0[(r0 + 1 + r) * SW + x + 1] = v[r];
+  __syncthreads();
+  // does the region touch a grid edge?  (uniform per CTA)
+  const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
+  const bool edge = gy_top <= 0 || gy_top + RH >= a.R || gx_left <= 0 || gx_left + RW >= a.C;
+  if (edge) {
+    const int rtop = static_cast<int>(-(gy_top + r0));
+    const int rbot = static_cast<int>(a.R - 1 - (gy_top + r0));
+    const int64_t gcol = gx_left + x;
+    v3_iterate<V, NWX, NWY, true>(a, pl0, pl1, v, p, x, r0, rtop, rbot, gcol == 0, gcol == a.C - 1);
+  } else {
+    v3_iterate<V, NWX, NWY, false>(a, pl0, pl1, v, p, x, r0, 0, 0, false, false);
+  }
+  // store: recompute the coordinates (keeps them out of the iteration's registers)
+  const int64_t oy = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
+  const int64_t ox = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
+  const int64_t sx = ox - h + x;
+  if (sx < ox || sx >= min(ox + OTX, a.vx1)) return;
+  const int ylo = h - r0, yhi = static_cast<int>(min(oy + OTY, a.vy1) - (oy - h)) - r0;
+  float* out = a.tout + (oy - h + r0) * a.ldo + sx;
+#pragma unroll
+  for (int r = 0; r < V; ++r)
+    if (r >= ylo && r < yhi) out[r * a.ldo] = v[r];
+}
+
+#ifndef NU_HS_V3_V
+#define NU_HS_V3_V 16
+#endif
+#ifndef NU_HS_V3_NWY
+#define NU_HS_V3_NWY 8
+#endif
+constexpr int kV3V = NU_HS_V3_V, kV3NWX = 4, kV3NWY = NU_HS_V3_NWY;
+
+#ifndef NU_HS_RPT
+#define NU_HS_RPT 32
+#endif
+#ifndef NU_HS_NWY
+#define NU_HS_NWY 3
+#endif
+constexpr int kRPT = NU_HS_RPT, kNWX = 4, kNWY = NU_HS_NWY;   // 96 x 128 region, 384 threads
+
 }  // namespace hs
 
 int hotspot_max_iters_per_launch() { return kHotspotMaxIters; }
+
+static int hotspot_variant() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("NORTHUP_HS_LEAF");
+    v = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 3;   // 1, 2: earlier leaves (DESIGN)
+  }
+  return v;
+}
 
 int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
                    int64_t ldo, int64_t wm, int64_t wn, int64_t gy0, int64_t gx0, int64_t R,
@@ -150,6 +372,28 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.ry_1 = coef[2];
   a.rz_1 = coef[3];
   a.amb = coef[4];
+  if (hotspot_variant() == 3) {
+    constexpr int RH = kV3V * kV3NWY, RW = 32 * kV3NWX;
+    const int oty = RH - 2 * iters, otx = RW - 2 * iters;
+    const int64_t gy3 = (a.vy1 - a.vy0 + oty - 1) / oty, gx3 = (a.vx1 - a.vx0 + otx - 1) / otx;
+    if (gy3 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy3);
+    const int smem3 = 2 * (RH + 2) * (RW + 2) * 4;
+    cudaFuncSetAttribute(hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem3);
+    hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY><<<dim3(static_cast<unsigned>(gx3), static_cast<unsigned>(gy3)),
+                                             kV3NWX * kV3NWY * 32, smem3, stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v3 launch");
+  }
+  if (hotspot_variant() == 2) {
+    const int oty = kRPT * kNWY - 2 * iters, otx = 32 * kNWX - 2 * iters;
+    const int64_t gy2 = (a.vy1 - a.vy0 + oty - 1) / oty, gx2 = (a.vx1 - a.vx0 + otx - 1) / otx;
+    if (gy2 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy2);
+    hotspot_kernel_v2<kRPT, kNWX, kNWY><<<dim3(static_cast<unsigned>(gx2), static_cast<unsigned>(gy2)),
+                                          kNWX * kNWY * 32, 0, stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v2 launch");
+  }
   const int64_t gy = (a.vy1 - a.vy0 + kTY - 1) / kTY, gx = (a.vx1 - a.vx0 + kTX - 1) / kTX;
   if (gy > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy);
   const size_t smem = 3ull * (kTY + 2 * iters) * (kTX + 2 * iters) * sizeof(float);
