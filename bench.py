@@ -46,6 +46,11 @@ CONFIGS = {
     "cfg5": dict(M=1048576, N=4096, K=4096, cap=8 * GiB, block=None,
                  desc="tall-skinny 1048576x4096x4096 fp32, A streamed from host"),
 }
+HOTSPOT = dict(R=32768, C=32768, iters=256, cap=8 * GiB,
+               desc="HotSpot-2D 32768^2 fp32 grid (P:349 32k inputs) x 256 iterations, pinned host -> "
+                    "HBM (8 GiB cap) -> SMEM, 1 GPU (S§8(f) NEXT-3)")
+HS_FLOPS_PER_UPDATE = 14                 # fp32 ops of one cell update, no contraction (hotspot.cu)
+FP32_LANES_PER_SM, N_SMS = 128, 148      # B200: 4 SMSPs x 32 fp32 lanes; 148 SMs
 NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25      # B200_PROFILING.md nominal dense ratio
 LEAF_KERNELS = {1: "nu::leaf::sm1::leaf_gemm_1sm_kernel", 2: "nu::leaf::sm2::leaf_gemm_2sm_kernel",
                 3: "nu::leaf::sm3::leaf_gemm_2sm_ldg_kernel", 4: "nu::leaf::sm4::leaf_gemm_2sm_tm_kernel"}
@@ -396,6 +401,128 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     return result
 
 
+# ------------------------------------------------------------ HotSpot-2D
+def run_hotspot(args, rank: int, world: int, local_rank: int):
+    """NEXT-3: HotSpot-2D over the tree.  value = in-HBM (single-node HBM tree,
+    grids resident); e2e = HOST -> HBM (8 GiB cap) -> SMEM out-of-core through
+    northup_hotspot with pinned host grids.  Unit: cell updates per second."""
+    import numpy as np
+    import torch
+    import nugen
+    import paper_conf_ipps_chey19_b200 as nu
+    from oracle import hotspot as ohs
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    R, C, iters, cap = HOTSPOT["R"], HOTSPOT["C"], HOTSPOT["iters"], HOTSPOT["cap"]
+    if args.quick:
+        R, C, cap = R // 4, C // 4, cap // 16
+    t, _ = nu.host_tree(1, cap, devices=[local_rank])
+    t.finalize()
+    Tb, Pb, Ob = t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0)
+    T, P, O = host_array(Tb.ptr, R, C), host_array(Pb.ptr, R, C), host_array(Ob.ptr, R, C)
+    nugen.fill(R, C, 6, nugen.MAT_T, "temp", out=T)
+    nugen.fill(R, C, 6, nugen.MAT_P, "power", out=P)
+    th = nu.hbm_tree(local_rank)
+    th.finalize()
+    Td, Pd = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+    Od = torch.empty_like(Td)
+    hT, hP, hO = (th.wrap_device(0, x.data_ptr(), x.numel() * 4) for x in (Td, Pd, Od))
+    stream = torch.cuda.current_stream(dev)
+    st_h, st_o = {}, {}
+
+    def timed(fn, steps, warmup):
+        for _ in range(warmup):
+            fn()
+        torch.cuda.synchronize(dev)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        evs[0].record(stream)
+        for i in range(steps):
+            fn()
+            evs[i + 1].record(stream)
+        torch.cuda.synchronize(dev)
+        return evs[0].elapsed_time(evs[-1]), [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
+
+    with ClockSampler(local_rank) as clk:
+        t_h, per_h = timed(lambda: st_h.update(th.hotspot(hT, hP, hO, R, C, iters)), args.steps, args.warmup)
+        t_o, per_o = timed(lambda: st_o.update(t.hotspot(Tb, Pb, Ob, R, C, iters)), args.steps, args.warmup)
+    o_hbm = Od.cpu().numpy()
+    bitwise = bool(np.array_equal(o_hbm, O))
+    cells = float(R) * C * iters
+    ms_h, ms_o = t_h / args.steps, t_o / args.steps
+    value = cells / (ms_h * 1e-3) / 1e9
+    e2e = cells / (ms_o * 1e-3) / 1e9
+    launches = st_h.get("leaf_launches", 0)
+    leaf_ms = statistics.mean(per_h) / max(1, launches)
+    li = st_h.get("bk", 8)
+    flops_per_launch = HS_FLOPS_PER_UPDATE * float(R) * C * li
+    achieved = flops_per_launch / (leaf_ms * 1e-3) / 1e12
+    ck = clk.summary()
+    f_max = (ck.get("sm_max_mhz") or 1965.0) * 1e6
+    peak = N_SMS * FP32_LANES_PER_SM * f_max / 1e12
+    # parity: sampled blocks against the fp64 oracle (window of border `iters`)
+    k64 = ohs.coeffs(R, C)
+    rng = np.random.default_rng(11)
+    worst, tmax = 0.0, 0.0
+    samples = [(0, 0), (R - 32, C - 32)] + [(int(y), int(x)) for y, x in
+                                            zip(rng.integers(0, R - 32, 2), rng.integers(0, C - 32, 2))]
+    t0 = time.perf_counter()
+    for (y0, x0) in samples:
+        wy0, wx0 = max(0, y0 - iters), max(0, x0 - iters)
+        wy1, wx1 = min(R, y0 + 32 + iters), min(C, x0 + 32 + iters)
+        tw = T[wy0:wy1, wx0:wx1].astype(np.float64)
+        pw = P[wy0:wy1, wx0:wx1].astype(np.float64)
+        for _ in range(iters):
+            tw = ohs._window_step(tw, pw, wy0, wx0, R, C, k64)
+        ref = tw[y0 - wy0:y0 - wy0 + 32, x0 - wx0:x0 - wx0 + 32]
+        worst = max(worst, float(np.abs(O[y0:y0 + 32, x0:x0 + 32] - ref).max()))
+        tmax = max(tmax, float(np.abs(ref).max()))
+    cpu_s = time.perf_counter() - t0
+    cpu_cells = sum((min(R, y + 32 + iters) - max(0, y - iters)) * (min(C, x + 32 + iters) - max(0, x - iters))
+                    for y, x in samples) * iters
+    tol = ohs.tolerance(iters, tmax)
+    result = {
+        "metric": "out-of-core HotSpot-2D cell updates/s (S§8(f) NEXT-3); % slowdown vs in-HBM; roofline frac",
+        "value": round(value, 3), "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_h, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32 (no contraction)",
+        "data": "synthetic (counter-hash temperature 330 +- 10 K, power [0, 0.5))",
+        "config": {"workload": "hotspot: " + HOTSPOT["desc"] + (" [quick: /4 sizes]" if args.quick else ""),
+                   "rows": R, "cols": C, "iters": iters, "hbm_cap_bytes": cap,
+                   "block": st_o.get("bm"), "halo_iters_per_visit": st_o.get("bk"),
+                   "leaf_iters_per_launch": li,
+                   "l2": "grids (4 GiB each) exceed the 126 MB L2; no flush needed"},
+        "e2e": {"value": round(e2e, 3), "unit": "Gcell-updates/s",
+                "h2d_bytes_per_step": int(st_o.get("bytes_h2d", 0)),
+                "d2h_bytes_per_step": int(st_o.get("bytes_d2h", 0)), "ms_per_step": round(ms_o, 3),
+                "leaf_launches_per_step": int(st_o.get("leaf_launches", 0)),
+                "pcie_roofline_gcups": round(cells / (st_o.get("bytes_h2d", 1) / 53e9) / 1e9, 1)},
+        "slowdown_pct_vs_in_hbm": round(100.0 * (ms_o / ms_h - 1.0), 2),
+        "paper_context": {"hotspot_ooc_gap_pct": 15, "note": "APU + SSD vs DRAM (PAPER.md P:381); context only"},
+        "roofline": {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "TFLOP/s",
+                     "frac": round(achieved / peak, 4), "traffic": None,
+                     "peak_basis": f"{N_SMS} SMs x {FP32_LANES_PER_SM} fp32 lanes x clocks.max.sm "
+                                   f"{f_max / 1e6:.0f} MHz (one fp32 op per lane per clock)",
+                     "kernel": "nu::hs::hotspot_kernel_v3", "launch": [R, C, li],
+                     "flops_per_launch": flops_per_launch,
+                     "flops_basis": f"{HS_FLOPS_PER_UPDATE} fp32 ops per useful cell update x R x C x "
+                                    f"iterations per launch (halo recomputation not counted)",
+                     "ms_per_launch": round(leaf_ms, 3), "launches_per_step": launches},
+        "gpu_launches": int(launches * args.steps + st_o.get("leaf_launches", 0) * args.steps),
+        "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise,
+                   "oracle_max_abs_err_sampled_blocks": worst, "oracle_tolerance": tol,
+                   "oracle_ok": bool(worst <= tol), "sampled_blocks": len(samples)},
+        "clocks": ck,
+        "cpu_baseline": {"value": round(cpu_cells / cpu_s / 1e9, 6), "unit": "Gcell-updates/s", "cores": 1,
+                         "kind": "oracle",
+                         "sample": f"{len(samples)} 32x32 blocks with {iters}-cell borders x {iters} iterations "
+                                   f"(fp64 numpy window sweeps), {cpu_s:.1f} s"},
+    }
+    th.destroy()
+    t.destroy()
+    return result
+
+
 # --------------------------------------------------------------- reference
 def run_reference(args):
     """The fp64 CPU oracle as the reference arm (bounded sample per step)."""
@@ -448,7 +575,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default=None, choices=sorted(CONFIGS))
+    ap.add_argument("--config", default=None, choices=sorted(CONFIGS) + ["hotspot"])
     ap.add_argument("--k-chunk", type=int, default=2048)
     ap.add_argument("--quick", action="store_true", help="sizes / 4 (smoke-testing the bench)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -472,6 +599,10 @@ def main():
         local_rank %= args.device_mod
 
     if args.impl == "reference":
+        if rank == 0 and args.config == "hotspot":
+            print(json.dumps({"impl": "reference", "unavailable": "the HotSpot-2D oracle is timed as cpu_baseline "
+                                                                  "in the ours line (no separate reference arm)"}))
+            return
         if rank == 0:
             print(json.dumps(run_reference(args)), flush=True)
         return
@@ -484,7 +615,8 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
         else:
             dist.init_process_group(args.dist_backend)
-    res = run_ours(args, rank, world, local_rank)
+    res = run_hotspot(args, rank, world, local_rank) if args.config == "hotspot" else \
+        run_ours(args, rank, world, local_rank)
     if rank == 0 and res is not None:
         print(json.dumps(res), flush=True)
     if world > 1:
