@@ -142,7 +142,7 @@ struct RunCtx {
   std::vector<char*> base;             // per plan buffer (host/device pointers)
   std::vector<const northup_buf_s*> file;   // per plan buffer: file handle or NULL
   const std::vector<char>* needs_event;
-  const std::vector<char>* needs_remote;   // local op a peer process waits for
+  const std::vector<uint64_t>* needs_remote;   // per local op: mask of sibling processes waiting
   const northup_gemm_opts* o;
   bool timing;
   int local = -1;                          // multi-process siblings: the local worker
@@ -217,7 +217,9 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       cudaEvent_t ev = w->events[op.deps[d]];
       if (q.worker != wi && c.local >= 0) {
         // a sibling in another process: device-side wait on its flag word
-        int rc = stream_wait_flag(s, c.t->peers[q.worker].flags + 1 + op.deps[d], c.gen);
+        // a sibling in another process: device-side wait on OUR flag word for
+        // that op, which the producer writes remotely after the op
+        int rc = stream_wait_flag(s, c.t->flags + P.num_workers + op.deps[d], c.gen);
         if (rc) return rc;
         continue;
       }
@@ -268,8 +270,14 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       mark(c, c.issued, i);
     }
     if (c.local >= 0 && (*c.needs_remote)[i]) {
-      int rc = stream_write_flag(s, c.t->flags + 1 + i, c.gen);
-      if (rc) return rc;
+      // publish op i to every sibling process that waits for it: a fenced
+      // remote store into its flag words (consumers only ever poll local memory)
+      const uint64_t mask = (*c.needs_remote)[i];
+      for (int q = 0; q < P.num_workers; ++q)
+        if (mask >> q & 1) {
+          int rc = stream_write_flag(s, c.t->peers[q].flags + P.num_workers + i, c.gen);
+          if (rc) return rc;
+        }
     }
   }
   if (c.local >= 0 && c.cross) {
@@ -283,9 +291,11 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       cudaStreamWaitEvent(w->streams[0], j, 0);
       cudaEventDestroy(j);
     }
-    int rc = stream_write_flag(w->streams[0], c.t->flags, c.gen);
+    int rc = 0;
     for (int q = 0; q < P.num_workers && !rc; ++q)
-      if (q != wi) rc = stream_wait_flag(w->streams[0], c.t->peers[q].flags, c.gen);
+      if (q != wi) rc = stream_write_flag(w->streams[0], c.t->peers[q].flags + wi, c.gen);
+    for (int q = 0; q < P.num_workers && !rc; ++q)
+      if (q != wi) rc = stream_wait_flag(w->streams[0], c.t->flags + q, c.gen);
     if (rc) return rc;
   }
   if (capture_out) {
@@ -461,7 +471,7 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   }
   ctx.needs_event = &needs;
   ctx.cross = cross;
-  std::vector<char> needs_remote(P.ops.size(), 0);
+  std::vector<uint64_t> needs_remote(P.ops.size(), 0);
   ctx.needs_remote = &needs_remote;
   if (lw >= 0 && cross) {
     if (t->peer_key != peer_key_of(P.M, P.N, P.K, o) ||
@@ -472,7 +482,8 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
         return fail(NU_ESTATE, "multi-process siblings: worker %d was not imported", q);
     for (const northup_op& op : P.ops)
       for (int d = 0; d < op.ndeps; ++d)
-        if (op.worker != lw && P.ops[op.deps[d]].worker == lw) needs_remote[op.deps[d]] = 1;
+        if (op.worker != lw && P.ops[op.deps[d]].worker == lw)
+          needs_remote[op.deps[d]] |= uint64_t(1) << op.worker;
     ctx.gen = ++t->gen;
   }
   ctx.issued.assign(P.ops.size(), 0);

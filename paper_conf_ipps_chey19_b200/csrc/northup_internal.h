@@ -88,7 +88,7 @@ struct northup_tree_s {
     uint32_t* flags = nullptr;   // IPC-mapped flag words of that sibling
   };
   std::vector<Peer> peers;             // per plan worker
-  uint32_t* flags = nullptr;           // this process's flag words: [0] = done, [1 + op] = op
+  uint32_t* flags = nullptr;           // this process's flag words: [w] = done of sibling w, [G + op]
   uint64_t flags_cap = 0;              // words
   std::vector<void*> flag_graveyard;   // outgrown flag buffers (peers may still map them)
   uint32_t gen = 0;                    // generation of the current call (monotonic)

@@ -9,15 +9,18 @@
 //   northup_peer_import(t, w, blob)   map sibling w's arena and flag words
 //
 // Every process builds the same plan (same tree, sizes and options), so op
-// indices agree.  A dependency of a local op on a sibling's op i becomes a
-// device-side wait `cuStreamWaitValue32(flags_w[1 + i] >= gen)`; the sibling
-// writes `gen` there with `cuStreamWriteValue32` after op i (the default write
-// carries a memory fence, so the data the op produced is visible first).  No
-// host thread blocks on a peer: the waits form a DAG because every dependency
-// points backwards in plan order and each stream is FIFO in plan order.  At
-// the end of a call every process writes its done word and waits for all
-// siblings' done words (a device-side join), so no sibling can still be
-// pulling from an arena when northup_gemm returns.
+// indices agree.  Each process owns G + nops flag words in its own HBM:
+// [w] = sibling w's done word, [G + i] = op i.  A dependency of a local op on a
+// sibling's op i is a device-side wait on the LOCAL word
+// `cuStreamWaitValue32(flags[G + i] >= gen)`; after op i the producing sibling
+// stores `gen` into the flag words of every process that waits for it with
+// `cuStreamWriteValue32` on the IPC-mapped peer address (a fenced remote
+// store: the op's data is visible first).  Consumers only poll local memory.
+// No host thread blocks on a peer: the waits form a DAG because every
+// dependency points backwards in plan order and each stream is FIFO in plan
+// order.  At the end of a call every process stores its done word into all
+// siblings and waits for theirs (a device-side join), so no sibling can still
+// be pulling from an arena when northup_gemm returns.
 #include <string.h>
 
 #include "northup_internal.h"
@@ -133,6 +136,7 @@ int northup_peer_export(northup_tree_t t, int64_t M, int64_t N, int64_t K, const
   if (rc) return rc;
   const int lw = local_worker(t, P);
   if (lw < 0) return fail(NU_ESTATE, "the local node is not a worker of this plan");
+  if (P.num_workers > 64) return fail(NU_ENOTSUP, "multi-process siblings support at most 64 GPUs");
   const Node& ln = t->nodes[t->local_node];
   cudaError_t e = cudaSetDevice(ln.phys);
   if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
@@ -147,7 +151,7 @@ int northup_peer_export(northup_tree_t t, int64_t M, int64_t N, int64_t K, const
   }
   if (!t->nodes[t->local_node].arena_owned)
     return fail(NU_ENOTSUP, "peer export needs a library-owned arena (not northup_tree_set_arena)");
-  const uint64_t words = P.ops.size() + 1;
+  const uint64_t words = P.ops.size() + P.num_workers;
   if (words > t->flags_cap) {
     // Outgrown flag buffers stay allocated until destroy: a slower sibling may
     // still wait on them (waits are GEQ on a monotonic generation).
