@@ -235,14 +235,30 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     shared_peers = False
     if world > 1 and not args.no_shared_staging:
         # NEXT-1: siblings of a grid row / column share A / B panels over
-        # NVLink; exchange the CUDA IPC handles of arenas and flag words
-        blob = t.peer_export(M, N, K, ooc_opts)
+        # NVLink; exchange the CUDA IPC handles of arenas and flag words.  If
+        # any rank cannot export or import, every rank falls back to
+        # unshared staging (no cross-process dependency is then planned).
+        try:
+            blob = t.peer_export(M, N, K, ooc_opts)
+        except nu.NorthupError as ex:
+            log(f"[rank {rank}] peer export failed ({ex}); falling back to unshared staging")
+            blob = None
         blobs = [None] * world
         dist.all_gather_object(blobs, blob)
-        for w, bl in enumerate(blobs):
-            if w != rank:
-                t.peer_import(w, bl)
-        shared_peers = True
+        ok = all(bl is not None for bl in blobs)
+        if ok:
+            try:
+                for w, bl in enumerate(blobs):
+                    if w != rank:
+                        t.peer_import(w, bl)
+            except nu.NorthupError as ex:
+                log(f"[rank {rank}] peer import failed ({ex}); falling back to unshared staging")
+                ok = False
+        oks = [None] * world
+        dist.all_gather_object(oks, ok)
+        shared_peers = all(oks)
+        if not shared_peers:
+            ooc_opts = nu.make_opts(k_chunk=kc, shared_staging=-1)
     stream = torch.cuda.current_stream(dev)
 
     def barrier():
