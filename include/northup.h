@@ -62,6 +62,11 @@ extern "C" {
 #define NU_SCHED_AUTO 0
 #define NU_SCHED_S1 1 /* paper-literal: row shard m stays at l+1, column shards stream */
 #define NU_SCHED_S2 2 /* C block resident, K panels stream, staggered C drain */
+#define NU_SCHED_QUEUE 3 /* S§8(f) NEXT-2: C is cut into tiles held in one
+                            work queue per HBM sibling; each sibling pops tiles from the tail of its
+                            own queue and, when empty, steals from the head of another's; a tile is
+                            an S2 sub-problem (C tile resident, K panels stream, tile drained).
+                            HOST root, single process; no shared staging, no graphs. */
 
 typedef struct northup_tree_s* northup_tree_t;
 typedef struct northup_buf_s* northup_buf_t;
@@ -217,6 +222,8 @@ typedef struct {
   int shared_staging;    /* 1 when the plan used NVLink-shared staging (opts->shared_staging) */
   uint64_t bytes_p2p;    /* bytes pulled from sibling HBM (shared staging), all GPUs */
   double t_p2p_ms;       /* sum over GPUs of busy time of sibling pulls (timing mode) */
+  int64_t tasks;         /* NU_SCHED_QUEUE: C tiles */
+  int64_t tasks_stolen;  /* NU_SCHED_QUEUE: tiles a sibling took from another sibling's queue */
 } northup_stats;
 
 /* C = A.B (no alpha/beta; C overwritten — reading R3), A (M x K), B (K x N),

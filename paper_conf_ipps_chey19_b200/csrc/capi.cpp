@@ -86,6 +86,8 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
       (A->storage != NU_FILE || B->storage != NU_FILE || C->storage != NU_FILE))
     return fail(NU_EINVAL, "a FILE root needs A, B and C as files (northup_open_file / alloc)");
 
+  if (o && o->schedule == NU_SCHED_QUEUE && (t->nodes[0].storage != NU_HOST || t->local_node >= 0))
+    return fail(NU_ENOTSUP, "NU_SCHED_QUEUE needs a HOST root in one process");
   t->busy = true;
   Plan plan;
   const bool a_al = reinterpret_cast<uintptr_t>(A->ptr) % 16 == 0;
@@ -97,7 +99,10 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
     st->t_plan_ms = t1 - t0;
     int prev = 0;
     cudaGetDevice(&prev);
-    rc = execute_plan(t, plan, A, B, C, o, st);
+    if (o && o->schedule == NU_SCHED_QUEUE)
+      rc = execute_queue(t, M, N, K, A, B, C, o, st);   // tiles popped at run time
+    else
+      rc = execute_plan(t, plan, A, B, C, o, st);
     if (!rc && o && o->replicate_result) rc = gather_replicas(t, plan, C, st);
     cudaSetDevice(prev);
   }

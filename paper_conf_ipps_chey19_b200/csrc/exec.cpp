@@ -25,7 +25,10 @@
 #include <mutex>
 #include <thread>
 
+#include <deque>
+
 #include "northup_internal.h"
+#include "plan_builder.h"
 
 struct WorkerState {
   int node = -1;
@@ -245,6 +248,8 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
                               cudaMemcpyDefault, s);
       if (e != cudaSuccess) return cuda_fail(e, "copy");
     } else if (op.op == NU_OP_LEAF) {
+      int slow_us = 0;
+      if (debug_slow_sibling(&slow_us) == wi && slow_us > 0) debug_spin(1000ll * slow_us, s);
       const float* a = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);
       const float* b = reinterpret_cast<const float*>(c.base[op.b_buf] + op.b_off * 4);
       float* cc = reinterpret_cast<float*>(c.base[op.c_buf] + op.c_off * 4);
@@ -564,6 +569,141 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     }
     st->t_io_ms = ctx.io_ms;
   }
+  return 0;
+}
+
+// ------------------------------------------------- NU_SCHED_QUEUE (NEXT-2)
+// One host thread per HBM sibling.  A thread pops a C tile from the tail of
+// its own queue (or, when that is empty, steals from the head of the longest
+// other queue), appends the tile's ops to its private op list through
+// its own rectangle tracker (so dependencies on its earlier tiles — panel
+// slots, the two C-tile buffers — are exact) and issues them on its streams.
+// A thread keeps at most two tiles in flight: before popping it waits for the
+// tile before the previous one, so a slower sibling pops fewer tiles.
+// NORTHUP_DEBUG_SLOW_SIBLING="w,us" holds sibling w's compute stream for us
+// microseconds before each leaf launch, in every schedule (a test hook that
+// emulates an asymmetric tree, Fig. 2).
+int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_buf_s* a, northup_buf_s* b,
+                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st) {
+  std::vector<int> hbm;
+  for (int ch : t->nodes[0].children) hbm.push_back(ch);
+  const int G = static_cast<int>(hbm.size());
+  const int64_t kc = (o && o->k_chunk > 0) ? o->k_chunk : kDefaultKChunk;
+  const int npass = o ? o->npass : 0;
+  QueueShape q;
+  int rc = choose_queue(t, hbm, M, N, K, kc, &q);
+  if (rc) return rc;
+  for (int w = 0; w < G; ++w) {
+    rc = ensure_arena(t, hbm[w], q.arena_bytes);
+    if (rc) return rc;
+  }
+  std::vector<std::deque<int64_t>> queues;
+  for (auto& v : queue_initial(G, q)) queues.emplace_back(v.begin(), v.end());
+  std::mutex qm;
+  int slow_us = 0;
+  const int slow_w = debug_slow_sibling(&slow_us);
+  std::vector<int> rcs(G, 0);
+  std::vector<std::string> errs(G);
+  std::vector<northup_stats> wst(G);
+  std::vector<int64_t> stolen(G, 0), popped(G, 0);
+
+  auto pop = [&](int w, bool* st_) -> int64_t {
+    std::lock_guard<std::mutex> g(qm);
+    if (!queues[w].empty()) {
+      const int64_t x = queues[w].back();
+      queues[w].pop_back();
+      return x;
+    }
+    int v = -1;
+    for (int u = 0; u < G; ++u)
+      if (u != w && !queues[u].empty() && (v < 0 || queues[u].size() > queues[v].size())) v = u;
+    if (v < 0) return -1;
+    const int64_t x = queues[v].front();
+    queues[v].pop_front();
+    *st_ = true;
+    return x;
+  };
+
+  auto body = [&](int w) -> int {
+    WorkerState* ws = worker_for_node(t, hbm[w]);
+    if (!ws) return fail(NU_ESTATE, "no worker state for node %d", hbm[w]);
+    cudaError_t e = cudaSetDevice(ws->device);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+    Plan Pw;
+    Builder B;
+    B.P = &Pw;
+    const int bA = B.add_buf(B_USER_A, 0, -1, 0), bB = B.add_buf(B_USER_B, 0, -1, 0);
+    const int bC = B.add_buf(B_USER_C, 0, -1, 0), bAr = B.add_buf(B_ARENA, hbm[w], 0, q.arena_bytes);
+    char* base[4] = {static_cast<char*>(a->ptr), static_cast<char*>(b->ptr), static_cast<char*>(c->ptr),
+                     static_cast<char*>(t->nodes[hbm[w]].arena)};
+    std::vector<cudaEvent_t> evs;
+    std::deque<cudaEvent_t> inflight;
+    int64_t pctr = 0, ntask = 0;
+    int result = 0;
+    for (;;) {
+      if (inflight.size() >= 2) {
+        e = cudaEventSynchronize(inflight.front());
+        if (e != cudaSuccess) { result = cuda_fail(e, "tile completion"); break; }
+        inflight.pop_front();
+      }
+      bool was_stolen = false;
+      const int64_t task = pop(w, &was_stolen);
+      if (task < 0) break;
+      popped[w]++;
+      stolen[w] += was_stolen;
+      const size_t first = Pw.ops.size();
+      emit_task(B, 0, bAr, q, task, static_cast<int>(ntask & 1), &pctr, bA, bB, bC, M, N, K, &wst[w]);
+      ++ntask;
+      if (B.overflow) { result = fail(NU_ENOTSUP, "dependency fan-in above 16"); break; }
+      for (size_t i = first; i < Pw.ops.size() && !result; ++i) {
+        const northup_op& op = Pw.ops[i];
+        cudaStream_t s = ws->streams[op.stream];
+        for (int d = 0; d < op.ndeps; ++d) cudaStreamWaitEvent(s, evs[op.deps[d]], 0);
+        if (op.op == NU_OP_COPY) {
+          e = cudaMemcpy2DAsync(base[op.dst_buf] + op.dst_off * 4, op.dst_ld * 4, base[op.src_buf] + op.src_off * 4,
+                                op.src_ld * 4, op.cols * 4, op.rows, cudaMemcpyDefault, s);
+          if (e != cudaSuccess) result = cuda_fail(e, "copy");
+        } else {
+          if (w == slow_w && slow_us > 0) debug_spin(1000ll * slow_us, s);
+          result = leaf_gemm_launch(reinterpret_cast<const float*>(base[op.a_buf] + op.a_off * 4), op.lda,
+                                    reinterpret_cast<const float*>(base[op.b_buf] + op.b_off * 4), op.ldb,
+                                    reinterpret_cast<float*>(base[op.c_buf] + op.c_off * 4), op.ldc, op.m, op.n,
+                                    op.k, op.accumulate, kc, npass, s);
+        }
+        cudaEvent_t ev;
+        e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventRecord(ev, s);
+        if (e != cudaSuccess && !result) result = cuda_fail(e, "event");
+        evs.push_back(ev);
+      }
+      if (result) break;
+      inflight.push_back(evs.back());   // the tile's drain (D2H) is its last op
+    }
+    for (cudaStream_t s : ws->streams) {
+      e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess && !result) result = cuda_fail(e, "stream synchronize");
+    }
+    for (cudaEvent_t ev : evs) cudaEventDestroy(ev);
+    return result;
+  };
+  std::vector<std::thread> th;
+  for (int w = 0; w < G; ++w)
+    th.emplace_back([&, w] {
+      rcs[w] = body(w);
+      if (rcs[w]) errs[w] = northup_last_error();
+    });
+  for (auto& x : th) x.join();
+  for (int w = 0; w < G; ++w)
+    if (rcs[w]) return fail(rcs[w], "queue worker %d: %s", w, errs[w].c_str());
+  st->bytes_h2d = st->bytes_d2h = 0;
+  st->leaf_launches = 0;
+  for (int w = 0; w < G; ++w) {
+    st->bytes_h2d += wst[w].bytes_h2d;
+    st->bytes_d2h += wst[w].bytes_d2h;
+    st->leaf_launches += wst[w].leaf_launches;   // one launch per leaf op (bk = k_chunk)
+    st->tasks_stolen += stolen[w];
+  }
+  st->tasks = q.Tr * q.Tc;
   return 0;
 }
 

@@ -4,6 +4,7 @@
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
 #include <stdlib.h>
 
 #include <atomic>
@@ -55,6 +56,27 @@ int default_leaf_variant() {
     env_variant = (v && v[0] >= '1' && v[0] <= '4') ? v[0] - '0' : kDefaultLeafVariant;
   }
   return env_variant;
+}
+
+// Test hook (NORTHUP_DEBUG_SLOW_SIBLING="w,us", exec.cpp): a one-thread kernel
+// that holds a stream for `ns` nanoseconds, emulating a slower sibling.
+__global__ void debug_spin_kernel(long long ns) {
+  const long long t0 = clock64();
+  const long long cycles = ns * 2;   // ~2 GHz
+  while (clock64() - t0 < cycles) __nanosleep(1000);
+}
+
+int debug_spin(long long ns, cudaStream_t s) {
+  debug_spin_kernel<<<1, 1, 0, s>>>(ns);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : cuda_fail(e, "debug_spin_kernel");
+}
+
+int debug_slow_sibling(int* us) {
+  int w = -1, t = 0;
+  if (const char* e = getenv("NORTHUP_DEBUG_SLOW_SIBLING")) sscanf(e, "%d,%d", &w, &t);
+  *us = t;
+  return w;
 }
 
 bool leaf_tma_legal(const void* p, int64_t ld) {

@@ -124,11 +124,29 @@ struct Plan {
 
 int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
                const northup_gemm_opts* o, Plan* out);
+int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_buf_s* a,
+                  northup_buf_s* b, northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
 // a_aligned / b_aligned: the root-tier device pointers are 16-B aligned
 // (only consulted for an HBM root, where the leaf reads them in place).
 int build_plan_ex(const northup_tree_s* t, int64_t M, int64_t N, int64_t K,
                   const northup_gemm_opts* o, bool a_aligned, bool b_aligned, Plan* out);
 int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc);
+
+// NU_SCHED_QUEUE (S§8(f) NEXT-2): C tiles in per-sibling work queues.
+struct QueueShape {
+  int64_t tm = 0, tn = 0, bk = 0;   // tile rows / cols, K panel
+  int64_t Tr = 0, Tc = 0;           // tile grid
+  uint64_t arena_bytes = 0;         // per sibling: 2 C-tile buffers + kSlots panel slots
+};
+int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N,
+                 int64_t K, int64_t kc, QueueShape* q);
+// Initial queues: tiles in row-major order, contiguous chunks per sibling.
+std::vector<std::vector<int64_t>> queue_initial(int G, const QueueShape& q);
+struct Builder;
+// Append the ops of tile `task` for sibling w (arena buffer `arena`, C-tile
+// buffer `cslot` of 2, panel-slot counter `pctr`) to B.
+void emit_task(Builder& B, int w, int arena, const QueueShape& q, int64_t task, int cslot,
+               int64_t* pctr, int A, int Bb, int C, int64_t M, int64_t N, int64_t K, northup_stats* st);
 int region_of(int G, int64_t M, int64_t N, int r, int64_t* r0, int64_t* r1, int64_t* c0,
               int64_t* c1);
 int validate_tree(const northup_tree_s* t);
@@ -152,6 +170,11 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
                    int64_t C, int iters, const float coef[5], cudaStream_t stream);
 int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t iters,
                        const northup_hotspot_opts* o, const northup_hotspot_coeffs* k, Plan* out);
+
+// Test hooks: a kernel that holds a stream for `ns` ns; the sibling (and
+// microseconds) named by NORTHUP_DEBUG_SLOW_SIBLING="w,us" (-1 = none).
+int debug_spin(long long ns, cudaStream_t s);
+int debug_slow_sibling(int* us);
 
 // --------------------------------------------------------------- executor
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,

@@ -810,6 +810,79 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
 
 }  // namespace
 
+// ------------------------------------------------- NU_SCHED_QUEUE (NEXT-2)
+// The paper's runtime keeps a task queue at each node and
+// balances work by popping local tasks and stealing remote ones (P:393-395,
+// there between CPU and GPU).  Here the tasks are C tiles of an M x N GEMM and
+// the queues belong to the HBM siblings: about four tiles per sibling, each an
+// S2 sub-problem with its C tile resident in one of two tile buffers (so the
+// next tile's panels stream while the previous one drains).
+int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N, int64_t K,
+                 int64_t kc, QueueShape* q) {
+  const int G = static_cast<int>(hbm.size());
+  uint64_t cap = 0;
+  for (int h : hbm)
+    if (t->nodes[h].capacity) cap = cap ? std::min(cap, t->nodes[h].capacity) : t->nodes[h].capacity;
+  int Pr = 1, Pc = 1;
+  partition_grid(G, M, N, &Pr, &Pc);
+  const int64_t bk = std::min<int64_t>(std::max<int64_t>(kc, 4), rup(K, 4));
+  auto bytes = [&](int64_t tm, int64_t tn) {
+    return 4ull * (2ull * tm * pad_ld(tn) + uint64_t(kSlots) * (uint64_t(tm) * pad_ld(bk) + uint64_t(bk) * pad_ld(tn)));
+  };
+  // start from a 2 x 2 split of each sibling's region, refine until it fits
+  int64_t Tr = std::min<int64_t>(M, 2 * Pr), Tc = std::min<int64_t>(N, 2 * Pc);
+  for (;;) {
+    const int64_t tm = rup(cdiv(M, Tr), 8), tn = rup(cdiv(N, Tc), 8);
+    if (!cap || bytes(tm, tn) <= cap) {
+      q->tm = tm;
+      q->tn = tn;
+      q->bk = bk;
+      q->Tr = cdiv(M, tm);
+      q->Tc = cdiv(N, tn);
+      q->arena_bytes = bytes(tm, tn);
+      return 0;
+    }
+    if (tm <= 8 && tn <= 8)
+      return fail(NU_ENOMEM, "HBM capacity %llu B below the smallest queue tile", (unsigned long long)cap);
+    if (tm >= tn && tm > 8) Tr = std::min<int64_t>(M, Tr * 2);
+    else Tc = std::min<int64_t>(N, Tc * 2);
+  }
+}
+
+std::vector<std::vector<int64_t>> queue_initial(int G, const QueueShape& q) {
+  const int64_t T = q.Tr * q.Tc;
+  std::vector<std::vector<int64_t>> out(G);
+  for (int w = 0; w < G; ++w)
+    for (int64_t i = T * w / G; i < T * (w + 1) / G; ++i) out[w].push_back(i);
+  return out;
+}
+
+void emit_task(Builder& B, int w, int arena, const QueueShape& q, int64_t task, int cslot, int64_t* pctr,
+               int A, int Bb, int C, int64_t M, int64_t N, int64_t K, northup_stats* st) {
+  const int64_t ti = task / q.Tc, tj = task % q.Tc;
+  const int64_t i0 = ti * q.tm, j0 = tj * q.tn;
+  const int64_t m = std::min(q.tm, M - i0), n = std::min(q.tn, N - j0);
+  const int64_t ldC = pad_ld(q.tn), ldA = pad_ld(q.bk), ldB = pad_ld(q.tn);
+  const int64_t offC = static_cast<int64_t>(cslot) * q.tm * ldC;
+  const int64_t base = 2 * q.tm * ldC;
+  for (int64_t k0 = 0, p = 0; k0 < K; k0 += q.bk, ++p) {
+    const int64_t kk = std::min(q.bk, K - k0);
+    const int sl = static_cast<int>((*pctr)++ % kSlots);
+    const int64_t offA = base + sl * (q.tm * ldA + q.bk * ldB), offB = offA + q.tm * ldA;
+    B.emit(make_copy(w, S_H2D, A, i0 * K + k0, K, arena, offA, ldA, m, kk),
+           {{A, i0 * K + k0, K, m, kk, false}, {arena, offA, ldA, m, kk, true}});
+    B.emit(make_copy(w, S_H2D, Bb, k0 * N + j0, N, arena, offB, ldB, kk, n),
+           {{Bb, k0 * N + j0, N, kk, n, false}, {arena, offB, ldB, kk, n, true}});
+    st->bytes_h2d += 4ull * (uint64_t(m) * kk + uint64_t(kk) * n);
+    B.emit(make_leaf(w, arena, offA, ldA, arena, offB, ldB, arena, offC, ldC, m, n, kk, p > 0 ? 1 : 0),
+           {{arena, offA, ldA, m, kk, false}, {arena, offB, ldB, kk, n, false}, {arena, offC, ldC, m, n, true}});
+    st->leaf_launches++;
+  }
+  B.emit(make_copy(w, S_D2H, arena, offC, ldC, C, i0 * N + j0, N, m, n),
+         {{arena, offC, ldC, m, n, false}, {C, i0 * N + j0, N, m, n, true}});
+  st->bytes_d2h += 4ull * m * n;
+}
+
 // Which HBM nodes compute, and what sits above them.
 int build_plan(const northup_tree_s* t, int64_t M, int64_t N, int64_t K, const northup_gemm_opts* o,
                Plan* out) {
@@ -846,7 +919,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   if (P.kc % 4) return fail(NU_EINVAL, "k_chunk must be a multiple of 4");
   P.npass = o ? o->npass : 0;   // 0 = library default (leaf_host.cu)
   const int sched = o ? o->schedule : NU_SCHED_AUTO;
-  if (sched < NU_SCHED_AUTO || sched > NU_SCHED_S2) return fail(NU_EINVAL, "unknown schedule");
+  if (sched < NU_SCHED_AUTO || sched > NU_SCHED_QUEUE) return fail(NU_EINVAL, "unknown schedule");
   Builder B;
   B.P = &P;
   const int A = B.add_buf(B_USER_A, 0, -1, 4ull * M * K);
@@ -908,6 +981,40 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   P.worker_node = hbm;
   st.num_gpus = G;
   if (M == 0 || N == 0 || K == 0) return 0;
+  if (sched == NU_SCHED_QUEUE) {
+    // The executor pops tiles at run time; the plan API shows the schedule
+    // with no steals: each sibling takes its own queue in order, siblings in
+    // round-robin (every op, dependency and byte count is the same as at run
+    // time; only the tile-to-sibling assignment is dynamic).
+    if (t->local_node >= 0) return fail(NU_ENOTSUP, "NU_SCHED_QUEUE runs in one process");
+    QueueShape q;
+    rc = choose_queue(t, hbm, M, N, K, P.kc, &q);
+    if (rc) return rc;
+    std::vector<int> arena(G);
+    for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, q.arena_bytes);
+    auto queues = queue_initial(G, q);
+    std::vector<int64_t> pctr(G, 0), done(G, 0);
+    for (bool more = true; more;) {
+      more = false;
+      for (int w = 0; w < G; ++w) {
+        if (done[w] >= static_cast<int64_t>(queues[w].size())) continue;
+        emit_task(B, w, arena[w], q, queues[w][done[w]], static_cast<int>(done[w] & 1), &pctr[w], A, Bb, C,
+                  M, N, K, &st);
+        ++done[w];
+        more = true;
+      }
+    }
+    st.bm = q.tm;
+    st.bn = q.tn;
+    st.bk = q.bk;
+    st.tasks = q.Tr * q.Tc;
+    st.hbm_peak_bytes = q.arena_bytes;
+    st.schedule = NU_SCHED_QUEUE;
+    st.ops = static_cast<int64_t>(P.ops.size());
+    for (const northup_op& op : P.ops)
+      if (op.op == NU_OP_COPY) st.copies++;
+    return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
+  }
   std::vector<EdgeCtx> xs;
   std::vector<int> uses;
   for (int w = 0; w < G; ++w) {

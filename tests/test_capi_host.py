@@ -461,3 +461,27 @@ def test_set_local_errors():
         t.peer_export(64, 64, 64)            # not finalized
     assert e.value.code == nu.NU_ESTATE
     t.destroy()
+
+
+# ------------------------------------------- queue scheduling (NEXT-2)
+@pytest.mark.parametrize("M,N,K,G,cap,kc", [
+    (512, 512, 640, 2, 0, 64), (600, 300, 200, 3, 0, 64), (1000, 700, 500, 4, 1_500_000, 128),
+    (130, 90, 70, 1, 0, 32)])
+def test_queue_plan_replays_exactly(M, N, K, G, cap, kc):
+    """NU_SCHED_QUEUE: tiles of ~4 per sibling, each an S2 sub-problem with two
+    C-tile buffers; the plan API's no-steal unrolling replays exactly in any
+    dependency-respecting order and moves the closed-form bytes."""
+    A = nugen.fill(M, K, 8, 1, "int")
+    B = nugen.fill(K, N, 8, 2, "int")
+    ref = A.astype(np.float64) @ B.astype(np.float64)
+    t, _ = nu.host_tree(G, cap)
+    p = t.plan(M, N, K, nu.make_opts(schedule=nu.NU_SCHED_QUEUE, k_chunk=kc))
+    s = p.stats()
+    assert s["schedule"] == nu.NU_SCHED_QUEUE and s["tasks"] >= min(4 * G, -(-M // 8) * -(-N // 8))
+    for seed in range(3):
+        assert np.array_equal(simulate(p, A, B, M, N, K, rng=random.Random(seed)), ref)
+    tr, tc = -(-M // s["bm"]), -(-N // s["bn"])
+    assert s["bytes_h2d"] == 4 * K * (M * tc + N * tr) and s["bytes_d2h"] == 4 * M * N
+    if cap:
+        assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
+    t.destroy()

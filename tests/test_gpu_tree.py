@@ -225,3 +225,27 @@ def test_shared_staging_virtual_siblings(G, M, N, K, cap, kind):
     assert s1["bytes_p2p"] > 0 and s1["bytes_h2d"] < s0["bytes_h2d"] and s1["t_p2p_ms"] > 0
     assert np.array_equal(C1, C0)
     check(C1, a, b, kind)
+
+
+@pytest.mark.parametrize("G,M,N,K,cap,kind", [(2, 1024, 768, 2048, 0, "int"), (4, 1500, 1300, 1100, 0, "uniform"),
+                                               (3, 900, 900, 1024, 4 << 20, "uniform")])
+def test_queue_schedule_matches_static_and_oracle(G, M, N, K, cap, kind):
+    """NEXT-2: tiles popped from per-sibling queues at run time give the
+    oracle's C, bitwise equal to the static S2 plan (same K-chunk sequence
+    per element)."""
+    Cq, a, b, sq = run_host(M, N, K, G=G, cap=cap, kind=kind, seed=6, k_chunk=512,
+                            schedule=nu.NU_SCHED_QUEUE)
+    Cs, _, _, _ = run_host(M, N, K, G=G, cap=cap, kind=kind, seed=6, k_chunk=512, schedule=nu.NU_SCHED_S2)
+    assert sq["schedule"] == nu.NU_SCHED_QUEUE and sq["tasks"] >= 4
+    check(Cq, a, b, kind)
+    assert np.array_equal(Cq, Cs)
+
+
+def test_queue_schedule_steals_from_a_slow_sibling(monkeypatch):
+    """A sibling that is slow to pop (test hook emulating an asymmetric tree,
+    Fig. 2) loses tiles to the fast one: steals happen and C is still exact."""
+    monkeypatch.setenv("NORTHUP_DEBUG_SLOW_SIBLING", "1,3000")   # +3 ms per leaf on sibling 1
+    M, N, K = 2048, 2048, 1024
+    C, a, b, st = run_host(M, N, K, G=2, kind="int", seed=2, k_chunk=512, schedule=nu.NU_SCHED_QUEUE)
+    assert st["tasks_stolen"] > 0
+    check(C, a, b, "int")
