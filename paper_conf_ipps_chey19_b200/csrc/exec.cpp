@@ -248,8 +248,8 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
                               cudaMemcpyDefault, s);
       if (e != cudaSuccess) return cuda_fail(e, "copy");
     } else if (op.op == NU_OP_LEAF) {
-      int slow_us = 0;
-      if (debug_slow_sibling(&slow_us) == wi && slow_us > 0) debug_spin(1000ll * slow_us, s);
+      int slow_pct = 0;
+      if (debug_slow_sibling(&slow_pct) == wi && slow_pct > 0) debug_spin(debug_slow_ns(slow_pct, op.m, op.n, op.k), s);
       const float* a = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);
       const float* b = reinterpret_cast<const float*>(c.base[op.b_buf] + op.b_off * 4);
       float* cc = reinterpret_cast<float*>(c.base[op.c_buf] + op.c_off * 4);
@@ -580,9 +580,9 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
 // slots, the two C-tile buffers — are exact) and issues them on its streams.
 // A thread keeps at most two tiles in flight: before popping it waits for the
 // tile before the previous one, so a slower sibling pops fewer tiles.
-// NORTHUP_DEBUG_SLOW_SIBLING="w,us" holds sibling w's compute stream for us
-// microseconds before each leaf launch, in every schedule (a test hook that
-// emulates an asymmetric tree, Fig. 2).
+// NORTHUP_DEBUG_SLOW_SIBLING="w,pct" holds sibling w's compute stream for pct %
+// of each leaf's nominal time before launching it, in every schedule (a test
+// hook that emulates an asymmetric tree, Fig. 2: a slower GPU).
 int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_buf_s* a, northup_buf_s* b,
                   northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st) {
   std::vector<int> hbm;
@@ -600,8 +600,8 @@ int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_bu
   std::vector<std::deque<int64_t>> queues;
   for (auto& v : queue_initial(G, q)) queues.emplace_back(v.begin(), v.end());
   std::mutex qm;
-  int slow_us = 0;
-  const int slow_w = debug_slow_sibling(&slow_us);
+  int slow_pct = 0;
+  const int slow_w = debug_slow_sibling(&slow_pct);
   std::vector<int> rcs(G, 0);
   std::vector<std::string> errs(G);
   std::vector<northup_stats> wst(G);
@@ -664,7 +664,7 @@ int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_bu
                                 op.src_ld * 4, op.cols * 4, op.rows, cudaMemcpyDefault, s);
           if (e != cudaSuccess) result = cuda_fail(e, "copy");
         } else {
-          if (w == slow_w && slow_us > 0) debug_spin(1000ll * slow_us, s);
+          if (w == slow_w && slow_pct > 0) debug_spin(debug_slow_ns(slow_pct, op.m, op.n, op.k), s);
           result = leaf_gemm_launch(reinterpret_cast<const float*>(base[op.a_buf] + op.a_off * 4), op.lda,
                                     reinterpret_cast<const float*>(base[op.b_buf] + op.b_off * 4), op.ldb,
                                     reinterpret_cast<float*>(base[op.c_buf] + op.c_off * 4), op.ldc, op.m, op.n,

@@ -58,7 +58,7 @@ int default_leaf_variant() {
   return env_variant;
 }
 
-// Test hook (NORTHUP_DEBUG_SLOW_SIBLING="w,us", exec.cpp): a one-thread kernel
+// Test hook (NORTHUP_DEBUG_SLOW_SIBLING="w,pct", exec.cpp): a one-thread kernel
 // that holds a stream for `ns` nanoseconds, emulating a slower sibling.
 __global__ void debug_spin_kernel(long long ns) {
   const long long t0 = clock64();

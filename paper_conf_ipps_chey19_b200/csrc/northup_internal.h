@@ -171,10 +171,15 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
 int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t iters,
                        const northup_hotspot_opts* o, const northup_hotspot_coeffs* k, Plan* out);
 
-// Test hooks: a kernel that holds a stream for `ns` ns; the sibling (and
-// microseconds) named by NORTHUP_DEBUG_SLOW_SIBLING="w,us" (-1 = none).
+// Test hooks: a kernel that holds a stream for `ns` ns; the sibling (and the
+// slowdown in percent) named by NORTHUP_DEBUG_SLOW_SIBLING="w,pct" (-1 = none).
+// The executors hold that sibling's compute stream for pct % of each leaf's
+// nominal time (2mnk at 300 TF/s) before launching it: a slower GPU.
 int debug_spin(long long ns, cudaStream_t s);
-int debug_slow_sibling(int* us);
+int debug_slow_sibling(int* pct);
+inline long long debug_slow_ns(int pct, int64_t m, int64_t n, int64_t k) {
+  return static_cast<long long>(pct / 100.0 * 2.0 * m * n * k / 3e14 * 1e9);
+}
 
 // --------------------------------------------------------------- executor
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,

@@ -814,7 +814,7 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
 // The paper's runtime keeps a task queue at each node and
 // balances work by popping local tasks and stealing remote ones (P:393-395,
 // there between CPU and GPU).  Here the tasks are C tiles of an M x N GEMM and
-// the queues belong to the HBM siblings: about four tiles per sibling, each an
+// the queues belong to the HBM siblings: two tiles per sibling, each an
 // S2 sub-problem with its C tile resident in one of two tile buffers (so the
 // next tile's panels stream while the previous one drains).
 int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N, int64_t K,
@@ -829,8 +829,12 @@ int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M
   auto bytes = [&](int64_t tm, int64_t tn) {
     return 4ull * (2ull * tm * pad_ld(tn) + uint64_t(kSlots) * (uint64_t(tm) * pad_ld(bk) + uint64_t(bk) * pad_ld(tn)));
   };
-  // start from a 2 x 2 split of each sibling's region, refine until it fits
-  int64_t Tr = std::min<int64_t>(M, 2 * Pr), Tc = std::min<int64_t>(N, 2 * Pc);
+  // two tiles per sibling: split each sibling's region in the direction that
+  // adds fewer PCIe bytes (every tile streams its A rows and B columns once:
+  // H2D = 4K (M Tc + N Tr)); refine further only until it fits
+  int64_t Tr = Pr, Tc = Pc;
+  if (M * Pc + N * 2 * Pr <= M * 2 * Pc + N * Pr) Tr = std::min<int64_t>(M, 2 * Pr);
+  else Tc = std::min<int64_t>(N, 2 * Pc);
   for (;;) {
     const int64_t tm = rup(cdiv(M, Tr), 8), tn = rup(cdiv(N, Tc), 8);
     if (!cap || bytes(tm, tn) <= cap) {

@@ -468,7 +468,7 @@ def test_set_local_errors():
     (512, 512, 640, 2, 0, 64), (600, 300, 200, 3, 0, 64), (1000, 700, 500, 4, 1_500_000, 128),
     (130, 90, 70, 1, 0, 32)])
 def test_queue_plan_replays_exactly(M, N, K, G, cap, kc):
-    """NU_SCHED_QUEUE: tiles of ~4 per sibling, each an S2 sub-problem with two
+    """NU_SCHED_QUEUE: two or more tiles per sibling, each an S2 sub-problem with two
     C-tile buffers; the plan API's no-steal unrolling replays exactly in any
     dependency-respecting order and moves the closed-form bytes."""
     A = nugen.fill(M, K, 8, 1, "int")
@@ -477,7 +477,7 @@ def test_queue_plan_replays_exactly(M, N, K, G, cap, kc):
     t, _ = nu.host_tree(G, cap)
     p = t.plan(M, N, K, nu.make_opts(schedule=nu.NU_SCHED_QUEUE, k_chunk=kc))
     s = p.stats()
-    assert s["schedule"] == nu.NU_SCHED_QUEUE and s["tasks"] >= min(4 * G, -(-M // 8) * -(-N // 8))
+    assert s["schedule"] == nu.NU_SCHED_QUEUE and s["tasks"] >= min(2 * G, -(-M // 8) * -(-N // 8))
     for seed in range(3):
         assert np.array_equal(simulate(p, A, B, M, N, K, rng=random.Random(seed)), ref)
     tr, tc = -(-M // s["bm"]), -(-N // s["bn"])

@@ -19,7 +19,7 @@ view = lambda b, r, c: np.ctypeslib.as_array((ctypes.c_float * (r * c)).from_add
 nugen.fill(M, K, 4, 1, out=view(A, M, K))
 nugen.fill(K, N, 4, 2, out=view(B, K, N))
 ref = None
-for slow in ("", "1,4000"):
+for slow in ("", "1,100"):     # sibling 1 takes twice as long per leaf
     os.environ["NORTHUP_DEBUG_SLOW_SIBLING"] = slow
     for name, sched in (("static_s2", nu.NU_SCHED_S2), ("queue", nu.NU_SCHED_QUEUE)):
         o = nu.make_opts(schedule=sched, shared_staging=-1)
