@@ -199,7 +199,9 @@ typedef struct {
                            over its PCIe link and pulls the rest from its grid-row / grid-column
                            peers' HBM (NVLink P2P; a local copy between virtual siblings).  C is
                            bitwise identical with and without it.  Disables `graph`. */
-  int reserved[4];
+  int queue_tiles;      /* NU_SCHED_QUEUE: C tiles per HBM sibling (0 = 2); more tiles balance
+                           better but stream more A/B bytes */
+  int reserved[3];
 } northup_gemm_opts;
 
 typedef struct {

@@ -50,7 +50,7 @@ class GemmOpts(ctypes.Structure):
                 ("k_chunk", ctypes.c_int64), ("npass", ctypes.c_int), ("resident", ctypes.c_int),
                 ("collect_timing", ctypes.c_int), ("a_panel_k", ctypes.c_int64),
                 ("graph", ctypes.c_int), ("shared_staging", ctypes.c_int),
-                ("reserved", ctypes.c_int * 4)]
+                ("queue_tiles", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
 
 
 class Stats(ctypes.Structure):
@@ -294,9 +294,11 @@ def partition_region(G: int, M: int, N: int, K: int, r: int) -> tuple[int, int, 
 
 def make_opts(schedule: int = NU_SCHED_AUTO, k_chunk: int = 0, npass: int = 0,
               collect_timing: bool = False, replicate_result: bool = False,
-              a_panel_k: int = 0, graph: bool = False, shared_staging: int = 0) -> GemmOpts:
+              a_panel_k: int = 0, graph: bool = False, shared_staging: int = 0,
+              queue_tiles: int = 0) -> GemmOpts:
     """northup_gemm_opts; shared_staging: 0 = auto (on for G > 1 uniform regions), -1 = off."""
     o = GemmOpts()
+    o.queue_tiles = queue_tiles
     o.shared_staging = shared_staging
     o.a_panel_k = a_panel_k
     o.graph = int(graph)

@@ -591,7 +591,7 @@ int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_bu
   const int64_t kc = (o && o->k_chunk > 0) ? o->k_chunk : kDefaultKChunk;
   const int npass = o ? o->npass : 0;
   QueueShape q;
-  int rc = choose_queue(t, hbm, M, N, K, kc, &q);
+  int rc = choose_queue(t, hbm, M, N, K, kc, o ? o->queue_tiles : 0, &q);
   if (rc) return rc;
   for (int w = 0; w < G; ++w) {
     rc = ensure_arena(t, hbm[w], q.arena_bytes);

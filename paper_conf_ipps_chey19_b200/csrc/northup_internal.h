@@ -139,7 +139,7 @@ struct QueueShape {
   uint64_t arena_bytes = 0;         // per sibling: 2 C-tile buffers + kSlots panel slots
 };
 int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N,
-                 int64_t K, int64_t kc, QueueShape* q);
+                 int64_t K, int64_t kc, int tiles, QueueShape* q);
 // Initial queues: tiles in row-major order, contiguous chunks per sibling.
 std::vector<std::vector<int64_t>> queue_initial(int G, const QueueShape& q);
 struct Builder;

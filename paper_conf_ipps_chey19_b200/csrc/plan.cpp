@@ -818,7 +818,7 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
 // S2 sub-problem with its C tile resident in one of two tile buffers (so the
 // next tile's panels stream while the previous one drains).
 int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N, int64_t K,
-                 int64_t kc, QueueShape* q) {
+                 int64_t kc, int tiles, QueueShape* q) {
   const int G = static_cast<int>(hbm.size());
   uint64_t cap = 0;
   for (int h : hbm)
@@ -829,12 +829,15 @@ int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M
   auto bytes = [&](int64_t tm, int64_t tn) {
     return 4ull * (2ull * tm * pad_ld(tn) + uint64_t(kSlots) * (uint64_t(tm) * pad_ld(bk) + uint64_t(bk) * pad_ld(tn)));
   };
-  // two tiles per sibling: split each sibling's region in the direction that
-  // adds fewer PCIe bytes (every tile streams its A rows and B columns once:
-  // H2D = 4K (M Tc + N Tr)); refine further only until it fits
+  // `tiles` (default 2) tiles per sibling: split each sibling's region, one
+  // factor of 2 at a time, in the direction that adds fewer PCIe bytes (every
+  // tile streams its A rows and B columns once: H2D = 4K (M Tc + N Tr));
+  // refine further only until it fits
   int64_t Tr = Pr, Tc = Pc;
-  if (M * Pc + N * 2 * Pr <= M * 2 * Pc + N * Pr) Tr = std::min<int64_t>(M, 2 * Pr);
-  else Tc = std::min<int64_t>(N, 2 * Pc);
+  for (int f = 1; f < std::max(tiles, 2); f *= 2) {
+    if (M * Tc + N * 2 * Tr <= M * 2 * Tc + N * Tr) Tr = std::min<int64_t>(M, 2 * Tr);
+    else Tc = std::min<int64_t>(N, 2 * Tc);
+  }
   for (;;) {
     const int64_t tm = rup(cdiv(M, Tr), 8), tn = rup(cdiv(N, Tc), 8);
     if (!cap || bytes(tm, tn) <= cap) {
@@ -992,7 +995,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     // time; only the tile-to-sibling assignment is dynamic).
     if (t->local_node >= 0) return fail(NU_ENOTSUP, "NU_SCHED_QUEUE runs in one process");
     QueueShape q;
-    rc = choose_queue(t, hbm, M, N, K, P.kc, &q);
+    rc = choose_queue(t, hbm, M, N, K, P.kc, o ? o->queue_tiles : 0, &q);
     if (rc) return rc;
     std::vector<int> arena(G);
     for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, q.arena_bytes);

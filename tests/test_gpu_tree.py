@@ -246,6 +246,7 @@ def test_queue_schedule_steals_from_a_slow_sibling(monkeypatch):
     Fig. 2) loses tiles to the fast one: steals happen and C is still exact."""
     monkeypatch.setenv("NORTHUP_DEBUG_SLOW_SIBLING", "1,300")   # sibling 1 is 4x slower
     M, N, K = 2048, 2048, 1024
-    C, a, b, st = run_host(M, N, K, G=2, kind="int", seed=2, k_chunk=512, schedule=nu.NU_SCHED_QUEUE)
+    C, a, b, st = run_host(M, N, K, G=2, kind="int", seed=2, k_chunk=512, schedule=nu.NU_SCHED_QUEUE,
+                           queue_tiles=8)
     assert st["tasks_stolen"] > 0
     check(C, a, b, "int")

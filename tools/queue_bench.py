@@ -9,7 +9,7 @@ import nugen
 import paper_conf_ipps_chey19_b200 as nu
 
 M = N = int(sys.argv[1]) if len(sys.argv) > 1 else 16384
-K = int(sys.argv[2]) if len(sys.argv) > 2 else 8192
+K = int(sys.argv[2]) if len(sys.argv) > 2 else 16384
 G = 2
 res = {"M": M, "N": N, "K": K, "G": G}
 t, _ = nu.host_tree(G, 8 << 30, devices=[0] * G)
@@ -19,10 +19,11 @@ view = lambda b, r, c: np.ctypeslib.as_array((ctypes.c_float * (r * c)).from_add
 nugen.fill(M, K, 4, 1, out=view(A, M, K))
 nugen.fill(K, N, 4, 2, out=view(B, K, N))
 ref = None
-for slow in ("", "1,100"):     # sibling 1 takes twice as long per leaf
+for slow in ("", "1,300"):     # sibling 1 takes 4x as long per leaf
     os.environ["NORTHUP_DEBUG_SLOW_SIBLING"] = slow
-    for name, sched in (("static_s2", nu.NU_SCHED_S2), ("queue", nu.NU_SCHED_QUEUE)):
-        o = nu.make_opts(schedule=sched, shared_staging=-1)
+    for name, sched, tiles in (("static_s2", nu.NU_SCHED_S2, 0), ("queue2", nu.NU_SCHED_QUEUE, 2),
+                               ("queue8", nu.NU_SCHED_QUEUE, 8)):
+        o = nu.make_opts(schedule=sched, shared_staging=-1, queue_tiles=tiles)
         t.gemm(A, B, C, M, N, K, o)
         ts = []
         for _ in range(2):
