@@ -49,7 +49,7 @@ CONFIGS = {
 HOTSPOT = dict(R=32768, C=32768, iters=256, cap=8 * GiB,
                desc="HotSpot-2D 32768^2 fp32 grid (P:349 32k inputs) x 256 iterations, pinned host -> "
                     "HBM (8 GiB cap) -> SMEM, 1 GPU (S§8(f) NEXT-3)")
-HS_FLOPS_PER_UPDATE = 14                 # fp32 ops of one cell update, no contraction (hotspot.cu)
+HS_FLOPS_PER_UPDATE = 14                 # flops of one cell update as the formula states (5 mul + 9 add/sub)
 FP32_LANES_PER_SM, N_SMS = 128, 148      # B200: 4 SMSPs x 32 fp32 lanes; 148 SMs
 NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25      # B200_PROFILING.md nominal dense ratio
 LEAF_KERNELS = {1: "nu::leaf::sm1::leaf_gemm_1sm_kernel", 2: "nu::leaf::sm2::leaf_gemm_2sm_kernel",
@@ -475,7 +475,7 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     achieved = flops_per_launch / (leaf_ms * 1e-3) / 1e12
     ck = clk.summary()
     f_max = (ck.get("sm_max_mhz") or 1965.0) * 1e6
-    peak = N_SMS * FP32_LANES_PER_SM * f_max / 1e12
+    peak = 2 * N_SMS * FP32_LANES_PER_SM * f_max / 1e12     # fp32 FMA = 2 flops per lane per clock
     # parity: sampled blocks against the fp64 oracle (window of border `iters`)
     k64 = ohs.coeffs(R, C)
     rng = np.random.default_rng(11)
@@ -501,7 +501,7 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
         "metric": "out-of-core HotSpot-2D cell updates/s (S§8(f) NEXT-3); % slowdown vs in-HBM; roofline frac",
         "value": round(value, 3), "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_h, 3), "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f32 (no contraction)",
+        "vs_baseline": None, "dtype": "f32 (fixed FADD/FFMA sequence, RH4)",
         "data": "synthetic (counter-hash temperature 330 +- 10 K, power [0, 0.5))",
         "config": {"workload": "hotspot: " + HOTSPOT["desc"] + (" [quick: /4 sizes]" if args.quick else ""),
                    "rows": R, "cols": C, "iters": iters, "hbm_cap_bytes": cap,
@@ -517,11 +517,12 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
         "paper_context": {"hotspot_ooc_gap_pct": 15, "note": "APU + SSD vs DRAM (PAPER.md P:381); context only"},
         "roofline": {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "TFLOP/s",
                      "frac": round(achieved / peak, 4), "traffic": None,
-                     "peak_basis": f"{N_SMS} SMs x {FP32_LANES_PER_SM} fp32 lanes x clocks.max.sm "
-                                   f"{f_max / 1e6:.0f} MHz (one fp32 op per lane per clock)",
+                     "peak_basis": f"dense fp32 peak: {N_SMS} SMs x {FP32_LANES_PER_SM} lanes x 2 flops (FMA) x "
+                                   f"clocks.max.sm {f_max / 1e6:.0f} MHz",
                      "kernel": "nu::hs::hotspot_kernel_v3", "launch": [R, C, li],
                      "flops_per_launch": flops_per_launch,
-                     "flops_basis": f"{HS_FLOPS_PER_UPDATE} fp32 ops per useful cell update x R x C x "
+                     "flops_basis": f"{HS_FLOPS_PER_UPDATE} flops per useful cell update (the update's "
+                                    f"5 multiplies + 9 adds; the kernel issues 3 FADD + 6 FFMA) x R x C x "
                                     f"iterations per launch (halo recomputation not counted)",
                      "ms_per_launch": round(leaf_ms, 3), "launches_per_step": launches},
         "gpu_launches": int(launches * args.steps + st_o.get("leaf_launches", 0) * args.steps),

@@ -9,12 +9,15 @@
 // shrinks by one cell per iteration on every side that is not a grid edge),
 // so HBM is read once and written once per `iters` iterations.
 //
-// Arithmetic contract: every cell update is
-//     t + cap_1 * (((p + ((s + n) - 2t) * ry_1) + ((e + w) - 2t) * rx_1) + (amb - t) * rz_1)
-// evaluated left to right in fp32 with round-to-nearest and no FMA
-// contraction (__fadd_rn/__fmul_rn), so the result of a cell is independent
-// of tiling, iterations per launch and launch order: in-HBM and out-of-core
-// runs agree bit for bit, and so does an fp32 numpy emulation of the update.
+// Arithmetic contract (RH4): every cell update is the fixed fp32
+// sequence (round-to-nearest, fma = one rounding)
+//     a = fma(-2, t, s + n);  b = fma(-2, t, e + w)
+//     d = fma(a, ry_1, p);  d = fma(b, rx_1, d);  d = fma(amb - t, rz_1, d)
+//     t' = fma(cap_1, d, t)
+// written with __fadd_rn/__fmaf_rn so the compiler cannot reassociate or
+// re-fuse it: 3 FADD + 6 FFMA per update.  The result of a cell is therefore
+// independent of tiling, iterations per launch and launch order: in-HBM and
+// out-of-core runs agree bit for bit, and so does an exact fp32 emulation.
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -43,12 +46,12 @@ struct Args {
 
 __device__ __forceinline__ float update(float t, float p, float n, float s, float e, float w,
                                         const Args& a) {
-  const float two_t = __fmul_rn(2.0f, t);
-  const float ly = __fmul_rn(__fsub_rn(__fadd_rn(s, n), two_t), a.ry_1);
-  const float lx = __fmul_rn(__fsub_rn(__fadd_rn(e, w), two_t), a.rx_1);
-  const float lz = __fmul_rn(__fsub_rn(a.amb, t), a.rz_1);
-  const float d = __fadd_rn(__fadd_rn(__fadd_rn(p, ly), lx), lz);
-  return __fadd_rn(t, __fmul_rn(a.cap_1, d));
+  const float ay = __fmaf_rn(-2.0f, t, __fadd_rn(s, n));
+  const float ax = __fmaf_rn(-2.0f, t, __fadd_rn(e, w));
+  float d = __fmaf_rn(ay, a.ry_1, p);
+  d = __fmaf_rn(ax, a.rx_1, d);
+  d = __fmaf_rn(__fsub_rn(a.amb, t), a.rz_1, d);
+  return __fmaf_rn(a.cap_1, d, t);
 }
 
 // 4-byte asynchronous global -> shared copies (LDGSTS): every element of the

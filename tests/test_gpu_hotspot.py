@@ -13,6 +13,7 @@ import torch
 import nugen
 import paper_conf_ipps_chey19_b200 as nu
 from oracle import hotspot as hs
+from fp32emu import emulate_fp32
 
 pytestmark = pytest.mark.gpu
 K = hs.coeffs(1024, 1024)
@@ -20,23 +21,6 @@ K = hs.coeffs(1024, 1024)
 
 def grids(R, C, seed):
     return (nugen.fill(R, C, seed, nugen.MAT_T, "temp"), nugen.fill(R, C, seed, nugen.MAT_P, "power"))
-
-
-def emulate_fp32(T, P, iters):
-    """The update in fp32, evaluated in the kernel's order (test-side check,
-    independent of the CUDA code): t + cap*(((p + ((s+n) - 2t)*ry) + ((e+w) - 2t)*rx) + (amb - t)*rz)."""
-    k = nu.hotspot_coeffs(*T.shape)
-    f = np.float32
-    cap, rx, ry, rz, amb = f(k.cap_1), f(k.rx_1), f(k.ry_1), f(k.rz_1), f(k.amb)
-    t = T.astype(np.float32).copy()
-    p = P.astype(np.float32)
-    for _ in range(iters):
-        g = np.pad(t, 1, mode="edge")
-        n, s, e, w = g[:-2, 1:-1], g[2:, 1:-1], g[1:-1, 2:], g[1:-1, :-2]
-        two_t = f(2) * t
-        d = ((p + ((s + n) - two_t) * ry) + ((e + w) - two_t) * rx) + (amb - t) * rz
-        t = (t + cap * d).astype(np.float32)
-    return t
 
 
 def check(out, T, P, iters):

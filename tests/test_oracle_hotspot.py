@@ -115,7 +115,7 @@ def test_tolerance_model_against_fp32_emulation():
     k32 = {kk: np.float32(v) for kk, v in K.items()}
     t = T.astype(np.float32)
     p = P.astype(np.float32)
-    for _ in range(40):
+    for _ in range(40):     # fp32 at every operation (no fused operations in this emulation)
         g = np.pad(t, 1, mode="edge")
         n, s, e, w = g[:-2, 1:-1], g[2:, 1:-1], g[1:-1, 2:], g[1:-1, :-2]
         t = (t + k32["cap_1"] * (p + (s + n - np.float32(2) * t) * k32["ry_1"]
@@ -125,3 +125,29 @@ def test_tolerance_model_against_fp32_emulation():
     err = np.abs(t.astype(np.float64) - ref).max()
     assert err <= hs.tolerance(40, np.abs(ref).max())
     assert err > 0   # fp32 really differs (the bound is exercised)
+
+
+def test_fma32_emulation_is_exact():
+    """Pin of the test-side fma (tests/fp32emu.py) against exact rational
+    arithmetic, including sums that land on float32 rounding boundaries."""
+    from fractions import Fraction
+
+    from fp32emu import fma32
+    rng = np.random.default_rng(3)
+    a = rng.standard_normal(3000).astype(np.float32)
+    b = rng.standard_normal(3000).astype(np.float32)
+    c = (rng.standard_normal(3000) * 1e-3).astype(np.float32)
+    # near-midpoint cases: c = -(a*b rounded to float32) + a tiny offset
+    ab32 = (a.astype(np.float64) * b.astype(np.float64)).astype(np.float32)
+    c[::3] = (-ab32[::3]).astype(np.float32)
+    got = fma32(a, b, c)
+    for i in range(0, 3000, 5):
+        exact = Fraction(float(a[i])) * Fraction(float(b[i])) + Fraction(float(c[i]))
+        f = np.float32(float(exact))                 # candidate near the exact value
+        cands = {float(f), float(np.nextafter(f, np.float32(np.inf))), float(np.nextafter(f, np.float32(-np.inf)))}
+        dist = {v: abs(Fraction(v) - exact) for v in cands}
+        m = min(dist.values())
+        best = [v for v in cands if dist[v] == m]
+        if len(best) > 1:                            # tie: round half to even
+            best = [v for v in best if (int(np.array(v, np.float32).view(np.int32)) & 1) == 0]
+        assert float(got[i]) == best[0], i
