@@ -226,6 +226,8 @@ typedef struct {
   double t_p2p_ms;       /* sum over GPUs of busy time of sibling pulls (timing mode) */
   int64_t tasks;         /* NU_SCHED_QUEUE: C tiles */
   int64_t tasks_stolen;  /* NU_SCHED_QUEUE: tiles a sibling took from another sibling's queue */
+  int file_direct_mode;  /* FILE root with HBM children (GDS edge): 1 = cuFile, 2 = pinned bounce */
+  int reserved_stat;
 } northup_stats;
 
 /* C = A.B (no alpha/beta; C overwritten — reading R3), A (M x K), B (K x N),

@@ -66,7 +66,8 @@ class Stats(ctypes.Structure):
                 ("hbm_peak_bytes", ctypes.c_uint64), ("graph_replayed", ctypes.c_int),
                 ("shared_staging", ctypes.c_int), ("bytes_p2p", ctypes.c_uint64),
                 ("t_p2p_ms", ctypes.c_double), ("tasks", ctypes.c_int64),
-                ("tasks_stolen", ctypes.c_int64)]
+                ("tasks_stolen", ctypes.c_int64), ("file_direct_mode", ctypes.c_int),
+                ("reserved_stat", ctypes.c_int)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -25,7 +25,10 @@
 #include <mutex>
 #include <thread>
 
+#include <dlfcn.h>
+
 #include <deque>
+#include <map>
 
 #include "northup_internal.h"
 #include "plan_builder.h"
@@ -158,6 +161,7 @@ struct RunCtx {
   std::vector<char> io_done;           // I/O op: finished
   std::atomic<bool> abort{false};
   double io_ms = 0;
+  int io_mode = 0;                     // file <-> HBM: 1 = cuFile, 2 = pinned bounce
 };
 
 static void mark(RunCtx& c, std::vector<char>& v, size_t i) {
@@ -385,9 +389,138 @@ static int file_block(const northup_buf_s* f, bool write, char* mem, int64_t mem
   return 0;
 }
 
+// ---- FILE <-> HBM directly (the GDS edge, NEXT-4) -------------------------
+// cuFile (GPUDirect Storage) is loaded with dlopen so the library does not
+// depend on it.  Where the file system has no GDS support cuFile runs in its
+// compat mode (/etc/cufile.json allow_compat_mode); if the driver cannot be
+// opened at all, transfers bounce through a pinned host buffer.
+namespace {
+struct CuFileApi {
+  bool tried = false, ok = false;
+  struct Err {
+    int err;
+    int cu_err;
+  };
+  Err (*driver_open)() = nullptr;
+  Err (*handle_register)(void**, void*) = nullptr;
+  void (*handle_deregister)(void*) = nullptr;
+  ssize_t (*read)(void*, void*, size_t, off_t, off_t) = nullptr;
+  ssize_t (*write)(void*, const void*, size_t, off_t, off_t) = nullptr;
+};
+CuFileApi g_cufile;
+std::mutex g_cufile_m;
+
+CuFileApi& cufile() {
+  std::lock_guard<std::mutex> g(g_cufile_m);
+  if (g_cufile.tried) return g_cufile;
+  g_cufile.tried = true;
+  void* h = dlopen("libcufile.so.0", RTLD_NOW | RTLD_LOCAL);
+  if (!h) h = dlopen("libcufile.so", RTLD_NOW | RTLD_LOCAL);
+  if (!h) return g_cufile;
+  g_cufile.driver_open = reinterpret_cast<CuFileApi::Err (*)()>(dlsym(h, "cuFileDriverOpen"));
+  g_cufile.handle_register = reinterpret_cast<CuFileApi::Err (*)(void**, void*)>(dlsym(h, "cuFileHandleRegister"));
+  g_cufile.handle_deregister = reinterpret_cast<void (*)(void*)>(dlsym(h, "cuFileHandleDeregister"));
+  g_cufile.read = reinterpret_cast<ssize_t (*)(void*, void*, size_t, off_t, off_t)>(dlsym(h, "cuFileRead"));
+  g_cufile.write = reinterpret_cast<ssize_t (*)(void*, const void*, size_t, off_t, off_t)>(dlsym(h, "cuFileWrite"));
+  if (!g_cufile.driver_open || !g_cufile.handle_register || !g_cufile.read || !g_cufile.write) return g_cufile;
+  g_cufile.ok = g_cufile.driver_open().err == 0;
+  return g_cufile;
+}
+
+// CUfileDescr_t as in cufile.h: type, union {int fd; void* handle;}, fs_ops.
+struct CuFileDescr {
+  int type;
+  union {
+    int fd;
+    void* handle;
+  } h;
+  const void* fs_ops;
+};
+}  // namespace
+
+struct DevIO {
+  std::map<const northup_buf_s*, void*> handles;   // cuFile handle per file
+  char* bounce = nullptr;                          // pinned fallback buffer
+  size_t bounce_bytes = 0;
+  int mode = 0;                                    // 1 = cuFile, 2 = bounce
+  ~DevIO() {
+    for (auto& kv : handles)
+      if (kv.second && g_cufile.handle_deregister) g_cufile.handle_deregister(kv.second);
+    if (bounce) cudaFreeHost(bounce);
+  }
+};
+
+// A rows x cols fp32 block between a file and DEVICE memory.
+static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* dmem, int64_t mem_ld,
+                          int64_t file_off, int64_t file_ld, int64_t rows, int64_t cols) {
+  CuFileApi& api = cufile();
+  void* fh = nullptr;
+  if (api.ok && !getenv("NORTHUP_NO_CUFILE")) {   // NORTHUP_NO_CUFILE: force the bounce (tests)
+    auto it = io.handles.find(f);
+    if (it == io.handles.end()) {
+      CuFileDescr d{};
+      d.type = 1;   // CU_FILE_HANDLE_TYPE_OPAQUE_FD
+      d.h.fd = f->direct_fd >= 0 ? f->direct_fd : f->fd;
+      void* h = nullptr;
+      if (api.handle_register(&h, &d).err != 0) h = nullptr;
+      it = io.handles.emplace(f, h).first;
+    }
+    fh = it->second;
+  }
+  auto xfer = [&](char* p, uint64_t bytes, uint64_t off) -> int {
+    if (fh) {
+      io.mode = 1;
+      while (bytes) {
+        const ssize_t r = write ? api.write(fh, p, bytes, static_cast<off_t>(off), 0)
+                                : api.read(fh, p, bytes, static_cast<off_t>(off), 0);
+        if (r <= 0) return fail(NU_EIO, "cuFile%s(%s) returned %zd", write ? "Write" : "Read", f->path.c_str(), r);
+        p += r;
+        bytes -= static_cast<uint64_t>(r);
+        off += static_cast<uint64_t>(r);
+      }
+      return 0;
+    }
+    io.mode = 2;
+    if (!io.bounce) {
+      io.bounce_bytes = 64ull << 20;
+      cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&io.bounce), io.bounce_bytes, cudaHostAllocPortable);
+      if (e != cudaSuccess) return cuda_fail(e, "bounce buffer");
+    }
+    while (bytes) {
+      const uint64_t n = std::min<uint64_t>(bytes, io.bounce_bytes);
+      if (write) {
+        cudaError_t e = cudaMemcpy(io.bounce, p, n, cudaMemcpyDefault);
+        if (e != cudaSuccess) return cuda_fail(e, "bounce D2H");
+        int rc = file_block(f, true, io.bounce, static_cast<int64_t>(n / 4), static_cast<int64_t>(off / 4),
+                            static_cast<int64_t>(n / 4), 1, static_cast<int64_t>(n / 4));
+        if (rc) return rc;
+      } else {
+        int rc = file_block(f, false, io.bounce, static_cast<int64_t>(n / 4), static_cast<int64_t>(off / 4),
+                            static_cast<int64_t>(n / 4), 1, static_cast<int64_t>(n / 4));
+        if (rc) return rc;
+        cudaError_t e = cudaMemcpy(p, io.bounce, n, cudaMemcpyDefault);
+        if (e != cudaSuccess) return cuda_fail(e, "bounce H2D");
+      }
+      p += n;
+      bytes -= n;
+      off += n;
+    }
+    return 0;
+  };
+  if (mem_ld == cols && file_ld == cols)
+    return xfer(dmem, static_cast<uint64_t>(rows * cols) * 4, static_cast<uint64_t>(file_off) * 4);
+  for (int64_t r = 0; r < rows; ++r) {
+    int rc = xfer(dmem + r * mem_ld * 4, static_cast<uint64_t>(cols) * 4,
+                  static_cast<uint64_t>(file_off + r * file_ld) * 4);
+    if (rc) return rc;
+  }
+  return 0;
+}
+
 static int run_io(RunCtx& c) {
   const Plan& P = *c.plan;
   const auto t0 = std::chrono::steady_clock::now();
+  DevIO dio;
   for (size_t i = 0; i < P.ops.size(); ++i) {
     const northup_op& op = P.ops[i];
     if (op.stream != S_IO) continue;
@@ -401,12 +534,20 @@ static int run_io(RunCtx& c) {
       if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize (I/O thread)");
     }
     int rc;
+    // memory side in HBM (FILE -> HBM edge) or in host DRAM (staging)
+    const int mb = op.op == NU_OP_IO_READ ? op.dst_buf : op.src_buf;
+    const bool dev = P.bufs[mb].kind == B_ARENA && c.t->nodes[P.bufs[mb].node].storage == NU_HBM;
+    if (dev) cudaSetDevice(c.t->nodes[P.bufs[mb].node].phys);
     if (op.op == NU_OP_IO_READ)
-      rc = file_block(c.file[op.src_buf], false, c.base[op.dst_buf] + op.dst_off * 4, op.dst_ld,
-                      op.src_off, op.src_ld, op.rows, op.cols);
+      rc = dev ? file_block_dev(dio, c.file[op.src_buf], false, c.base[op.dst_buf] + op.dst_off * 4, op.dst_ld,
+                                op.src_off, op.src_ld, op.rows, op.cols)
+               : file_block(c.file[op.src_buf], false, c.base[op.dst_buf] + op.dst_off * 4, op.dst_ld,
+                            op.src_off, op.src_ld, op.rows, op.cols);
     else
-      rc = file_block(c.file[op.dst_buf], true, c.base[op.src_buf] + op.src_off * 4, op.src_ld,
-                      op.dst_off, op.dst_ld, op.rows, op.cols);
+      rc = dev ? file_block_dev(dio, c.file[op.dst_buf], true, c.base[op.src_buf] + op.src_off * 4, op.src_ld,
+                                op.dst_off, op.dst_ld, op.rows, op.cols)
+               : file_block(c.file[op.dst_buf], true, c.base[op.src_buf] + op.src_off * 4, op.src_ld,
+                            op.dst_off, op.dst_ld, op.rows, op.cols);
     if (rc) return rc;
     mark(c, c.io_done, i);
   }
@@ -415,6 +556,7 @@ static int run_io(RunCtx& c) {
     if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0)
       return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(errno));
   c.io_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  c.io_mode = dio.mode;
   return 0;
 }
 
@@ -568,6 +710,7 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
       st->t_p2p_ms += busy[wi][S_D2D];
     }
     st->t_io_ms = ctx.io_ms;
+    st->file_direct_mode = ctx.io_mode;
   }
   return 0;
 }

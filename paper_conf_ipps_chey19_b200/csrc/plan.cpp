@@ -808,6 +808,99 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
   return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
 }
 
+// FILE root -> HBM siblings directly (S§8(f) NEXT-4: the GDS edge, P:240's
+// mmap alternative / GPUfs P:45): no DRAM staging level.  Each sibling keeps
+// its C block resident in HBM and reads the K panels of A (K-panel-major file,
+// R15) and B (row-major) from the files straight into its HBM panel slots;
+// finished C blocks are written from HBM to the C file.  The I/O thread does
+// the transfers with cuFile (GPUDirect Storage; compat mode where the file
+// system has no GDS support) and falls back to a pinned bounce buffer when
+// cuFile cannot be opened.  Slots have unpadded rows where the file's rows are
+// contiguous, so one panel is one read.
+int build_file_direct(Builder& B, const northup_tree_s* t, const std::vector<int>& hbm, int64_t M,
+                      int64_t N, int64_t K, int A, int Bb, int C, int64_t kc, int64_t a_panel_k,
+                      northup_stats* st) {
+  const int G = static_cast<int>(hbm.size());
+  const int io = G;   // the I/O pseudo-worker
+  const int64_t bk = a_panel_k > 0 ? a_panel_k : kc;
+  std::vector<int64_t> r0(G), r1(G), c0(G), c1(G);
+  int64_t mmax = 0, nmax = 0;
+  uint64_t cap = uint64_t(1) << 62;
+  for (int w = 0; w < G; ++w) {
+    int rc = region_of(G, M, N, w, &r0[w], &r1[w], &c0[w], &c1[w]);
+    if (rc) return rc;
+    mmax = std::max(mmax, r1[w] - r0[w]);
+    nmax = std::max(nmax, c1[w] - c0[w]);
+    if (t->nodes[hbm[w]].capacity) cap = std::min<uint64_t>(cap, t->nodes[hbm[w]].capacity);
+  }
+  // A slot rows: bk when the panel width keeps 16-B rows (TMA), else padded
+  const bool bk4 = bk % 4 == 0 && K % 4 == 0;
+  auto lda_of = [&](int64_t kk) { return bk4 ? kk : pad_ld(kk); };
+  auto hbm_bytes = [&](int64_t bm, int64_t bn) {
+    const int64_t ldb = (bn == N && N % 4 == 0) ? bn : pad_ld(bn);
+    return 4ull * (uint64_t(bm) * pad_ld(bn) + uint64_t(kSlots) * (uint64_t(bm) * lda_of(bk) + uint64_t(bk) * ldb));
+  };
+  int64_t bm = mmax, bn = nmax;
+  while (hbm_bytes(bm, bn) > cap) {
+    if (bm > 128) bm = rup(cdiv(bm, 2), 128);
+    else if (bn > 256) bn = rup(cdiv(bn, 2), 256);
+    else return fail(NU_ENOMEM, "HBM capacity %llu B below the minimum block", (unsigned long long)cap);
+  }
+  const int64_t ldC = pad_ld(bn), ldBs = (bn == N && N % 4 == 0) ? bn : pad_ld(bn);
+  std::vector<int> arena(G);
+  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+  st->bm = bm;
+  st->bn = bn;
+  st->bk = bk;
+  st->hbm_peak_bytes = hbm_bytes(bm, bn);
+  st->schedule = NU_SCHED_S2;
+  const int64_t npan = cdiv(K, bk);
+  std::vector<int64_t> slot(G, 0);
+  const int64_t nbr = cdiv(mmax, bm), nbc = cdiv(nmax, bn);
+  for (int64_t bi = 0; bi < nbr; ++bi)
+    for (int64_t bj = 0; bj < nbc; ++bj) {
+      for (int64_t p = 0; p < npan; ++p) {
+        const int64_t k0 = p * bk, kk = std::min(bk, K - k0);
+        const int64_t ldA = lda_of(kk);
+        for (int w = 0; w < G; ++w) {
+          const int64_t i0 = bi * bm, j0 = bj * bn;
+          const int64_t m = std::min(bm, (r1[w] - r0[w]) - i0), n = std::min(bn, (c1[w] - c0[w]) - j0);
+          if (m <= 0 || n <= 0) continue;
+          const int64_t gr = r0[w] + i0, gc = c0[w] + j0;
+          const int sl = static_cast<int>(slot[w]++ % kSlots);
+          const int64_t offSA = bm * ldC + sl * (bm * lda_of(bk) + bk * ldBs);
+          const int64_t offSB = offSA + bm * lda_of(bk);
+          // file -> HBM: A rows of this block in panel p, B rows of panel p
+          if (a_panel_k > 0)
+            B.emit(make_io(io, NU_OP_IO_READ, A, k0 * M + gr * kk, kk, arena[w], offSA, ldA, m, kk),
+                   {{A, k0 * M + gr * kk, kk, m, kk, false}, {arena[w], offSA, ldA, m, kk, true}});
+          else
+            B.emit(make_io(io, NU_OP_IO_READ, A, gr * K + k0, K, arena[w], offSA, ldA, m, kk),
+                   {{A, gr * K + k0, K, m, kk, false}, {arena[w], offSA, ldA, m, kk, true}});
+          B.emit(make_io(io, NU_OP_IO_READ, Bb, k0 * N + gc, N, arena[w], offSB, ldBs, kk, n),
+                 {{Bb, k0 * N + gc, N, kk, n, false}, {arena[w], offSB, ldBs, kk, n, true}});
+          st->bytes_file_read += 4ull * (uint64_t(m) * kk + uint64_t(kk) * n);
+          B.emit(make_leaf(w, arena[w], offSA, ldA, arena[w], offSB, ldBs, arena[w], 0, ldC, m, n, kk,
+                           p > 0 ? 1 : 0),
+                 {{arena[w], offSA, ldA, m, kk, false}, {arena[w], offSB, ldBs, kk, n, false},
+                  {arena[w], 0, ldC, m, n, true}});
+          st->leaf_launches++;
+        }
+      }
+      // HBM -> file: the C block (Listing 4 file_write from the HBM level)
+      for (int w = 0; w < G; ++w) {
+        const int64_t i0 = bi * bm, j0 = bj * bn;
+        const int64_t m = std::min(bm, (r1[w] - r0[w]) - i0), n = std::min(bn, (c1[w] - c0[w]) - j0);
+        if (m <= 0 || n <= 0) continue;
+        const int64_t gr = r0[w] + i0, gc = c0[w] + j0;
+        B.emit(make_io(io, NU_OP_IO_WRITE, arena[w], 0, ldC, C, gr * N + gc, N, m, n),
+               {{arena[w], 0, ldC, m, n, false}, {C, gr * N + gc, N, m, n, true}});
+        st->bytes_file_write += 4ull * m * n;
+      }
+    }
+  return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
+}
+
 }  // namespace
 
 // ------------------------------------------------- NU_SCHED_QUEUE (NEXT-2)
@@ -951,9 +1044,25 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     return rc;
   }
   if (root.storage == NU_FILE) {
+    bool direct = !root.children.empty();
+    for (int c : root.children) direct = direct && t->nodes[c].storage == NU_HBM;
+    if (direct) {
+      // FILE -> HBM siblings (the GDS edge, NEXT-4)
+      std::vector<int> hbm(root.children.begin(), root.children.end());
+      P.num_workers = static_cast<int>(hbm.size());
+      P.worker_node = hbm;
+      st.num_gpus = P.num_workers;
+      P.file_root = true;
+      if (M == 0 || N == 0 || K == 0) return 0;
+      rc = build_file_direct(B, t, hbm, M, N, K, A, Bb, C, P.kc, o ? o->a_panel_k : 0, &st);
+      st.ops = static_cast<int64_t>(P.ops.size());
+      for (const northup_op& op : P.ops)
+        if (op.op == NU_OP_IO_READ || op.op == NU_OP_IO_WRITE) st.copies++;
+      return rc;
+    }
     // FILE -> HOST (DRAM staging) -> HBM siblings
     if (root.children.size() != 1 || t->nodes[root.children[0]].storage != NU_HOST)
-      return fail(NU_ENOTSUP, "a FILE root needs exactly one HOST staging child (no GDS edge)");
+      return fail(NU_ENOTSUP, "a FILE root needs HBM children (GDS edge) or one HOST staging child");
     const int staging = root.children[0];
     std::vector<int> hbm;
     for (int c : t->nodes[staging].children) {

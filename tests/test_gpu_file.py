@@ -72,3 +72,49 @@ def test_file_alloc_and_move(tmp_path):
     assert len(list(tmp_path.iterdir())) == 1
     t.destroy()
     assert len(list(tmp_path.iterdir())) == 0
+
+
+def direct_tree(G, cap=0):
+    """FILE -> HBM siblings directly (the GDS edge, NEXT-4): no DRAM staging node."""
+    t = nu.Tree()
+    root = t.add_node(-1, nu.NU_FILE)
+    for g in range(G):
+        h = t.add_node(root, nu.NU_HBM, 0, cap)
+        t.add_node(h, nu.NU_SMEM, 0, 227 * 1024, nu.NU_PROC_SM100)
+    return t
+
+
+@pytest.mark.parametrize("M,N,K,G,cap,panel,kind,bounce", [
+    (512, 768, 1024, 1, 0, 256, "uniform", False),
+    (640, 900, 1500, 2, 0, 512, "int", False),
+    (1000, 1200, 3000, 1, 8_000_000, 1024, "int", False),   # capacity -> several C blocks
+    (300, 200, 130, 2, 0, 0, "int", False),                  # row-major A: per-row reads
+    (640, 900, 1500, 2, 0, 512, "int", True),                # forced pinned-bounce path
+])
+def test_file_direct_to_hbm(tmp_path, monkeypatch, M, N, K, G, cap, panel, kind, bounce):
+    if bounce:
+        monkeypatch.setenv("NORTHUP_NO_CUFILE", "1")
+    A = nugen.fill(M, K, 7, 1, kind)
+    B = nugen.fill(K, N, 7, 2, kind)
+    a_path, b_path, c_path = tmp_path / "A.bin", tmp_path / "B.bin", tmp_path / "C.bin"
+    A.tofile(a_path)
+    B.tofile(b_path)
+    if panel:
+        nu.file_tile_kpanels(str(a_path), str(tmp_path / "A_t.bin"), M, K, panel)
+        a_path = tmp_path / "A_t.bin"
+    t = direct_tree(G, cap)
+    t.finalize()
+    fa = t.open_file(0, str(a_path), 4 * M * K)
+    fb = t.open_file(0, str(b_path), 4 * K * N)
+    fc = t.open_file(0, str(c_path), 4 * M * N)
+    st = t.gemm(fa, fb, fc, M, N, K, nu.make_opts(a_panel_k=panel))
+    t.destroy()
+    assert st["file_direct_mode"] == (2 if bounce else st["file_direct_mode"]) and st["file_direct_mode"] in (1, 2)
+    C = np.fromfile(c_path, dtype=np.float32).reshape(M, N)
+    ref = oracle.gemm(A, B)
+    if kind == "int":
+        assert np.array_equal(C.astype(np.float64), ref)
+    else:
+        e, _ = oracle.normwise_err(C, ref, oracle.row_norms(A), oracle.col_norms(B))
+        assert e <= 1e-5, e
+    assert st["bytes_file_write"] == 4 * M * N
