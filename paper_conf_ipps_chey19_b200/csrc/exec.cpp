@@ -26,6 +26,7 @@
 #include <thread>
 
 #include <dlfcn.h>
+#include <cstdio>
 
 #include <deque>
 #include <map>
@@ -414,6 +415,12 @@ CuFileApi& cufile() {
   std::lock_guard<std::mutex> g(g_cufile_m);
   if (g_cufile.tried) return g_cufile;
   g_cufile.tried = true;
+  // opt-in: cuFile's compat mode hung on this pool's boxes (virtio disk, no
+  // nvidia-fs), so the pinned bounce is the default and NORTHUP_CUFILE=1 asks
+  // for GPUDirect Storage
+  const char* want = getenv("NORTHUP_CUFILE");
+  if (!want || want[0] != '1') return g_cufile;
+  const bool dbg = getenv("NORTHUP_CUFILE_DEBUG") != nullptr;
   void* h = dlopen("libcufile.so.0", RTLD_NOW | RTLD_LOCAL);
   if (!h) h = dlopen("libcufile.so", RTLD_NOW | RTLD_LOCAL);
   if (!h) return g_cufile;
@@ -423,7 +430,9 @@ CuFileApi& cufile() {
   g_cufile.read = reinterpret_cast<ssize_t (*)(void*, void*, size_t, off_t, off_t)>(dlsym(h, "cuFileRead"));
   g_cufile.write = reinterpret_cast<ssize_t (*)(void*, const void*, size_t, off_t, off_t)>(dlsym(h, "cuFileWrite"));
   if (!g_cufile.driver_open || !g_cufile.handle_register || !g_cufile.read || !g_cufile.write) return g_cufile;
+  if (dbg) fprintf(stderr, "[northup] cuFileDriverOpen ...\n");
   g_cufile.ok = g_cufile.driver_open().err == 0;
+  if (dbg) fprintf(stderr, "[northup] cuFileDriverOpen -> %s\n", g_cufile.ok ? "ok" : "failed");
   return g_cufile;
 }
 
@@ -455,14 +464,16 @@ static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* d
                           int64_t file_off, int64_t file_ld, int64_t rows, int64_t cols) {
   CuFileApi& api = cufile();
   void* fh = nullptr;
-  if (api.ok && !getenv("NORTHUP_NO_CUFILE")) {   // NORTHUP_NO_CUFILE: force the bounce (tests)
+  if (api.ok) {
     auto it = io.handles.find(f);
     if (it == io.handles.end()) {
       CuFileDescr d{};
       d.type = 1;   // CU_FILE_HANDLE_TYPE_OPAQUE_FD
       d.h.fd = f->direct_fd >= 0 ? f->direct_fd : f->fd;
       void* h = nullptr;
+      if (getenv("NORTHUP_CUFILE_DEBUG")) fprintf(stderr, "[northup] cuFileHandleRegister(fd %d) ...\n", d.h.fd);
       if (api.handle_register(&h, &d).err != 0) h = nullptr;
+      if (getenv("NORTHUP_CUFILE_DEBUG")) fprintf(stderr, "[northup] cuFileHandleRegister -> %p\n", h);
       it = io.handles.emplace(f, h).first;
     }
     fh = it->second;
@@ -470,6 +481,9 @@ static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* d
   auto xfer = [&](char* p, uint64_t bytes, uint64_t off) -> int {
     if (fh) {
       io.mode = 1;
+      if (getenv("NORTHUP_CUFILE_DEBUG"))
+        fprintf(stderr, "[northup] cuFile%s %llu B at %llu\n", write ? "Write" : "Read", (unsigned long long)bytes,
+                (unsigned long long)off);
       while (bytes) {
         const ssize_t r = write ? api.write(fh, p, bytes, static_cast<off_t>(off), 0)
                                 : api.read(fh, p, bytes, static_cast<off_t>(off), 0);

@@ -308,6 +308,119 @@ __global__ void __launch_bounds__(NWX * NWY * 32, NU_HS_V3_MINB) hotspot_kernel_
     if (r >= ylo && r < yhi) out[r * a.ldo] = v[r];
 }
 
+// ---------------------------------------------------------------------------
+// v4: v3 with packed fp32x2 arithmetic (sm_100 FADD2 / FFMA2).  Thread
+// (lane, warp) keeps the same V-cell column run as v3, held as V/2 pairs
+// (row j, row j + V/2) in 64-bit registers, so one packed instruction updates
+// two cells.  The shared-memory planes store the runs in the same pair layout
+// (pair-row j of run `seg` at pair-row seg*V/2 + j + 1), so the W/E neighbour
+// pairs are aligned 8-byte loads and the new pair one 8-byte store.  Each lane
+// of FADD2/FFMA2 is an IEEE round-to-nearest add / fused multiply-add, and
+// amb - t is formed as fma(-1, t, amb) (one rounding of the exact difference),
+// so every cell follows the RH4 sequence bit for bit: v4 equals v1-v3.
+__device__ __forceinline__ float2 update2(float2 t, float2 p, float2 n, float2 s, float2 e, float2 w,
+                                          float2 ry, float2 rx, float2 rz, float2 cap, float2 amb) {
+  const float2 m2 = make_float2(-2.0f, -2.0f), m1 = make_float2(-1.0f, -1.0f);
+  const float2 ay = __ffma2_rn(m2, t, __fadd2_rn(s, n));
+  const float2 ax = __ffma2_rn(m2, t, __fadd2_rn(e, w));
+  float2 d = __ffma2_rn(ay, ry, p);
+  d = __ffma2_rn(ax, rx, d);
+  d = __ffma2_rn(__ffma2_rn(m1, t, amb), rz, d);
+  return __ffma2_rn(cap, d, t);
+}
+
+template <int V, int NWX, int NWY, bool EDGE>
+__device__ __forceinline__ void v4_iterate(const Args& a, float2* __restrict__ pl0, float2* __restrict__ pl1,
+                                           float2 (&v)[V / 2], const float2 (&p)[V / 2], int x, int pr0,
+                                           int rtop, int rbot, bool wclamp, bool eclamp) {
+  constexpr int SW = NWX * 32 + 2, H = V / 2;
+  const float2 ry = make_float2(a.ry_1, a.ry_1), rx = make_float2(a.rx_1, a.rx_1);
+  const float2 rz = make_float2(a.rz_1, a.rz_1), cap = make_float2(a.cap_1, a.cap_1);
+  const float2 amb = make_float2(a.amb, a.amb);
+  float2* cur = pl0;
+  float2* nxt = pl1;
+  for (int k = 0; k < a.iters; ++k) {
+    const float2* crow = cur + pr0 * SW + (x + 1);   // this thread's first pair
+    const float above = crow[-SW].y;                 // row -1 of the run
+    const float below = crow[H * SW].x;              // row V of the run
+    float2 prev = make_float2(above, v[H - 1].x);    // north pair of pair 0
+    const float mid = v[0].y;                        // row H (south of row H - 1), pre-update
+#pragma unroll
+    for (int j = 0; j < H; ++j) {
+      const float2 c = v[j];
+      float2 n = prev;
+      float2 s = j < H - 1 ? v[j + 1] : make_float2(mid, below);
+      float2 w = crow[j * SW - 1];
+      float2 e = crow[j * SW + 1];
+      if (EDGE) {
+        if (j == rtop) n.x = c.x;
+        if (j + H == rtop) n.y = c.y;
+        if (j == rbot) s.x = c.x;
+        if (j + H == rbot) s.y = c.y;
+        if (wclamp) w = c;
+        if (eclamp) e = c;
+      }
+      v[j] = update2(c, p[j], n, s, e, w, ry, rx, rz, cap, amb);
+      nxt[(pr0 + j) * SW + x + 1] = v[j];
+      prev = c;
+    }
+    __syncthreads();
+    float2* t = cur;
+    cur = nxt;
+    nxt = t;
+  }
+}
+
+template <int V, int NWX, int NWY>
+__global__ void __launch_bounds__(NWX * NWY * 32, 1) hotspot_kernel_v4(Args a) {
+  constexpr int RW = NWX * 32, RH = NWY * V, H = V / 2, SW = RW + 2, SPR = NWY * H + 2;
+  extern __shared__ float2 sm4[];
+  float2* pl0 = sm4;
+  float2* pl1 = sm4 + SPR * SW;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int seg = warp / NWX;
+  const int x = (warp % NWX) * 32 + lane, r0 = seg * V, pr0 = seg * H + 1;
+  const int h = a.iters;
+  const int OTY = RH - 2 * h, OTX = RW - 2 * h;
+  const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
+  const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
+  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
+  const int64_t wx = rx + x;
+  const bool xin = wx >= 0 && wx < a.wn;
+  float2 v[H], p[H];
+#pragma unroll
+  for (int j = 0; j < H; ++j) {
+    const int64_t wy0 = ry + r0 + j, wy1 = wy0 + H;
+    const bool in0 = xin && wy0 >= 0 && wy0 < a.wm, in1 = xin && wy1 >= 0 && wy1 < a.wm;
+    v[j] = make_float2(in0 ? __ldg(a.tin + wy0 * a.ldt + wx) : 0.0f, in1 ? __ldg(a.tin + wy1 * a.ldt + wx) : 0.0f);
+    p[j] = make_float2(in0 ? __ldg(a.pw + wy0 * a.ldp + wx) : 0.0f, in1 ? __ldg(a.pw + wy1 * a.ldp + wx) : 0.0f);
+  }
+#pragma unroll
+  for (int j = 0; j < H; ++j) pl0[(pr0 + j) * SW + x + 1] = v[j];
+  __syncthreads();
+  const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
+  const bool edge = gy_top <= 0 || gy_top + RH >= a.R || gx_left <= 0 || gx_left + RW >= a.C;
+  if (edge) {
+    const int rtop = static_cast<int>(-(gy_top + r0));
+    const int rbot = static_cast<int>(a.R - 1 - (gy_top + r0));
+    const int64_t gcol = gx_left + x;
+    v4_iterate<V, NWX, NWY, true>(a, pl0, pl1, v, p, x, pr0, rtop, rbot, gcol == 0, gcol == a.C - 1);
+  } else {
+    v4_iterate<V, NWX, NWY, false>(a, pl0, pl1, v, p, x, pr0, 0, 0, false, false);
+  }
+  const int64_t oy = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
+  const int64_t ox = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
+  const int64_t sx = ox - h + x;
+  if (sx < ox || sx >= min(ox + OTX, a.vx1)) return;
+  const int ylo = h - r0, yhi = static_cast<int>(min(oy + OTY, a.vy1) - (oy - h)) - r0;
+  float* out = a.tout + (oy - h + r0) * a.ldo + sx;
+#pragma unroll
+  for (int j = 0; j < H; ++j) {
+    if (j >= ylo && j < yhi) out[j * a.ldo] = v[j].x;
+    if (j + H >= ylo && j + H < yhi) out[(j + H) * a.ldo] = v[j].y;
+  }
+}
+
 #ifndef NU_HS_V3_V
 #define NU_HS_V3_V 16
 #endif
@@ -329,12 +442,9 @@ constexpr int kRPT = NU_HS_RPT, kNWX = 4, kNWY = NU_HS_NWY;   // 96 x 128 region
 int hotspot_max_iters_per_launch() { return kHotspotMaxIters; }
 
 static int hotspot_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("NORTHUP_HS_LEAF");
-    v = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 3;   // 1, 2: earlier leaves (DESIGN)
-  }
-  return v;
+  // read per launch (a getenv next to a kernel launch), so tests can switch leaves
+  const char* e = getenv("NORTHUP_HS_LEAF");
+  return (e && e[0] >= '1' && e[0] <= '4') ? e[0] - '0' : 3;   // 1, 2, 3: earlier leaves (DESIGN)
 }
 
 int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
@@ -375,6 +485,19 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.ry_1 = coef[2];
   a.rz_1 = coef[3];
   a.amb = coef[4];
+  if (hotspot_variant() == 4) {
+    constexpr int RH = kV3V * kV3NWY, RW = 32 * kV3NWX;
+    const int oty = RH - 2 * iters, otx = RW - 2 * iters;
+    const int64_t gy4 = (a.vy1 - a.vy0 + oty - 1) / oty, gx4 = (a.vx1 - a.vx0 + otx - 1) / otx;
+    if (gy4 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy4);
+    const int smem4 = 2 * (kV3NWY * kV3V / 2 + 2) * (RW + 2) * 8;
+    cudaFuncSetAttribute(hotspot_kernel_v4<kV3V, kV3NWX, kV3NWY>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem4);
+    hotspot_kernel_v4<kV3V, kV3NWX, kV3NWY><<<dim3(static_cast<unsigned>(gx4), static_cast<unsigned>(gy4)),
+                                             kV3NWX * kV3NWY * 32, smem4, stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v4 launch");
+  }
   if (hotspot_variant() == 3) {
     constexpr int RH = kV3V * kV3NWY, RW = 32 * kV3NWX;
     const int oty = RH - 2 * iters, otx = RW - 2 * iters;

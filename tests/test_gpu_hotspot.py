@@ -116,3 +116,29 @@ def test_in_hbm_leaf_iters_invariance():
     b = run_in_hbm(513, 640, 17, leaf_iters=1)[0]
     c = run_in_hbm(513, 640, 17, leaf_iters=5)[0]
     assert np.array_equal(a, b) and np.array_equal(a, c)
+
+
+@pytest.mark.parametrize("variant", ["1", "2", "3", "4"])
+@pytest.mark.parametrize("R,C,iters", [(700, 900, 8), (129, 131, 3), (1, 257, 5), (300, 2, 7)])
+def test_leaf_variants_bitwise(variant, R, C, iters, monkeypatch):
+    """Every leaf (v1 shared-memory tiles, v2 register shuffles, v3 register
+    runs, v4 packed fp32x2 runs) evaluates RH4's sequence per cell, so each
+    equals the exact fp32 emulation bit for bit — whole grids (edge CTAs) and
+    grids large enough for clamp-free interior CTAs."""
+    monkeypatch.setenv("NORTHUP_HS_LEAF", variant)
+    T, P = grids(R, C, seed=R + 3 * C)
+    dev = torch.device("cuda", 0)
+    t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+    o = torch.full_like(t, float("nan"))
+    nu.hotspot_leaf(t, p, o, iters)
+    full = emulate_fp32(T, P, iters)
+    assert np.array_equal(o.cpu().numpy(), full)
+    # a sub-window: only its valid region is written, equal to the full-grid evolution
+    if R > 2 * iters + 2 and C > 2 * iters + 2:
+        y0, y1, x0, x1 = 1, R - 1, 1, C - 1
+        tw = torch.from_numpy(np.ascontiguousarray(T[y0:y1, x0:x1])).to(dev)
+        pw = torch.from_numpy(np.ascontiguousarray(P[y0:y1, x0:x1])).to(dev)
+        ow = torch.full_like(tw, float("nan"))
+        nu.hotspot_leaf(tw, pw, ow, iters, gy0=y0, gx0=x0, rows=R, cols=C)
+        out = ow.cpu().numpy()
+        assert np.array_equal(out[iters:-iters, iters:-iters], full[y0 + iters:y1 - iters, x0 + iters:x1 - iters])

@@ -1,7 +1,7 @@
 """NEXT-4 GDS edge on one B200: a GEMM whose A, B, C live in files, through
 (a) FILE -> HOST staging -> HBM (DRAM bounce level in the tree),
-(b) FILE -> HBM directly with cuFile (compat mode on this pool's virtio disk),
-(c) FILE -> HBM directly through the library's pinned bounce buffer.
+(b) FILE -> HBM directly through the library's pinned bounce buffer (default),
+    or with cuFile when NORTHUP_CUFILE=1 (compat mode on this pool's virtio disk).
 A is preprocessed to the K-panel-major layout (R15, outside the timing)."""
 import json, os, sys, time, tempfile
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -29,9 +29,10 @@ def tree(kind):
     return t
 
 
-for kind in ("staging", "direct_cufile", "direct_bounce"):
-    if kind == "direct_bounce":
-        os.environ["NORTHUP_NO_CUFILE"] = "1"
+# cuFile is opt-in (NORTHUP_CUFILE=1, read once per process): with it set the
+# direct leg runs through cuFile, else through the pinned bounce buffer
+direct = "direct_cufile" if os.environ.get("NORTHUP_CUFILE") == "1" else "direct_bounce"
+for kind in ("staging", direct):
     t = tree("staging" if kind == "staging" else "direct")
     t.finalize()
     fa = t.open_file(0, f"{d}/A_t.bin", 4 * M * K)
