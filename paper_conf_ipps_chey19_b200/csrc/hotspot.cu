@@ -371,8 +371,11 @@ __device__ __forceinline__ void v4_iterate(const Args& a, float2* __restrict__ p
   }
 }
 
+#ifndef NU_HS_V4_MINB
+#define NU_HS_V4_MINB 1
+#endif
 template <int V, int NWX, int NWY>
-__global__ void __launch_bounds__(NWX * NWY * 32, 1) hotspot_kernel_v4(Args a) {
+__global__ void __launch_bounds__(NWX * NWY * 32, NU_HS_V4_MINB) hotspot_kernel_v4(Args a) {
   constexpr int RW = NWX * 32, RH = NWY * V, H = V / 2, SW = RW + 2, SPR = NWY * H + 2;
   extern __shared__ float2 sm4[];
   float2* pl0 = sm4;
@@ -428,6 +431,16 @@ __global__ void __launch_bounds__(NWX * NWY * 32, 1) hotspot_kernel_v4(Args a) {
 #define NU_HS_V3_NWY 8
 #endif
 constexpr int kV3V = NU_HS_V3_V, kV3NWX = 4, kV3NWY = NU_HS_V3_NWY;
+#ifndef NU_HS_V4_NWX
+#define NU_HS_V4_NWX 4
+#endif
+#ifndef NU_HS_V4_NWY
+#define NU_HS_V4_NWY 8
+#endif
+#ifndef NU_HS_V4_V
+#define NU_HS_V4_V 16
+#endif
+constexpr int kV4V = NU_HS_V4_V, kV4NWX = NU_HS_V4_NWX, kV4NWY = NU_HS_V4_NWY;
 
 #ifndef NU_HS_RPT
 #define NU_HS_RPT 32
@@ -486,15 +499,15 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.rz_1 = coef[3];
   a.amb = coef[4];
   if (hotspot_variant() == 4) {
-    constexpr int RH = kV3V * kV3NWY, RW = 32 * kV3NWX;
+    constexpr int RH = kV4V * kV4NWY, RW = 32 * kV4NWX;
     const int oty = RH - 2 * iters, otx = RW - 2 * iters;
     const int64_t gy4 = (a.vy1 - a.vy0 + oty - 1) / oty, gx4 = (a.vx1 - a.vx0 + otx - 1) / otx;
     if (gy4 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy4);
-    const int smem4 = 2 * (kV3NWY * kV3V / 2 + 2) * (RW + 2) * 8;
-    cudaFuncSetAttribute(hotspot_kernel_v4<kV3V, kV3NWX, kV3NWY>,
+    const int smem4 = 2 * (kV4NWY * kV4V / 2 + 2) * (RW + 2) * 8;
+    cudaFuncSetAttribute(hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem4);
-    hotspot_kernel_v4<kV3V, kV3NWX, kV3NWY><<<dim3(static_cast<unsigned>(gx4), static_cast<unsigned>(gy4)),
-                                             kV3NWX * kV3NWY * 32, smem4, stream>>>(a);
+    hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY><<<dim3(static_cast<unsigned>(gx4), static_cast<unsigned>(gy4)),
+                                             kV4NWX * kV4NWY * 32, smem4, stream>>>(a);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v4 launch");
   }
