@@ -75,6 +75,17 @@ constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
 #ifndef NU_LEAF3_EPI_BUFS
 #define NU_LEAF3_EPI_BUFS 2
 #endif
+// NU_LEAF3_EPI_RED = 1: the epilogue writes C straight from registers (st.global.v4 for
+// the first K chunk, red.global.add.v4.f32 — fp32 RN add in L2, like the TMA reduce —
+// for the others), so TMEM is handed back right after the last tcgen05.ld instead of
+// after the staging boxes drain, and no shared memory is spent on staging.
+#ifndef NU_LEAF3_EPI_RED
+#define NU_LEAF3_EPI_RED 0
+#endif
+#if NU_LEAF3_EPI_RED
+#undef NU_LEAF3_EPI_BUFS
+#define NU_LEAF3_EPI_BUFS 0
+#endif
 constexpr int EPI_WARP0 = 2 + XFORM_WARPS;         // warps 10..
 constexpr int EPI_WARPS = NU_LEAF3_EPI_WARPS;      // 4 or 8: one or two per TMEM lane quarter
 static_assert(EPI_WARPS == 4 || EPI_WARPS == 8, "epilogue warps cover the lane quarters evenly");
@@ -378,6 +389,59 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const uint32_t stage0 = smem_u32(epi_base + (warp - EPI_WARP0) * EPI_BUFS * BOX_BYTES);
     const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16);
     uint32_t chunk_it = 0, box_it = 0;
+#if NU_LEAF3_EPI_RED
+    (void)stage0;
+    (void)box_it;
+    for (int t = cid; t < num_tiles; t += nclusters) {
+      int mb, nb;
+      tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
+      const int grow = mb * BM + rank * BM_CTA + 32 * q + lane;   // this thread's row of C
+      const bool rok = grow < p.M;
+      float* crow = p.C + static_cast<int64_t>(rok ? grow : 0) * p.ldc;
+      for (int ch = 0; ch < nchunks; ++ch, ++chunk_it) {
+        mbar_wait(bar_tfull, chunk_it & 1);
+        tc_fence_after();
+        const bool add = (ch > 0) || p.accumulate;
+#pragma unroll 1
+        for (int c = cbeg; c < cbeg + EPI_COLS / 32; ++c) {
+          uint32_t v[32];
+          __syncwarp();
+          tmem_ld32(t_row + c * 32, v);
+          if (c == cbeg + EPI_COLS / 32 - 1) {
+            tc_fence_before();
+            mbar_arrive_cluster(tempty_leader0);
+          }
+          const int col0 = nb * BN + c * 32;
+          if (!rok) continue;
+          float* dst = crow + col0;
+          if (col0 + 32 <= p.N) {
+            if (add) {
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst + 4 * i),
+                             "r"(v[4 * i]), "r"(v[4 * i + 1]), "r"(v[4 * i + 2]), "r"(v[4 * i + 3])
+                             : "memory");
+            } else {
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(dst + 4 * i), "r"(v[4 * i]),
+                             "r"(v[4 * i + 1]), "r"(v[4 * i + 2]), "r"(v[4 * i + 3])
+                             : "memory");
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              if (col0 + j >= p.N) break;
+              if (add)
+                asm volatile("red.relaxed.gpu.global.add.f32 [%0], %1;" ::"l"(dst + j), "r"(v[j]) : "memory");
+              else
+                asm volatile("st.global.b32 [%0], %1;" ::"l"(dst + j), "r"(v[j]) : "memory");
+            }
+          }
+        }
+      }
+    }
+#else
     for (int t = cid; t < num_tiles; t += nclusters) {
       int mb, nb;
       tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
@@ -416,6 +480,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       }
     }
     if (lane == 0) bulk_wait_all();
+#endif
   }
 
   tc_fence_before();
