@@ -125,20 +125,61 @@ __device__ __forceinline__ void umma_bf16_2sm_ts(uint32_t tmem_d, uint32_t tmem_
       : "memory");
 }
 
+// NU_LEAF3_L2HINT (build-time, L2 residency experiment): bit 0 = A/B panel loads with an
+// evict_last policy, bit 1 = C stores / reductions with evict_first (C streams through
+// L2 once per launch and would otherwise push the panels out).
+#ifndef NU_LEAF3_L2HINT
+#define NU_LEAF3_L2HINT 0
+#endif
+__device__ __forceinline__ uint64_t l2_policy_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
+__device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0,
+                                                 int c1, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3}], [%4], %5;" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar), "l"(pol)
+      : "memory");
+}
+
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
+#if NU_LEAF3_L2HINT & 2
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3}], [%1], %4;" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(src), "r"(c0), "r"(c1), "l"(l2_policy_first())
+               : "memory");
+#else
   asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                    reinterpret_cast<uint64_t>(map)),
                "r"(src), "r"(c0), "r"(c1)
                : "memory");
+#endif
 }
 
 __device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* map, uint32_t src, int c0,
                                                   int c1) {
+#if NU_LEAF3_L2HINT & 2
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group.L2::cache_hint [%0, {%2, %3}], [%1], %4;" ::"l"(
+          reinterpret_cast<uint64_t>(map)),
+      "r"(src), "r"(c0), "r"(c1), "l"(l2_policy_first())
+      : "memory");
+#else
   asm volatile(
       "cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
           reinterpret_cast<uint64_t>(map)),
       "r"(src), "r"(c0), "r"(c1)
       : "memory");
+#endif
 }
 
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
@@ -216,6 +257,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     // ------------------------------------------------------ TMA producer (own half)
     if (lane == 0) {
       uint32_t it = 0;
+#if NU_LEAF3_L2HINT & 1
+      const uint64_t pol_last = l2_policy_last();
+#endif
       for (int t = cid; t < num_tiles; t += nclusters) {
         int mb, nb;
         tile_coords(t, p.tiles_m, p.tiles_n, p.band, mb, nb);
@@ -228,10 +272,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           mbar_arrive_expect_tx(full, TMA_BYTES);
           const uint32_t sa = smem_u32(raw_base + s * TMA_BYTES);
           const uint32_t sb = sa + A_BYTES;
+#if NU_LEAF3_L2HINT & 1
+          tma_load_2d_hint(sa, &tmA, full, kb * BK, row0, pol_last);
+#else
           tma_load_2d(sa, &tmA, full, kb * BK, row0);
+#endif
 #pragma unroll
           for (int c = 0; c < BN_CTA / B_CHUNK; ++c)
+#if NU_LEAF3_L2HINT & 1
+            tma_load_2d_hint(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK, pol_last);
+#else
             tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK);
+#endif
         }
       }
     }
