@@ -48,3 +48,4 @@ def test_ours_quick_json_line():
     assert d["parity"]["bitwise_in_hbm_vs_out_of_core"] and d["parity"]["bitwise_tree_vs_leaf"]
     assert d["parity"]["oracle_ok"] and d["cpu_baseline"]["kind"] == "oracle"
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
+    assert d["cfg2_in_hbm_tflops"] > 0 and "slowdown_pct_vs_cfg2_in_hbm" in d
