@@ -449,15 +449,102 @@ struct CuFileDescr {
 
 struct DevIO {
   std::map<const northup_buf_s*, void*> handles;   // cuFile handle per file
-  char* bounce = nullptr;                          // pinned fallback buffer
+  char* bounce = nullptr;                          // pinned fallback buffer: two halves
   size_t bounce_bytes = 0;
   int mode = 0;                                    // 1 = cuFile, 2 = bounce
+  struct Dev {
+    cudaStream_t s = nullptr;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+  };
+  std::map<int, Dev> dev;                          // copy stream + per-half events per device
   ~DevIO() {
     for (auto& kv : handles)
       if (kv.second && g_cufile.handle_deregister) g_cufile.handle_deregister(kv.second);
+    for (auto& kv : dev) {
+      cudaSetDevice(kv.first);
+      if (kv.second.s) cudaStreamSynchronize(kv.second.s), cudaStreamDestroy(kv.second.s);
+      for (cudaEvent_t e : kv.second.ev)
+        if (e) cudaEventDestroy(e);
+    }
     if (bounce) cudaFreeHost(bounce);
   }
 };
+
+// The pinned-bounce transfer of a rows x cols block between a file and device
+// memory, pipelined over the two halves of the bounce buffer: while the DMA
+// engine copies one group of rows (cudaMemcpy2DAsync on a private stream), the
+// I/O thread reads (or writes) the next group from (to) the file.
+static int bounce_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* dmem, int64_t mem_ld,
+                            int64_t file_off, int64_t file_ld, int64_t rows, int64_t cols) {
+  io.mode = 2;
+  if (!io.bounce) {
+    io.bounce_bytes = 64ull << 20;
+    cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&io.bounce), io.bounce_bytes, cudaHostAllocPortable);
+    if (e != cudaSuccess) return cuda_fail(e, "bounce buffer");
+  }
+  int d = 0;
+  cudaGetDevice(&d);
+  DevIO::Dev& D = io.dev[d];
+  if (!D.s) {
+    cudaError_t e = cudaStreamCreateWithFlags(&D.s, cudaStreamNonBlocking);
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i) e = cudaEventCreateWithFlags(&D.ev[i], cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_fail(e, "bounce stream");
+  }
+  const uint64_t half = io.bounce_bytes / 2, row_bytes = static_cast<uint64_t>(cols) * 4;
+  if (row_bytes > half) {   // one row larger than a half: split the columns
+    for (int64_t c0 = 0; c0 < cols; c0 += static_cast<int64_t>(half / 4)) {
+      const int64_t nc = std::min<int64_t>(static_cast<int64_t>(half / 4), cols - c0);
+      int rc = bounce_block_dev(io, f, write, dmem + c0 * 4, mem_ld, file_off + c0, file_ld, rows, nc);
+      if (rc) return rc;
+    }
+    return 0;
+  }
+  const int64_t per = static_cast<int64_t>(half / row_bytes);
+  const int64_t ngroups = (rows + per - 1) / per;
+  auto group = [&](int64_t g, int64_t* r0, int64_t* nr) {
+    *r0 = g * per;
+    *nr = std::min(per, rows - *r0);
+  };
+  cudaError_t e = cudaSuccess;
+  if (!write) {
+    for (int64_t g = 0; g < ngroups; ++g) {
+      int64_t r0, nr;
+      group(g, &r0, &nr);
+      const int sl = static_cast<int>(g & 1);
+      char* hb = io.bounce + sl * half;
+      if ((e = cudaEventSynchronize(D.ev[sl])) != cudaSuccess) return cuda_fail(e, "bounce wait");
+      int rc = file_block(f, false, hb, cols, file_off + r0 * file_ld, file_ld, nr, cols);
+      if (rc) return rc;
+      e = cudaMemcpy2DAsync(dmem + r0 * mem_ld * 4, static_cast<size_t>(mem_ld) * 4, hb, row_bytes, row_bytes,
+                            static_cast<size_t>(nr), cudaMemcpyHostToDevice, D.s);
+      if (e == cudaSuccess) e = cudaEventRecord(D.ev[sl], D.s);
+      if (e != cudaSuccess) return cuda_fail(e, "bounce H2D");
+    }
+  } else {
+    for (int64_t g = 0; g <= ngroups; ++g) {
+      if (g < ngroups) {   // start the D2H of group g ...
+        int64_t r0, nr;
+        group(g, &r0, &nr);
+        const int sl = static_cast<int>(g & 1);
+        char* hb = io.bounce + sl * half;
+        e = cudaMemcpy2DAsync(hb, row_bytes, dmem + r0 * mem_ld * 4, static_cast<size_t>(mem_ld) * 4, row_bytes,
+                              static_cast<size_t>(nr), cudaMemcpyDeviceToHost, D.s);
+        if (e == cudaSuccess) e = cudaEventRecord(D.ev[sl], D.s);
+        if (e != cudaSuccess) return cuda_fail(e, "bounce D2H");
+      }
+      if (g > 0) {         // ... while group g - 1 goes to the file
+        int64_t r0, nr;
+        group(g - 1, &r0, &nr);
+        const int sl = static_cast<int>((g - 1) & 1);
+        if ((e = cudaEventSynchronize(D.ev[sl])) != cudaSuccess) return cuda_fail(e, "bounce wait");
+        int rc = file_block(f, true, io.bounce + sl * half, cols, file_off + r0 * file_ld, file_ld, nr, cols);
+        if (rc) return rc;
+      }
+    }
+  }
+  if ((e = cudaStreamSynchronize(D.s)) != cudaSuccess) return cuda_fail(e, "bounce sync");
+  return 0;
+}
 
 // A rows x cols fp32 block between a file and DEVICE memory.
 static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* dmem, int64_t mem_ld,
@@ -478,46 +565,19 @@ static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* d
     }
     fh = it->second;
   }
+  if (!fh) return bounce_block_dev(io, f, write, dmem, mem_ld, file_off, file_ld, rows, cols);
   auto xfer = [&](char* p, uint64_t bytes, uint64_t off) -> int {
-    if (fh) {
-      io.mode = 1;
-      if (getenv("NORTHUP_CUFILE_DEBUG"))
-        fprintf(stderr, "[northup] cuFile%s %llu B at %llu\n", write ? "Write" : "Read", (unsigned long long)bytes,
-                (unsigned long long)off);
-      while (bytes) {
-        const ssize_t r = write ? api.write(fh, p, bytes, static_cast<off_t>(off), 0)
-                                : api.read(fh, p, bytes, static_cast<off_t>(off), 0);
-        if (r <= 0) return fail(NU_EIO, "cuFile%s(%s) returned %zd", write ? "Write" : "Read", f->path.c_str(), r);
-        p += r;
-        bytes -= static_cast<uint64_t>(r);
-        off += static_cast<uint64_t>(r);
-      }
-      return 0;
-    }
-    io.mode = 2;
-    if (!io.bounce) {
-      io.bounce_bytes = 64ull << 20;
-      cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&io.bounce), io.bounce_bytes, cudaHostAllocPortable);
-      if (e != cudaSuccess) return cuda_fail(e, "bounce buffer");
-    }
+    io.mode = 1;
+    if (getenv("NORTHUP_CUFILE_DEBUG"))
+      fprintf(stderr, "[northup] cuFile%s %llu B at %llu\n", write ? "Write" : "Read", (unsigned long long)bytes,
+              (unsigned long long)off);
     while (bytes) {
-      const uint64_t n = std::min<uint64_t>(bytes, io.bounce_bytes);
-      if (write) {
-        cudaError_t e = cudaMemcpy(io.bounce, p, n, cudaMemcpyDefault);
-        if (e != cudaSuccess) return cuda_fail(e, "bounce D2H");
-        int rc = file_block(f, true, io.bounce, static_cast<int64_t>(n / 4), static_cast<int64_t>(off / 4),
-                            static_cast<int64_t>(n / 4), 1, static_cast<int64_t>(n / 4));
-        if (rc) return rc;
-      } else {
-        int rc = file_block(f, false, io.bounce, static_cast<int64_t>(n / 4), static_cast<int64_t>(off / 4),
-                            static_cast<int64_t>(n / 4), 1, static_cast<int64_t>(n / 4));
-        if (rc) return rc;
-        cudaError_t e = cudaMemcpy(p, io.bounce, n, cudaMemcpyDefault);
-        if (e != cudaSuccess) return cuda_fail(e, "bounce H2D");
-      }
-      p += n;
-      bytes -= n;
-      off += n;
+      const ssize_t r = write ? api.write(fh, p, bytes, static_cast<off_t>(off), 0)
+                              : api.read(fh, p, bytes, static_cast<off_t>(off), 0);
+      if (r <= 0) return fail(NU_EIO, "cuFile%s(%s) returned %zd", write ? "Write" : "Read", f->path.c_str(), r);
+      p += r;
+      bytes -= static_cast<uint64_t>(r);
+      off += static_cast<uint64_t>(r);
     }
     return 0;
   };
