@@ -212,10 +212,13 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       w->tev.push_back(ev);
     }
   }
+  const bool dbg = getenv("NORTHUP_DEBUG_EXEC") != nullptr;
   for (size_t i = 0; i < nops; ++i) {
     const northup_op& op = P.ops[i];
     if (op.worker != wi) continue;
     cudaStream_t s = w->streams[op.stream];
+    if (dbg) fprintf(stderr, "[northup] worker %d issues op %zu (kind %d, stream %d, %d deps)\n", wi, i, op.op,
+                     op.stream, op.ndeps);
     for (int d = 0; d < op.ndeps; ++d) {
       const northup_op& q = P.ops[op.deps[d]];
       if (q.stream == S_IO) {
@@ -327,6 +330,24 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
     if (e != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
     e = cudaGraphLaunch(*capture_out, w->streams[0]);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
+  }
+  if (c.local >= 0 && c.cross) {
+    // multi-process siblings: the streams wait on flags other processes write, so a
+    // peer that died would block them forever; poll with a deadline instead
+    // (NORTHUP_PEER_TIMEOUT_S, default 600 s) and fail loudly
+    const char* to = getenv("NORTHUP_PEER_TIMEOUT_S");
+    const double limit = to ? atof(to) : 600.0;
+    const auto t0 = std::chrono::steady_clock::now();
+    if (dbg) fprintf(stderr, "[northup] worker %d: all ops issued, polling (limit %.0f s)\n", wi, limit);
+    for (cudaStream_t s : w->streams) {
+      while ((e = cudaStreamQuery(s)) == cudaErrorNotReady) {
+        if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > limit)
+          return fail(NU_ECUDA, "multi-process siblings: no progress from the peer processes for %.0f s "
+                                "(did a sibling fail?)", limit);
+        std::this_thread::sleep_for(std::chrono::microseconds(20));
+      }
+      if (e != cudaSuccess) return cuda_fail(e, "stream synchronize");
+    }
   }
   for (cudaStream_t s : w->streams) {
     e = cudaStreamSynchronize(s);
@@ -706,6 +727,13 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
         if (op.worker != lw && P.ops[op.deps[d]].worker == lw)
           needs_remote[op.deps[d]] |= uint64_t(1) << op.worker;
     ctx.gen = ++t->gen;
+    // every kernel loaded before any stream waits on another process: with lazy
+    // module loading a first launch behind such a wait blocks the issuing thread
+    WorkerState* lwst = worker_for_node(t, P.worker_node[lw]);
+    if (lwst) {
+      cudaSetDevice(lwst->device);
+      preload_kernels();
+    }
   }
   ctx.issued.assign(P.ops.size(), 0);
   if (ctx.timing) t->timeline.clear();

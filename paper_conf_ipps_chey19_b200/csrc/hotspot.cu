@@ -454,6 +454,15 @@ constexpr int kRPT = NU_HS_RPT, kNWX = 4, kNWY = NU_HS_NWY;   // 96 x 128 region
 
 int hotspot_max_iters_per_launch() { return kHotspotMaxIters; }
 
+void hotspot_preload() {
+  using namespace hs;
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, hotspot_kernel);
+  cudaFuncGetAttributes(&fa, hotspot_kernel_v2<kRPT, kNWX, kNWY>);
+  cudaFuncGetAttributes(&fa, hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY>);
+  cudaFuncGetAttributes(&fa, hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY>);
+}
+
 static int hotspot_variant() {
   // read per launch (a getenv next to a kernel launch), so tests can switch leaves
   const char* e = getenv("NORTHUP_HS_LEAF");

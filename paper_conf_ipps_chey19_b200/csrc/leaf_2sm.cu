@@ -417,6 +417,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
 
 }  // namespace sm2
 
+void preload_sm2() {
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, sm2::leaf_gemm_2sm_kernel);
+}
+
 int launch_sm2(LaunchArgs& a) {
   using namespace sm2;
   int rc;

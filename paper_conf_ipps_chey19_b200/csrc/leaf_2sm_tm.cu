@@ -554,6 +554,11 @@ bool launch_sm4_ok(const LaunchArgs& a) {
   return a.p.npass == 2 && !a.p.b_kmajor && a.p.vec_ok;
 }
 
+void preload_sm4() {
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, sm4::leaf_gemm_2sm_tm_kernel);
+}
+
 int launch_sm4(LaunchArgs& a) {
   using namespace sm4;
   int rc;

@@ -197,6 +197,12 @@ int launch_sm1(LaunchArgs& a);   // v0: 1-CTA 128 x 256 tile
 int launch_sm2(LaunchArgs& a);   // v1: CTA pair (cta_group::2) 256 x 256 tile, TMA-fed
 int launch_sm3(LaunchArgs& a);   // v2: CTA pair, split warps load global memory directly
 int launch_sm4(LaunchArgs& a);   // v3: CTA pair, A' operand in TMEM, TMA-store epilogue
+// Load each variant's kernel now (lazy module loading would otherwise load it at its
+// first launch, which can block behind a stream that waits on another process).
+void preload_sm1();
+void preload_sm2();
+void preload_sm3();
+void preload_sm4();
 bool launch_sm4_ok(const LaunchArgs& a);
 
 }  // namespace leaf

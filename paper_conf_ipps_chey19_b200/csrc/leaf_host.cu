@@ -66,6 +66,18 @@ __global__ void debug_spin_kernel(long long ns) {
   while (clock64() - t0 < cycles) __nanosleep(1000);
 }
 
+// Load every kernel the executor may launch on the current device (see
+// leaf_common.cuh preload_sm*): run before work that waits on other processes.
+void preload_kernels() {
+  leaf::preload_sm1();
+  leaf::preload_sm2();
+  leaf::preload_sm3();
+  leaf::preload_sm4();
+  hotspot_preload();
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, debug_spin_kernel);
+}
+
 int debug_spin(long long ns, cudaStream_t s) {
   debug_spin_kernel<<<1, 1, 0, s>>>(ns);
   cudaError_t e = cudaGetLastError();

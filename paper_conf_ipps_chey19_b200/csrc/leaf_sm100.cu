@@ -289,6 +289,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
 }  // namespace sm1
 
+void preload_sm1() {
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, sm1::leaf_gemm_1sm_kernel);
+}
+
 int launch_sm1(LaunchArgs& a) {
   using namespace sm1;
   int rc;

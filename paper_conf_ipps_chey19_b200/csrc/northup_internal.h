@@ -176,6 +176,9 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
 // The executors hold that sibling's compute stream for pct % of each leaf's
 // nominal time (2mnk at 300 TF/s) before launching it: a slower GPU.
 int debug_spin(long long ns, cudaStream_t s);
+// Force-load the kernels (lazy module loading) on the current device; hotspot.cu's part.
+void preload_kernels();
+void hotspot_preload();
 int debug_slow_sibling(int* pct);
 inline long long debug_slow_ns(int pct, int64_t m, int64_t n, int64_t k) {
   return static_cast<long long>(pct / 100.0 * 2.0 * m * n * k / 3e14 * 1e9);

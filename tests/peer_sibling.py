@@ -46,10 +46,20 @@ def main():
         for w in range(G):
             if w != rank:
                 t.peer_import(w, open(os.path.join(d, f"blob{w}"), "rb").read())
+    if os.environ.get("PEER_SKIP_GEMM") == str(rank):
+        # a sibling that never runs its part: the others must fail, not hang
+        wait_for([os.path.join(d, f"err{w}") for w in range(G) if w != rank], timeout=240)
+        open(os.path.join(d, f"done{rank}"), "w").close()
+        return
     outs = []
     for _ in range(reps):
         c[...] = np.nan
-        st = t.gemm(A, B, C, M, N, K, o)
+        try:
+            st = t.gemm(A, B, C, M, N, K, o)
+        except nu.NorthupError as ex:
+            open(os.path.join(d, f"err{rank}"), "w").write(str(ex))
+            print("NorthupError:", ex, flush=True)
+            os._exit(3)
         outs.append(c.copy())
     np.save(os.path.join(d, f"c{rank}.npy"), np.stack(outs))
     with open(os.path.join(d, f"st{rank}.txt"), "w") as f:

@@ -19,13 +19,18 @@ pytestmark = pytest.mark.gpu
 HERE = os.path.dirname(os.path.abspath(__file__))
 
 
-def run_siblings(tmp, G, M, N, K, kc, shared, kind, reps=2):
+def spawn(tmp, G, M, N, K, kc, shared, kind, reps, env=None):
     d = tmp / f"rdv_{G}_{shared}_{kind}"
     d.mkdir()
     procs = [subprocess.Popen([sys.executable, os.path.join(HERE, "peer_sibling.py"), str(d), str(r),
                                str(G), str(M), str(N), str(K), str(kc), str(shared), kind, str(reps)],
-                              stdout=subprocess.PIPE, stderr=subprocess.STDOUT)
+                              stdout=subprocess.PIPE, stderr=subprocess.STDOUT, env=env)
              for r in range(G)]
+    return d, procs
+
+
+def run_siblings(tmp, G, M, N, K, kc, shared, kind, reps=2):
+    d, procs = spawn(tmp, G, M, N, K, kc, shared, kind, reps)
     outs = []
     for p in procs:
         try:
@@ -61,3 +66,23 @@ def test_multiprocess_shared_staging(tmp_path, G, M, N, K, kind):
     else:
         e, where = oracle.normwise_err(Cs[0], ref, oracle.row_norms(a), oracle.col_norms(b))
         assert e <= 1e-5, (e, where)
+
+
+def test_multiprocess_dead_peer_fails_loudly(tmp_path):
+    """A sibling process that never runs its part: the other sibling's call
+    returns NU_ECUDA after NORTHUP_PEER_TIMEOUT_S instead of blocking forever
+    on the device-side flag waits."""
+    env = dict(os.environ, PEER_SKIP_GEMM="1", NORTHUP_PEER_TIMEOUT_S="5")
+    d, procs = spawn(tmp_path, 2, 512, 512, 1024, 256, 0, "int", 1, env=env)
+    outs = []
+    try:
+        for p in procs:
+            out, _ = p.communicate(timeout=180)
+            outs.append(out.decode(errors="replace"))
+    finally:
+        for p in procs:
+            if p.poll() is None:
+                p.kill()
+    assert procs[0].returncode == 3, outs[0]
+    assert "no progress from the peer processes" in outs[0]
+    assert procs[1].returncode == 0, outs[1]
