@@ -60,6 +60,10 @@ int finalize_workers(northup_tree_s* t) {
       e = cudaStreamCreateWithFlags(&w->streams[s], cudaStreamNonBlocking);
     t->workers.push_back(w);
     if (e != cudaSuccess) return cuda_fail(e, "stream creation");
+    // load every kernel now: with lazy module loading a kernel's first launch can
+    // block the issuing thread behind a stream that waits on another worker's or
+    // process's progress (cross-sibling waits), which can close a cycle
+    preload_kernels();
   }
   // Shared staging pulls panels from sibling HBM: enable NVLink P2P between
   // every pair of distinct devices (without it the copies still work, staged
@@ -727,13 +731,6 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
         if (op.worker != lw && P.ops[op.deps[d]].worker == lw)
           needs_remote[op.deps[d]] |= uint64_t(1) << op.worker;
     ctx.gen = ++t->gen;
-    // every kernel loaded before any stream waits on another process: with lazy
-    // module loading a first launch behind such a wait blocks the issuing thread
-    WorkerState* lwst = worker_for_node(t, P.worker_node[lw]);
-    if (lwst) {
-      cudaSetDevice(lwst->device);
-      preload_kernels();
-    }
   }
   ctx.issued.assign(P.ops.size(), 0);
   if (ctx.timing) t->timeline.clear();
