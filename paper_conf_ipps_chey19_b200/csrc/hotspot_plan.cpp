@@ -229,10 +229,38 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
     const int64_t itq = std::min(h, iters - q * h);
     const int dst = ((Q - 1 - q) % 2 == 0) ? OUT : S;
     const int ldg_src = C, ldg_dst = C;
+    // Blocks of one pass are independent (they read the pass's source grid and
+    // write its destination), so each sibling's first block of the first pass and
+    // last block of the last pass are split 2 x 2: the pipeline fills after a
+    // quarter-size window and drains a quarter-size block (a little more border
+    // recomputation on those two blocks only).
+    std::vector<Win> blks;
+    std::vector<int> owner;
     for (int64_t by = 0; by < nby; ++by) {
       const int w = static_cast<int>(by * G / nby);   // block rows split over the siblings
+      const bool w_first_row = by == 0 || static_cast<int>((by - 1) * G / nby) != w;
+      const bool w_last_row = by == nby - 1 || static_cast<int>((by + 1) * G / nby) != w;
       for (int64_t bx = 0; bx < nbx; ++bx) {
         const Win blk{by * b, std::min(R, (by + 1) * b), bx * b, std::min(C, (bx + 1) * b)};
+        const bool split = ((q == 0 && w_first_row && bx == 0) || (q == Q - 1 && w_last_row && bx == nbx - 1)) &&
+                           blk.y1 - blk.y0 >= 256 && blk.x1 - blk.x0 >= 256;
+        if (!split) {
+          blks.push_back(blk);
+          owner.push_back(w);
+          continue;
+        }
+        const int64_t ym = blk.y0 + rup(cdiv(blk.y1 - blk.y0, 2), 64), xm = blk.x0 + rup(cdiv(blk.x1 - blk.x0, 2), 64);
+        for (const Win& sb : {Win{blk.y0, ym, blk.x0, xm}, Win{blk.y0, ym, xm, blk.x1}, Win{ym, blk.y1, blk.x0, xm},
+                              Win{ym, blk.y1, xm, blk.x1}}) {
+          blks.push_back(sb);
+          owner.push_back(w);
+        }
+      }
+    }
+    for (size_t bi = 0; bi < blks.size(); ++bi) {
+      const int w = owner[bi];
+      {
+        const Win blk = blks[bi];
         const Win win_g{std::max<int64_t>(0, blk.y0 - itq), std::min(R, blk.y1 + itq),
                         std::max<int64_t>(0, blk.x0 - itq), std::min(C, blk.x1 + itq)};
         const int64_t wm = win_g.y1 - win_g.y0, wn = win_g.x1 - win_g.x0;

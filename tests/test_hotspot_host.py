@@ -78,6 +78,8 @@ def simulate_hotspot(plan, T, P, R, C, rng=None):
     (50, 30, 7, 3, 0, 12, 7, 8),        # 3 siblings, ragged blocks
     (70, 45, 11, 2, 0, 16, 2, 1),       # 6 passes (odd/even grid alternation), leaf_iters 1
     (96, 96, 10, 1, 200_000, 0, 5, 0),  # capacity picks the block
+    (600, 520, 9, 2, 0, 300, 4, 4),     # 3 passes, 2 siblings: first / last blocks split 2 x 2
+    (512, 512, 6, 1, 0, 256, 0, 0),     # one pass: its first and last blocks split
 ])
 def test_hotspot_plan_replays_exactly(R, C, iters, G, cap, block, halo, leaf):
     T, P = grids(R, C, seed=R + C + iters)
@@ -90,6 +92,9 @@ def test_hotspot_plan_replays_exactly(R, C, iters, G, cap, block, halo, leaf):
         assert np.array_equal(out, ref), f"order seed {seed} broke a dependency"
     s = p.stats()
     b, h = s["bm"], s["bk"]
+    if b >= 256:   # split blocks: more windows than the plain b x b grid
+        nwin = sum(1 for o in p.ops() if o["op"] == nu.NU_OP_COPY and o["stream"] == 0) // 2
+        assert nwin > -(-R // b) * -(-C // b) * -(-iters // h)
     assert s["bytes_d2h"] == 4 * R * C * -(-iters // h)          # every pass writes the grid once
     if cap:
         assert all(x["bytes"] <= cap for x in p.bufs() if x["kind"] == 3)

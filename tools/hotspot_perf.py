@@ -47,7 +47,7 @@ Tb, Pb, Ob = t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0)
 view = lambda b: np.ctypeslib.as_array((ctypes.c_float * (R * C)).from_address(b.ptr)).reshape(R, C)
 view(Tb)[...] = T
 view(Pb)[...] = P
-o = nu.hotspot_opts()
+o = nu.hotspot_opts(block=int(os.environ.get("HS_BLOCK", "0")))
 t.hotspot(Tb, Pb, Ob, R, C, ITERS, o)
 ms = []
 for _ in range(2):
