@@ -268,7 +268,7 @@ int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, 
 typedef struct {
   int op;
   int worker;   /* GPU worker index (0 .. num_gpus-1) */
-  int stream;   /* 0 = H2D, 1 = compute, 2 = D2H, 3 = file I/O, 4 = D2D (sibling pulls) */
+  int stream;   /* 0 = H2D, 1 = compute, 2 = D2H, 3 = file reads, 4 = D2D (sibling pulls), 5 = file writes */
   int accumulate;
   int src_buf, dst_buf; /* COPY */
   int a_buf, b_buf, c_buf; /* LEAF / ZERO(c) */

@@ -225,7 +225,7 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
                      op.stream, op.ndeps);
     for (int d = 0; d < op.ndeps; ++d) {
       const northup_op& q = P.ops[op.deps[d]];
-      if (q.stream == S_IO) {
+      if (is_io_stream(q.stream)) {
         if (!wait_flag(c, c.io_done, op.deps[d])) return fail(NU_EIO, "aborted: file I/O failed");
         continue;
       }
@@ -616,16 +616,22 @@ static int file_block_dev(DevIO& io, const northup_buf_s* f, bool write, char* d
   return 0;
 }
 
-static int run_io(RunCtx& c) {
+// One I/O queue (`queue` = S_IO file reads or S_IOW file writes) on its own
+// host thread, so a round's C write-back overlaps the next round's panel reads.
+static int run_io(RunCtx& c, int queue) {
   const Plan& P = *c.plan;
   const auto t0 = std::chrono::steady_clock::now();
   DevIO dio;
   for (size_t i = 0; i < P.ops.size(); ++i) {
     const northup_op& op = P.ops[i];
-    if (op.stream != S_IO) continue;
+    if (op.stream != queue) continue;
     for (int d = 0; d < op.ndeps; ++d) {
       const northup_op& q = P.ops[op.deps[d]];
-      if (q.stream == S_IO) continue;
+      if (is_io_stream(q.stream)) {   // the other I/O queue (this one runs in order)
+        if (q.stream != queue && !wait_flag(c, c.io_done, op.deps[d]))
+          return fail(NU_EIO, "aborted: file I/O failed");
+        continue;
+      }
       if (!wait_flag(c, c.issued, op.deps[d])) return fail(NU_ECUDA, "aborted: a GPU worker failed");
       WorkerState* w = worker_for_node(c.t, P.worker_node[q.worker]);
       cudaSetDevice(w->device);
@@ -651,11 +657,16 @@ static int run_io(RunCtx& c) {
     mark(c, c.io_done, i);
   }
   // O_SYNC semantics of P:242: C is durable when northup_gemm returns.
-  for (size_t b = 0; b < c.file.size(); ++b)
-    if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0)
-      return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(errno));
-  c.io_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
-  c.io_mode = dio.mode;
+  if (queue == S_IOW)
+    for (size_t b = 0; b < c.file.size(); ++b)
+      if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0)
+        return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(errno));
+  const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  {
+    std::lock_guard<std::mutex> g(c.m);
+    c.io_ms = std::max(c.io_ms, ms);
+    c.io_mode = std::max(c.io_mode, dio.mode);
+  }
   return 0;
 }
 
@@ -710,10 +721,10 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   for (const northup_op& op : P.ops) {
     for (int d = 0; d < op.ndeps; ++d) {
       needs[op.deps[d]] = 1;
-      cross |= P.ops[op.deps[d]].worker != op.worker && P.ops[op.deps[d]].stream != S_IO &&
-               op.stream != S_IO;
+      cross |= P.ops[op.deps[d]].worker != op.worker && !is_io_stream(P.ops[op.deps[d]].stream) &&
+               !is_io_stream(op.stream);
     }
-    has_io |= op.stream == S_IO;
+    has_io |= is_io_stream(op.stream);
   }
   ctx.needs_event = &needs;
   ctx.cross = cross;
@@ -763,8 +774,8 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     destroy_graphs(t);
     t->graph_execs.assign(W, nullptr);
   }
-  std::vector<int> rcs(W + 1, 0);
-  std::vector<std::string> errs(W + 1);
+  std::vector<int> rcs(W + 2, 0);        // workers, then the read and the write I/O threads
+  std::vector<std::string> errs(W + 2);
   std::vector<std::vector<double>> busy(W, std::vector<double>(S_NUM, 0.0));
   auto worker_body = [&](int wi) {
     cudaGraphExec_t ge = nullptr;
@@ -776,10 +787,10 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
       ctx.cv.notify_all();
     }
   };
-  auto io_body = [&] {
-    rcs[W] = run_io(ctx);
-    if (rcs[W]) {
-      errs[W] = northup_last_error();
+  auto io_body = [&](int k) {
+    rcs[W + k] = run_io(ctx, k == 0 ? S_IO : S_IOW);
+    if (rcs[W + k]) {
+      errs[W + k] = northup_last_error();
       ctx.abort = true;
       ctx.cv.notify_all();
     }
@@ -792,10 +803,13 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   } else {
     std::vector<std::thread> th;
     for (int wi : mine) th.emplace_back(worker_body, wi);
-    if (has_io) th.emplace_back(io_body);
+    if (has_io) {
+      th.emplace_back(io_body, 0);
+      th.emplace_back(io_body, 1);
+    }
     for (auto& x : th) x.join();
   }
-  for (int wi = 0; wi <= W; ++wi)
+  for (int wi = 0; wi <= W + 1; ++wi)
     if (rcs[wi]) {
       if (use_graph) destroy_graphs(t);
       return fail(rcs[wi], "%s %d: %s", wi < W ? "worker" : "I/O thread", wi, errs[wi].c_str());

@@ -98,7 +98,10 @@ struct northup_tree_s {
 namespace nu {
 
 // --------------------------------------------------------------- plan
-enum Stream { S_H2D = 0, S_COMP = 1, S_D2H = 2, S_IO = 3, S_D2D = 4, S_NUM = 5 };
+// S_NUM CUDA streams per worker (S_IO's slot unused); S_IO / S_IOW are the
+// file-read and file-write queues of the I/O pseudo-worker (one host thread each)
+enum Stream { S_H2D = 0, S_COMP = 1, S_D2H = 2, S_IO = 3, S_D2D = 4, S_NUM = 5, S_IOW = 5, S_KEYS = 6 };
+inline bool is_io_stream(int s) { return s == S_IO || s == S_IOW; }
 enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3, B_DRAM = 4 };
 
 struct PlanBuf {

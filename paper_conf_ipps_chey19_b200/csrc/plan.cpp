@@ -688,7 +688,8 @@ int build_in_hbm(Builder& B, int node, int64_t M, int64_t N, int64_t K, int A, i
 // strip by strip and are written back to the C file (Listing 4 file_write).
 northup_op make_io(int io_worker, int op, int src, int64_t src_off, int64_t src_ld, int dst,
                    int64_t dst_off, int64_t dst_ld, int64_t rows, int64_t cols) {
-  northup_op o = make_copy(io_worker, S_IO, src, src_off, src_ld, dst, dst_off, dst_ld, rows, cols);
+  northup_op o = make_copy(io_worker, op == NU_OP_IO_WRITE ? S_IOW : S_IO, src, src_off, src_ld, dst, dst_off,
+                           dst_ld, rows, cols);
   o.op = op;
   return o;
 }

@@ -78,9 +78,9 @@ struct Builder {
         if (q.worker == op.worker && q.stream == op.stream) continue;
         // root-tier regions of different siblings are disjoint by construction
         // (their 2-D bounding intervals may still overlap)
-        if (user_disjoint && user && q.worker != op.worker && q.stream != S_IO && op.stream != S_IO)
+        if (user_disjoint && user && q.worker != op.worker && !is_io_stream(q.stream) && !is_io_stream(op.stream))
           continue;
-        const int key = q.worker * S_NUM + q.stream;
+        const int key = q.worker * S_KEYS + q.stream;
         bool found = false;
         for (auto& kv : last)
           if (kv.first == key) {
