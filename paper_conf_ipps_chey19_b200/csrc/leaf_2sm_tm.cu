@@ -151,6 +151,19 @@ __device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const CUtensorMap
       : "memory");
 }
 
+// NU_LEAF3_PF = d > 0: the TMA producer also prefetches the tiles of k-block
+// kb + d into L2 (cp.async.bulk.prefetch.tensor), so a raw-ring load that would
+// miss L2 (panel re-reads, ~20 % of sectors) finds its data there.
+#ifndef NU_LEAF3_PF
+#define NU_LEAF3_PF 0
+#endif
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, int c1) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
+
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
 #if NU_LEAF3_L2HINT & 2
   asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3}], [%1], %4;" ::"l"(
@@ -283,6 +296,28 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             tma_load_2d_hint(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK, pol_last);
 #else
             tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK);
+#endif
+#if NU_LEAF3_PF > 0
+          {
+            int pk = kb + NU_LEAF3_PF, prow = row0, pcol = col0;
+            if (pk >= nkb) {   // the next tile's first k-blocks
+              const int tn = t + nclusters;
+              if (tn < num_tiles) {
+                int mb2, nb2;
+                tile_coords(tn, p.tiles_m, p.tiles_n, p.band, mb2, nb2);
+                prow = mb2 * BM + rank * BM_CTA;
+                pcol = nb2 * BN + rank * BN_CTA;
+                pk -= nkb;
+              } else {
+                pk = -1;
+              }
+            }
+            if (pk >= 0 && pk < nkb) {
+              tma_prefetch_2d(&tmA, pk * BK, prow);
+#pragma unroll
+              for (int c = 0; c < BN_CTA / B_CHUNK; ++c) tma_prefetch_2d(&tmB, pcol + c * B_CHUNK, pk * BK);
+            }
+          }
 #endif
         }
       }
