@@ -67,7 +67,12 @@ constexpr int A_BYTES = BM_CTA * BK * 4;           // 16 KiB
 constexpr int B_BYTES = BN_CTA * BK * 4;           // 16 KiB
 constexpr int TMA_BYTES = A_BYTES + B_BYTES;
 constexpr int XB_BYTES = 2 * BK * BN_CTA * 2;      // B' bf16: 64 virtual k x 128 n = 16 KiB
-constexpr int XFORM_WARPS = 8;                     // warps 2..9: two per TMEM lane quarter
+#ifndef NU_LEAF3_XFORM_WARPS
+#define NU_LEAF3_XFORM_WARPS 8
+#endif
+constexpr int XFORM_WARPS = NU_LEAF3_XFORM_WARPS;  // warps 2..: 8 = two, 16 = four per TMEM lane quarter
+static_assert(XFORM_WARPS == 8 || XFORM_WARPS == 16, "split warps cover the lane quarters evenly");
+constexpr int XF_KPW = 32 / (XFORM_WARPS / 4);      // real k of a stage each split warp converts (16 / 8)
 constexpr int XFORM_THREADS = 32 * XFORM_WARPS;
 #ifndef NU_LEAF3_EPI_WARPS
 #define NU_LEAF3_EPI_WARPS 8
@@ -101,13 +106,19 @@ constexpr int BAR_BYTES = 256;
 constexpr int SMEM_BYTES = RS * TMA_BYTES + LS * XB_BYTES + EPI_BYTES + BAR_BYTES + 1024;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 
-__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* v) {
   asm volatile(
       "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
       "{%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, %16};" ::"r"(taddr),
       "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
       "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
       : "memory");
+}
+
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t* v) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(taddr),
+               "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
 }
 
 __device__ __forceinline__ void tmem_wait_st() {
@@ -379,11 +390,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     // ---------------------------------------------------- split (own half)
     const int tid = threadIdx.x - 64;
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
-    const int h = (warp - 2) >> 2;          // which 16 of the stage's 32 k
+    const int h = (warp - 2) >> 2;          // which XF_KPW of the stage's 32 k
     const int r = 32 * q + lane;            // A row of this CTA's half
     const uint32_t xform_leader0 = mapa(bar_xform, 0);
     const uint32_t rawfull_leader0 = mapa(bar_rawfull, 0);
-    const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + TM_XA + 16 * h;
+    const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + TM_XA + XF_KPW * h;
     uint32_t it = 0;
     long long w_full = 0, w_lem = 0;
     for (int t = cid; t < num_tiles; t += nclusters) {
@@ -399,15 +410,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         w_full += c1 - c0;
         w_lem += clock64() - c1;
         const uint32_t raw = smem_u32(raw_base + s * TMA_BYTES);
-        // A' row r, real k 16h..16h+15 -> TMEM columns 16h..16h+15 of slot j
+        // A' row r, real k XF_KPW*h .. +XF_KPW-1 -> the same TMEM columns of slot j
         {
           const uint32_t rowa = raw + r * 128;
           const int sw = r & 7;
-          uint32_t v[16];
+          uint32_t v[XF_KPW];
 #pragma unroll
-          for (int g = 0; g < 2; ++g) {
-            const uint4 x0 = lds128(rowa + (((4 * h + 2 * g) ^ sw) << 4));
-            const uint4 x1 = lds128(rowa + (((4 * h + 2 * g + 1) ^ sw) << 4));
+          for (int g = 0; g < XF_KPW / 8; ++g) {
+            const uint4 x0 = lds128(rowa + ((((XF_KPW / 4) * h + 2 * g) ^ sw) << 4));
+            const uint4 x1 = lds128(rowa + ((((XF_KPW / 4) * h + 2 * g + 1) ^ sw) << 4));
             const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
                                 __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
                                 __uint_as_float(x1.z), __uint_as_float(x1.w)};
@@ -423,7 +434,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
               v[8 * g + 4 + e] = pack_bf16(lo[2 * e], lo[2 * e + 1]);
             }
           }
-          tmem_st16(t_row + 32 * j, v);
+          if constexpr (XF_KPW == 16)
+            tmem_st16(t_row + 32 * j, v);
+          else
+            tmem_st8(t_row + 32 * j, v);
         }
         // B' (MN-major SW128 bf16, 64 virtual k x 128 n): as leaf_2sm.cu
         const uint32_t xb = smem_u32(xb_base + j * XB_BYTES);
