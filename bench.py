@@ -255,6 +255,10 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     m, n = r1 - r0, c1 - c0
     seed = int(name[-1])
     kc = args.k_chunk
+    if cfg["block"]:
+        # a fixed block (cfg1's 64 x 64 x 64) fixes the K-panel sequence: the in-HBM
+        # reference accumulates in the same chunks, so the two stay bitwise comparable
+        kc = cfg["block"][2]
 
     # --- the out-of-core tree: HOST root -> HBM (cap) -> SMEM/TMEM leaf.  N > 1:
     # the same tree on every rank (one HBM sibling per rank); this rank runs
