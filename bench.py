@@ -418,13 +418,14 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     leaf_ms = statistics.mean(per_hbm) / launches_per_step
     flops_per_launch = 2.0 * m * n * min(K, kc_eff)
     achieved = flops_per_launch / (leaf_ms * 1e-3) / 1e12
-    traffic = None
+    traffic = tensor_active = None
     tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
             tj = json.load(f)
         if (tj.get("M"), tj.get("N"), tj.get("launch_K")) == (m, n, min(K, kc_eff)):
             traffic = tj.get("dram_bytes")
+            tensor_active = tj.get("tensor_pipe_active_pct")
     clock_ghz = None
     result = None
     if rank == 0:
@@ -497,6 +498,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                          "kernel": LEAF_KERNELS.get(nu.lib().northup_debug_leaf_variant(), "?"),
                          "launch": [m, n, min(K, kc_eff)], "launches_per_step": launches_per_step,
                          "flops_per_launch": flops_per_launch, "ms_per_launch": round(leaf_ms, 3),
+                         "tensor_pipe_active_pct_ncu": tensor_active,
                          "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "
                                           "(profiles/leaf_traffic.json); algorithmic bytes per launch "
                                           f"= A/B panel + C read+write = {4 * (m + n) * min(K, kc_eff) + 8 * m * n:.3e}"},
