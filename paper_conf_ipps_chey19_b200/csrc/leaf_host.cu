@@ -66,6 +66,22 @@ __global__ void debug_spin_kernel(long long ns) {
   while (clock64() - t0 < cycles) __nanosleep(1000);
 }
 
+// Multi-process siblings (peer.cpp): store a generation into a flag word that
+// may live in another process's (and another GPU's) memory, after everything
+// earlier on the stream.  A one-thread kernel with a system-scope release store
+// works for any peer-mapped address, where a stream memory operation on peer
+// memory is not guaranteed to.
+__global__ void flag_store_kernel(uint32_t* addr, uint32_t v) {
+  __threadfence_system();
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(addr), "r"(v) : "memory");
+}
+
+int flag_store_launch(uint32_t* addr, uint32_t v, cudaStream_t s) {
+  flag_store_kernel<<<1, 1, 0, s>>>(addr, v);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : cuda_fail(e, "flag_store_kernel");
+}
+
 // Load every kernel the executor may launch on the current device (see
 // leaf_common.cuh preload_sm*): run before work that waits on other processes.
 void preload_kernels() {
@@ -76,6 +92,7 @@ void preload_kernels() {
   hotspot_preload();
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, debug_spin_kernel);
+  cudaFuncGetAttributes(&fa, flag_store_kernel);
 }
 
 int debug_spin(long long ns, cudaStream_t s) {

@@ -181,6 +181,8 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
 int debug_spin(long long ns, cudaStream_t s);
 // Force-load the kernels (lazy module loading) on the current device; hotspot.cu's part.
 void preload_kernels();
+// One-thread kernel: system-scope release store of v to addr (multi-process flag words).
+int flag_store_launch(uint32_t* addr, uint32_t v, cudaStream_t s);
 void hotspot_preload();
 int debug_slow_sibling(int* pct);
 inline long long debug_slow_ns(int pct, int64_t m, int64_t n, int64_t k) {

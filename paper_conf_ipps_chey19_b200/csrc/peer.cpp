@@ -13,14 +13,16 @@
 // [w] = sibling w's done word, [G + i] = op i.  A dependency of a local op on a
 // sibling's op i is a device-side wait on the LOCAL word
 // `cuStreamWaitValue32(flags[G + i] >= gen)`; after op i the producing sibling
-// stores `gen` into the flag words of every process that waits for it with
-// `cuStreamWriteValue32` on the IPC-mapped peer address (a fenced remote
-// store: the op's data is visible first).  Consumers only poll local memory.
+// stores `gen` into the flag words of every process that waits for it through
+// the IPC-mapped peer address (a one-thread kernel: __threadfence_system, then a
+// system-scope release store, so the op's data is visible first).  Consumers
+// only poll local memory.
 // No host thread blocks on a peer: the waits form a DAG because every
 // dependency points backwards in plan order and each stream is FIFO in plan
 // order.  At the end of a call every process stores its done word into all
 // siblings and waits for theirs (a device-side join), so no sibling can still
 // be pulling from an arena when northup_gemm returns.
+#include <stdlib.h>
 #include <string.h>
 
 #include "northup_internal.h"
@@ -90,6 +92,11 @@ int stream_wait_flag(cudaStream_t s, const uint32_t* addr, uint32_t gen) {
 }
 
 int stream_write_flag(cudaStream_t s, uint32_t* addr, uint32_t gen) {
+  // the store into a sibling's flag word: a one-thread kernel with a release store
+  // at system scope (valid for any peer-mapped address, including another GPU's
+  // memory over NVLink); NORTHUP_FLAG_MEMOP=1 uses cuStreamWriteValue32 instead
+  static const bool memop = getenv("NORTHUP_FLAG_MEMOP") != nullptr;
+  if (!memop) return flag_store_launch(addr, gen, s);
   int rc = load_mem_ops();
   if (rc) return rc;
   int r = g_write(s, reinterpret_cast<unsigned long long>(addr), gen, kWriteDefault);
