@@ -87,6 +87,16 @@ def test_host_root_gemm(M, N, K, G, cap, sched, kc, kind):
     assert st["num_gpus"] == G
 
 
+@pytest.mark.parametrize("M,N,K", [(1, 4097, 300), (4097, 1, 300), (257, 3, 1), (3, 5, 70000), (33, 2049, 7)])
+def test_host_root_skinny_and_ragged(M, N, K):
+    """Degenerate shapes through the HOST -> HBM tree (vectors, K = 1, a long K
+    against a tiny C, ragged edges in every dimension): exact on integer inputs,
+    within the bound on uniform ones."""
+    for kind in ("int", "uniform"):
+        C, a, b, st = run_host(M, N, K, kind=kind)
+        check(C, a, b, kind)
+
+
 def test_zero_k_and_empty():
     C, a, b, st = run_host(7, 9, 0)
     assert (C == 0).all()
