@@ -47,6 +47,20 @@ def sampled_check(a, b, c, seed=0, n=65536):
     return max(worst, e_rows, e_cols)
 
 
+def freivalds_uniform(a, b, c, seed, reps=2):
+    """S§8(c): every row of C at once — for random +-1 vectors r, the necessary
+    condition |((C - C_ref) r)_i| <= 1e-5 ||A_i,:||_2 sum_j ||B_:,j||_2 (returns
+    the worst ratio; C_ref r is computed as A (B r) in fp64)."""
+    rng = np.random.default_rng(seed + 100)
+    rn, cn = oracle.row_norms(a), oracle.col_norms(b)
+    worst = 0.0
+    for _ in range(reps):
+        r = np.where(rng.random(b.shape[1]) < 0.5, -1.0, 1.0)
+        e, _, _ = oracle.freivalds(a, b, c, r, rn, cn)
+        worst = max(worst, e)
+    return worst
+
+
 def run_config(M, N, K, cap, kind, seed):
     t, _ = nu.host_tree(1, cap)
     t.finalize()
@@ -82,6 +96,7 @@ def test_large_config_sampled_and_freivalds(name, M, N, K, cap):
     t, a, b, c, st = run_config(M, N, K, cap, "uniform", seed)
     assert st["hbm_peak_bytes"] <= cap
     assert sampled_check(a, b, c, seed) <= TOL
+    assert freivalds_uniform(a, b, c, seed) <= TOL
     t.destroy()
     # integer inputs: exact result -> Freivalds with +-1 vectors must match exactly
     t, a, b, c, st = run_config(M, N, K, cap, "int", seed)
@@ -100,4 +115,5 @@ def test_cfg4_one_gpu_sampled():
     t, a, b, c, st = run_config(M, N, K, 8 * GiB, "uniform", 4)
     assert st["bm"] * st["bn"] < M * N and st["hbm_peak_bytes"] <= 8 * GiB
     assert sampled_check(a, b, c, 4) <= TOL
+    assert freivalds_uniform(a, b, c, 4) <= TOL
     t.destroy()
