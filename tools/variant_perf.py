@@ -6,19 +6,20 @@ import torch
 import paper_conf_ipps_chey19_b200 as nu
 
 dev = torch.device("cuda:0")
-res = {"variant": os.environ.get("NORTHUP_LEAF", "default")}
+KC = int(os.environ.get("KC", "2048"))
+res = {"variant": os.environ.get("NORTHUP_LEAF", "default"), "k_chunk": KC}
 for SZ in [int(s) for s in os.environ.get("SZS", "8192,16384").split(",")]:
     A = torch.rand((SZ, SZ), device=dev) * 2 - 1
     B = torch.rand((SZ, SZ), device=dev) * 2 - 1
     C = torch.empty((SZ, SZ), device=dev)
     it = 10 if SZ <= 16384 else 3
     for _ in range(2):
-        nu.leaf_gemm(A, B, C, k_chunk=2048)
+        nu.leaf_gemm(A, B, C, k_chunk=KC)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
     for _ in range(it):
-        nu.leaf_gemm(A, B, C, k_chunk=2048)
+        nu.leaf_gemm(A, B, C, k_chunk=KC)
     e1.record()
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / it
