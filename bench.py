@@ -730,6 +730,9 @@ def main():
         return
 
     if world > 1:
+        # a sibling process that fails leaves its peers' streams waiting on its flag
+        # words; end the run after 3 minutes instead of the library's 10
+        os.environ.setdefault("NORTHUP_PEER_TIMEOUT_S", "180")
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
