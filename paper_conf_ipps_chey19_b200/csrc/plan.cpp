@@ -704,7 +704,8 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
                     int64_t a_panel_k, northup_stats* st) {
   const int G = static_cast<int>(hbm.size());
   const int io = G;   // the I/O pseudo-worker
-  const int64_t bk = a_panel_k > 0 ? a_panel_k : kc;
+  // a K shorter than the panel is one panel of width K (the file layout agrees: R15)
+  const int64_t bk = std::min<int64_t>(a_panel_k > 0 ? a_panel_k : kc, std::max<int64_t>(K, 1));
   // per-worker regions and one common C-block shape that fits every HBM node
   std::vector<int64_t> r0(G), r1(G), c0(G), c1(G);
   int64_t mmax = 0, nmax = 0;
@@ -828,7 +829,7 @@ int build_file_direct(Builder& B, const northup_tree_s* t, const std::vector<int
                       northup_stats* st) {
   const int G = static_cast<int>(hbm.size());
   const int io = G;   // the I/O pseudo-worker
-  const int64_t bk = a_panel_k > 0 ? a_panel_k : kc;
+  const int64_t bk = std::min<int64_t>(a_panel_k > 0 ? a_panel_k : kc, std::max<int64_t>(K, 1));
   std::vector<int64_t> r0(G), r1(G), c0(G), c1(G);
   int64_t mmax = 0, nmax = 0;
   uint64_t cap = uint64_t(1) << 62;
