@@ -168,6 +168,9 @@ __device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const CUtensorMap
 #ifndef NU_LEAF3_PF
 #define NU_LEAF3_PF 0
 #endif
+#ifndef NU_LEAF3_NOSPLIT
+#define NU_LEAF3_NOSPLIT 0
+#endif
 __device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, int c1) {
   asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
                    reinterpret_cast<uint64_t>(map)),
@@ -410,6 +413,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         w_full += c1 - c0;
         w_lem += clock64() - c1;
         const uint32_t raw = smem_u32(raw_base + s * TMA_BYTES);
+#if !NU_LEAF3_NOSPLIT   // timing experiment only: skip the conversion (wrong results)
         // A' row r, real k XF_KPW*h .. +XF_KPW-1 -> the same TMEM columns of slot j
         {
           const uint32_t rowa = raw + r * 128;
@@ -470,6 +474,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
                  make_uint4(pack_bf16(hi[0], hi[1]), pack_bf16(hi[2], hi[3]),
                             pack_bf16(hi[4], hi[5]), pack_bf16(hi[6], hi[7])));
         }
+#endif
         tmem_wait_st();
         fence_proxy_async_smem();
         tc_fence_before();
