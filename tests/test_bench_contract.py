@@ -49,3 +49,18 @@ def test_ours_quick_json_line():
     assert d["parity"]["oracle_ok"] and d["cpu_baseline"]["kind"] == "oracle"
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
     assert d["cfg2_in_hbm_tflops"] > 0 and "slowdown_pct_vs_cfg2_in_hbm" in d
+
+
+def test_ooc_roofline_terms():
+    """S§8(d): R = min(P_eff, BW_h2d * I_h2d, BW_d2h * I_d2h), I_e = flops / bytes on edge e."""
+    sys.path.insert(0, ROOT)
+    import bench
+    pcie = {"bidir_h2d_gbs": 50.0, "bidir_d2h_gbs": 51.0}
+    flops = 2.0 * 32768 ** 3
+    r = bench.ooc_roofline(flops, 8 << 30, 4 << 30, 344.0, pcie)
+    assert r["intensity_flop_per_byte"] == {"h2d": 8192.0, "d2h": 16384.0}
+    assert abs(r["terms"]["pcie_h2d"] - 50e9 * 8192 / 1e12) < 1e-3
+    assert r["bound"] == "tensor" and r["peak"] == 344.0
+    r5 = bench.ooc_roofline(2.0 * 1048576 * 4096 * 4096, 16 << 30, 16 << 30, 344.0, pcie)
+    assert r5["bound"] == "pcie_h2d" and abs(r5["peak"] - 50e9 * 2048 / 1e12) < 1e-2
+    assert bench.ooc_roofline(1e12, 0, 0, 344.0, pcie)["bound"] == "tensor"   # in-HBM: no edges
