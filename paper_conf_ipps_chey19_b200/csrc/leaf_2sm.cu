@@ -67,9 +67,51 @@ constexpr int BAR_BYTES = 256;
 constexpr int SMEM_BYTES = (RS + LS) * STAGE_BYTES + BAR_BYTES + 1024;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 
+// NU_LEAF2_PRESPLIT (build-time experiment, npass 2 only): a pre-pass writes the
+// bf16 operands A' (M x 2K8, per k8 group [hi of 8 k | lo of 8 k]) and B'
+// (2K8 x N, per k8 group [lo rows; hi rows]) to HBM once, and the producer
+// TMA-loads them straight into the lo ring in the layouts the split warps
+// would have written (SW128 K-major A', SW128 MN-major B'); the split warps
+// only forward the barriers.
+#ifndef NU_LEAF2_PRESPLIT
+#define NU_LEAF2_PRESPLIT 0
+#endif
+__global__ void presplit_a_kernel(const float* __restrict__ A, int64_t lda, int M, int K, int K8,
+                                  __nv_bfloat16* __restrict__ Ap) {
+  const int64_t n = static_cast<int64_t>(M) * K8;
+  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < n;
+       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    const int64_t i = idx / K8;
+    const int k = static_cast<int>(idx - i * K8);
+    const float f = k < K ? A[i * lda + k] : 0.0f;
+    const float h = trunc13(f);
+    const int64_t o = i * 2 * K8 + 16 * (k >> 3) + (k & 7);
+    Ap[o] = __float2bfloat16_rn(h);
+    Ap[o + 8] = __float2bfloat16_rn(f - h);
+  }
+}
+__global__ void presplit_b_kernel(const float* __restrict__ B, int64_t ldb, int K, int N, int K8,
+                                  __nv_bfloat16* __restrict__ Bp) {
+  const int64_t n = static_cast<int64_t>(K8) * N;
+  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < n;
+       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    const int k = static_cast<int>(idx / N);
+    const int64_t j = idx - static_cast<int64_t>(k) * N;
+    const float f = k < K ? B[static_cast<int64_t>(k) * ldb + j] : 0.0f;
+    const float h = trunc13(f);
+    const int64_t v = 16 * (k >> 3) + (k & 7);
+    Bp[v * N + j] = __float2bfloat16_rn(f - h);
+    Bp[(v + 8) * N + j] = __float2bfloat16_rn(h);
+  }
+}
+
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     leaf_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tmA,
-                         const __grid_constant__ CUtensorMap tmB, const Params p) {
+                         const __grid_constant__ CUtensorMap tmB, const Params p
+#if NU_LEAF2_PRESPLIT
+                         , const __grid_constant__ CUtensorMap tmAp, const __grid_constant__ CUtensorMap tmBp
+#endif
+                         ) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -83,7 +125,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   const uint32_t bar_tfull = bar_lempty + 8 * LS;
   const uint32_t bar_tempty = bar_tfull + 16;
   const uint32_t bar_rawfull = bar_tempty + 16;      // [RS] leader: both CTAs' raw tiles landed
+#if NU_LEAF2_PRESPLIT
+  const uint32_t bar_lofull = bar_rawfull + 8 * RS;  // [LS] the pre-split A'/B' tiles landed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (3 * RS + 3 * LS + 4));
+#else
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 8 * (3 * RS + 2 * LS + 4));
+#endif
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -101,6 +148,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     for (int j = 0; j < LS; ++j) {
       mbar_init(bar_xform + 8 * j, 2);   // one elected arrive per CTA
       mbar_init(bar_lempty + 8 * j, 1);
+#if NU_LEAF2_PRESPLIT
+      mbar_init(bar_lofull + 8 * j, 1);
+#endif
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(bar_tfull + 8 * a, 1);
@@ -146,6 +196,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
 #pragma unroll
           for (int c = 0; c < BN_CTA / B_CHUNK; ++c)
             tma_load_2d(sb + c * B_CHUNK_BYTES, &tmB, full, col0 + c * B_CHUNK, kb * BK);
+#if NU_LEAF2_PRESPLIT
+          {
+            const uint32_t j = it % LS, juse = it / LS;
+            mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
+            const uint32_t lf = bar_lofull + 8 * j;
+            mbar_arrive_expect_tx(lf, STAGE_BYTES);
+            const uint32_t sl = smem_u32(lo_base + j * STAGE_BYTES);
+            tma_load_2d(sl, &tmAp, lf, kb * 2 * BK, row0);                 // A': 64 virtual k x 128 rows
+            tma_load_2d(sl + XA_BYTES, &tmBp, lf, col0, kb * 2 * BK);      // B': 64 n x 64 virtual k
+            tma_load_2d(sl + XA_BYTES + 8192, &tmBp, lf, col0 + 64, kb * 2 * BK);
+          }
+#endif
         }
       }
     }
@@ -245,6 +307,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         long long c0 = clock64();
         mbar_wait(bar_full + 8 * s, use & 1);
         if (p.npass == 2 && tid == 0) mbar_arrive_cluster(rawfull_leader0 + 8 * s);
+#if NU_LEAF2_PRESPLIT
+        mbar_wait(bar_lofull + 8 * j, juse & 1);
+        if (tid == 0) mbar_arrive_cluster(xform_leader0 + 8 * j);
+        w_full += clock64() - c0;
+        continue;
+#endif
         long long c1 = clock64();
         mbar_wait(bar_lempty + 8 * j, (juse & 1) ^ 1);
         w_full += c1 - c0;
@@ -443,7 +511,29 @@ int launch_sm2(LaunchArgs& a) {
   const int tiles = p.tiles_m * p.tiles_n;
   const int pairs = a.sms / 2;
   const int grid = 2 * (tiles < pairs ? tiles : pairs);
+#if NU_LEAF2_PRESPLIT
+  // experiment: one grow-only scratch per process, pre-pass on the same stream
+  static char* scratch = nullptr;
+  static size_t scratch_bytes = 0;
+  const int K8 = (p.K + 7) / 8 * 8;
+  const size_t need = 2ull * 2 * K8 * (static_cast<size_t>(p.M) + p.N) + 1024;
+  if (need > scratch_bytes) {
+    cudaStreamSynchronize(a.stream);
+    if (scratch) cudaFree(scratch);
+    if (cudaMalloc(&scratch, need) != cudaSuccess) return fail(NU_ENOMEM, "presplit scratch");
+    scratch_bytes = need;
+  }
+  __nv_bfloat16* Ap = reinterpret_cast<__nv_bfloat16*>(scratch);
+  __nv_bfloat16* Bp = Ap + static_cast<size_t>(p.M) * 2 * K8;
+  presplit_a_kernel<<<1184, 256, 0, a.stream>>>(a.A, a.lda, p.M, p.K, K8, Ap);
+  presplit_b_kernel<<<1184, 256, 0, a.stream>>>(a.B, a.ldb, p.K, p.N, K8, Bp);
+  CUtensorMap tmAp, tmBp;
+  if ((rc = encode_2d_bf16(&tmAp, Ap, 2 * K8, p.M, 2 * K8, 64, BM_CTA))) return rc;
+  if ((rc = encode_2d_bf16(&tmBp, Bp, p.N, 2 * K8, p.N, 64, 2 * BK))) return rc;
+  leaf_gemm_2sm_kernel<<<grid, NUM_THREADS, SMEM_BYTES, a.stream>>>(tmA, tmB, p, tmAp, tmBp);
+#else
   leaf_gemm_2sm_kernel<<<grid, NUM_THREADS, SMEM_BYTES, a.stream>>>(tmA, tmB, p);
+#endif
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "leaf (2sm) launch: %s", cudaGetErrorString(e));
 }

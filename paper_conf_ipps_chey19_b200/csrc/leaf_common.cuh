@@ -193,6 +193,8 @@ struct LaunchArgs {
 int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t outer,
               uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer,
               CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B);
+int encode_2d_bf16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                   uint32_t box_inner, uint32_t box_outer);
 int launch_sm1(LaunchArgs& a);   // v0: 1-CTA 128 x 256 tile
 int launch_sm2(LaunchArgs& a);   // v1: CTA pair (cta_group::2) 256 x 256 tile, TMA-fed
 int launch_sm3(LaunchArgs& a);   // v2: CTA pair, split warps load global memory directly

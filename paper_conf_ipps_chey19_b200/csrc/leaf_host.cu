@@ -47,6 +47,21 @@ int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t oute
   return 0;
 }
 
+// bf16 2-D map with 128-B swizzle (the pre-split operands of NU_LEAF2_PRESPLIT).
+int encode_2d_bf16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                   uint32_t box_inner, uint32_t box_outer) {
+  int rc = get_encode();
+  if (rc) return rc;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld_elems * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
+                        estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? 0 : fail(NU_EINVAL, "cuTensorMapEncodeTiled (bf16) failed (%d)", (int)r);
+}
+
 }  // namespace leaf
 
 int default_leaf_variant() {
