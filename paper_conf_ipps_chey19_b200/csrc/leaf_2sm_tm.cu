@@ -102,6 +102,14 @@ constexpr int BOX_BYTES = 32 * 32 * 4;             // 32 rows x 32 cols fp32, SW
 constexpr int EPI_BYTES = EPI_WARPS * EPI_BUFS * BOX_BYTES;
 constexpr int TMEM_COLS = 512;
 constexpr int TM_XA = 256;                         // first A' column
+// NU_LEAF3_AHI_TMEM (build-time): the split also stores the raw A tile (tf32 hi is the
+// hardware's truncation of it) into TMEM, and the hi.hi MMA reads A from TMEM: the MMA
+// no longer reads A from shared memory (-16 KiB of shared-memory traffic per stage).
+#ifndef NU_LEAF3_AHI_TMEM
+#define NU_LEAF3_AHI_TMEM 0
+#endif
+constexpr int TM_AH = TM_XA + 32 * NU_LEAF3_LS;     // first A_hi column (AHI_TMEM)
+static_assert(!NU_LEAF3_AHI_TMEM || TM_AH + 32 * NU_LEAF3_LS <= 512, "TMEM columns");
 constexpr int BAR_BYTES = 256;
 constexpr int SMEM_BYTES = RS * TMA_BYTES + LS * XB_BYTES + EPI_BYTES + BAR_BYTES + 1024;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
@@ -123,6 +131,17 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t* v) {
 
 __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+
+// D[tmem] (+)= A[tmem] . B[smem], kind::tf32, pair MMA.
+__device__ __forceinline__ void umma_tf32_2sm_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db,
+                                                 uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accum)
+      : "memory");
 }
 
 // D[tmem] (+)= A[tmem] . B[smem], kind::f16 (bf16 in, fp32 accumulate), pair MMA.
@@ -358,6 +377,20 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             const uint32_t b_hi = a_hi + A_BYTES;
             const uint32_t b_x = smem_u32(xb_base + j * XB_BYTES);
             const uint32_t a_x = tmem_base + TM_XA + 32 * j;
+#if NU_LEAF3_AHI_TMEM
+            (void)a_hi;
+            (void)suse;
+            c0 = clock64();
+            mbar_wait_cluster(bar_xform + 8 * j, juse & 1);   // both splits: raw landed, A_hi in TMEM
+            w_xf += clock64() - c0;
+            tc_fence_after();
+            const uint32_t a_h = tmem_base + TM_AH + 32 * j;
+#pragma unroll
+            for (int k = 0; k < BK / UMMA_K; ++k)
+              umma_tf32_2sm_ts(tmem_base, a_h + 8 * k,
+                               umma_desc(b_hi + k * 1024, B_CHUNK_BYTES, 512, LAYOUT_SW128_BASE32B), idesc,
+                               (kb == kb0 && k == 0) ? 0u : 1u);
+#else
             c0 = clock64();
             mbar_wait_cluster(bar_rawfull + 8 * s, suse & 1);
             w_xf += clock64() - c0;
@@ -371,6 +404,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             mbar_wait_cluster(bar_xform + 8 * j, juse & 1);
             w_xf += clock64() - c0;
             tc_fence_after();
+#endif
 #pragma unroll
             for (int k = 0; k < BK / UMMA_K; ++k)
               umma_bf16_2sm_ts(tmem_base, a_x + 8 * k, umma_desc(b_x + k * 2048, 8192, 1024),
@@ -398,6 +432,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const uint32_t xform_leader0 = mapa(bar_xform, 0);
     const uint32_t rawfull_leader0 = mapa(bar_rawfull, 0);
     const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + TM_XA + XF_KPW * h;
+#if NU_LEAF3_AHI_TMEM
+    const uint32_t t_rowh = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + TM_AH + XF_KPW * h;
+#endif
     uint32_t it = 0;
     long long w_full = 0, w_lem = 0;
     for (int t = cid; t < num_tiles; t += nclusters) {
@@ -419,10 +456,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
           const uint32_t rowa = raw + r * 128;
           const int sw = r & 7;
           uint32_t v[XF_KPW];
+#if NU_LEAF3_AHI_TMEM
+          uint32_t vr[XF_KPW];
+#endif
 #pragma unroll
           for (int g = 0; g < XF_KPW / 8; ++g) {
             const uint4 x0 = lds128(rowa + ((((XF_KPW / 4) * h + 2 * g) ^ sw) << 4));
             const uint4 x1 = lds128(rowa + ((((XF_KPW / 4) * h + 2 * g + 1) ^ sw) << 4));
+#if NU_LEAF3_AHI_TMEM
+            vr[8 * g + 0] = x0.x, vr[8 * g + 1] = x0.y, vr[8 * g + 2] = x0.z, vr[8 * g + 3] = x0.w;
+            vr[8 * g + 4] = x1.x, vr[8 * g + 5] = x1.y, vr[8 * g + 6] = x1.z, vr[8 * g + 7] = x1.w;
+#endif
             const float f[8] = {__uint_as_float(x0.x), __uint_as_float(x0.y), __uint_as_float(x0.z),
                                 __uint_as_float(x0.w), __uint_as_float(x1.x), __uint_as_float(x1.y),
                                 __uint_as_float(x1.z), __uint_as_float(x1.w)};
@@ -442,6 +486,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
             tmem_st16(t_row + 32 * j, v);
           else
             tmem_st8(t_row + 32 * j, v);
+#if NU_LEAF3_AHI_TMEM
+          if constexpr (XF_KPW == 16)
+            tmem_st16(t_rowh + 32 * j, vr);
+          else
+            tmem_st8(t_rowh + 32 * j, vr);
+#endif
         }
         // B' (MN-major SW128 bf16, 64 virtual k x 128 n): as leaf_2sm.cu
         const uint32_t xb = smem_u32(xb_base + j * XB_BYTES);
