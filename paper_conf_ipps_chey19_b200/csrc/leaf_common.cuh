@@ -3,6 +3,7 @@
 #pragma once
 
 #include <cuda.h>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -206,6 +207,31 @@ void preload_sm2();
 void preload_sm3();
 void preload_sm4();
 bool launch_sm4_ok(const LaunchArgs& a);
+
+// cuTensorMapEncodeTiled, general rank (strides in bytes for dims 1..rank-1).
+int encode_tiled(CUtensorMap* map, CUtensorMapDataType type, int rank, const void* base,
+                 const cuuint64_t* dims, const cuuint64_t* strides, const cuuint32_t* box,
+                 CUtensorMapSwizzle swz);
+
+// A split operand (split.cu, R22): `p` holds the hi/lo fp16 pairs in
+// the layout of a row-major fp32 matrix with leading dimension `ld` (floats),
+// `e` one exponent per row (A) or column (B) of the panel.
+struct SplitOperand {
+  const float* p;
+  int64_t ld;
+  const int* e;
+};
+int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64_t ldd, int* ea, int sms,
+                   cudaStream_t s);
+int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64_t ldd, int* eb,
+                   unsigned* bmax, cudaStream_t s);
+int64_t split_b_max_n();
+void preload_split();
+void preload_x3();
+// GEMM of one K panel (kl <= the panel) on split operands.
+int x3_gemm(const SplitOperand& A, const SplitOperand& B, float* C, int64_t ldc, int m, int n, int kl,
+            int accumulate, int kb_per_chunk, int npass, int band, int sms, int dev, float* dbg,
+            cudaStream_t stream);
 
 }  // namespace leaf
 }  // namespace nu

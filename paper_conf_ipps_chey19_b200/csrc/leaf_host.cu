@@ -8,6 +8,7 @@
 #include <stdlib.h>
 
 #include <atomic>
+#include <mutex>
 
 #include "leaf_common.cuh"
 #include "northup_internal.h"
@@ -47,6 +48,20 @@ int encode_2d(CUtensorMap* map, const float* base, uint64_t inner, uint64_t oute
   return 0;
 }
 
+int encode_tiled(CUtensorMap* map, CUtensorMapDataType type, int rank, const void* base, const cuuint64_t* dims,
+                 const cuuint64_t* strides, const cuuint32_t* box, CUtensorMapSwizzle swz) {
+  int rc = get_encode();
+  if (rc) return rc;
+  cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+  CUresult r = g_encode(map, type, rank, const_cast<void*>(base), dims, strides, box, estr,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    return fail(NU_EINVAL, "cuTensorMapEncodeTiled (rank %d) failed (%d): base=%p dim0=%llu", rank, (int)r, base,
+                (unsigned long long)dims[0]);
+  return 0;
+}
+
 // bf16 2-D map with 128-B swizzle (the pre-split operands of NU_LEAF2_PRESPLIT).
 int encode_2d_bf16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
                    uint32_t box_inner, uint32_t box_outer) {
@@ -68,7 +83,7 @@ int default_leaf_variant() {
   static int env_variant = -1;
   if (env_variant < 0) {
     const char* v = getenv("NORTHUP_LEAF");
-    env_variant = (v && v[0] >= '1' && v[0] <= '4') ? v[0] - '0' : kDefaultLeafVariant;
+    env_variant = (v && v[0] >= '1' && v[0] <= '5') ? v[0] - '0' : kDefaultLeafVariant;
   }
   return env_variant;
 }
@@ -104,6 +119,7 @@ void preload_kernels() {
   leaf::preload_sm2();
   leaf::preload_sm3();
   leaf::preload_sm4();
+  leaf::preload_x3();
   hotspot_preload();
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, debug_spin_kernel);
@@ -127,12 +143,146 @@ bool leaf_tma_legal(const void* p, int64_t ld) {
   return (reinterpret_cast<uintptr_t>(p) % 16 == 0) && (ld % 4 == 0) && ld > 0;
 }
 
-// variant: 0 = default (env NORTHUP_LEAF=1..4 may override), 1 = v0 (1 CTA), 2 = v1.2 (pair),
+// ------------------------------------------------------------------ the x3 leaf
+// Stream-ordered scratch for leaf calls that bring none (northup_leaf_gemm):
+// a private pool per device that keeps its memory (no release at syncs).
+static std::mutex g_pool_mu;
+static cudaMemPool_t g_pool[kMaxDevices];
+
+static int scratch_alloc(int dev, uint64_t bytes, cudaStream_t s, char** out) {
+  {
+    std::lock_guard<std::mutex> g(g_pool_mu);
+    if (!g_pool[dev]) {
+      cudaMemPoolProps pr = {};
+      pr.allocType = cudaMemAllocationTypePinned;
+      pr.handleTypes = cudaMemHandleTypeNone;
+      pr.location.type = cudaMemLocationTypeDevice;
+      pr.location.id = dev;
+      cudaError_t e = cudaMemPoolCreate(&g_pool[dev], &pr);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemPoolCreate (leaf scratch)");
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(g_pool[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  cudaError_t e = cudaMallocFromPoolAsync(reinterpret_cast<void**>(out), bytes, g_pool[dev], s);
+  return e == cudaSuccess ? 0 : fail(NU_ENOMEM, "leaf scratch (%llu B): %s", (unsigned long long)bytes,
+                                     cudaGetErrorString(e));
+}
+
+static inline uint64_t al256(uint64_t b) { return (b + 255) / 256 * 256; }
+
+uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit) {
+  const uint64_t Kp = static_cast<uint64_t>((panel + 31) / 32 * 32);
+  uint64_t s = al256(4ull * m * Kp) + al256(4ull * m);
+  if (!b_presplit) s += al256(4ull * Kp * static_cast<uint64_t>((n + 31) / 32 * 32)) + 2 * al256(4ull * n);
+  return s;
+}
+
+int64_t leaf_acc_chunk() {
+  static int64_t v = -1;
+  if (v < 0) {
+    const char* e = getenv("NORTHUP_ACC_CHUNK");
+    v = (e && atoll(e) >= 32) ? atoll(e) / 32 * 32 : kAccChunk;
+  }
+  return v;
+}
+
+static int sms_of(int dev) {
+  static std::atomic<int> num_sms[kMaxDevices];
+  if (num_sms[dev].load() == 0) {
+    int n = 0;
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    num_sms[dev].store(n > 0 ? n : 148);
+  }
+  return num_sms[dev].load();
+}
+
+int leaf_run(const LeafCall& c) {
+  using namespace leaf;
+  const int64_t M = c.M, N = c.N, K = c.K;
+  if (M < 0 || N < 0 || K < 0) return fail(NU_EINVAL, "negative dimension");
+  if (M == 0 || N == 0) return 0;
+  if (K == 0) {
+    if (c.accumulate) return 0;
+    cudaError_t e = cudaMemset2DAsync(c.C, c.ldc * 4, 0, N * 4, M, c.stream);
+    return e == cudaSuccess ? 0 : fail(NU_ECUDA, "memset: %s", cudaGetErrorString(e));
+  }
+  if (M > INT32_MAX || N > INT32_MAX || K > INT32_MAX) return fail(NU_EINVAL, "dimension exceeds int32");
+  if (c.lda < K || c.ldb < N || c.ldc < N) return fail(NU_EINVAL, "leading dimension too small");
+  if (!c.A || !c.B || !c.C) return fail(NU_EINVAL, "null operand");
+  if (c.eb_presplit && (c.ldb % 8 || reinterpret_cast<uintptr_t>(c.B) % 16))
+    return fail(NU_EINVAL, "pre-split B needs a 16-B aligned base and ldb %% 8 == 0");
+  if (!c.eb_presplit && N > split_b_max_n())
+    return fail(NU_EINVAL, "leaf N = %lld above %lld", (long long)N, (long long)split_b_max_n());
+  int64_t panel = c.panel > 0 ? c.panel : kDefaultKChunk;
+  panel = (panel + 31) / 32 * 32;
+  const int npass = (c.npass == 1 || c.npass == 4) ? c.npass : 3;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= kMaxDevices) return fail(NU_EINVAL, "device ordinal out of range");
+  const int sms = sms_of(dev);
+  static int env_band = -1;
+  if (env_band < 0) {
+    const char* v = getenv("NORTHUP_RASTER_BAND");
+    env_band = (v && atoi(v) > 0) ? atoi(v) : kRasterBand;
+  }
+  const int64_t pk = std::min<int64_t>(panel, (K + 31) / 32 * 32);
+  const uint64_t need = leaf_scratch_bytes(M, N, pk, c.eb_presplit != nullptr);
+  char* scratch = c.scratch;
+  bool pooled = false;
+  if (!scratch) {
+    int rc = scratch_alloc(dev, need, c.stream, &scratch);
+    if (rc) return rc;
+    pooled = true;
+  } else if (c.scratch_bytes < need) {
+    return fail(NU_ENOMEM, "leaf scratch %llu B < %llu B", (unsigned long long)c.scratch_bytes,
+                (unsigned long long)need);
+  }
+  const int64_t Kp = (pk + 31) / 32 * 32;
+  float* Ap = reinterpret_cast<float*>(scratch);
+  int* ea = reinterpret_cast<int*>(scratch + al256(4ull * M * Kp));
+  char* bpart = scratch + al256(4ull * M * Kp) + al256(4ull * M);
+  const int64_t ldq = (N + 31) / 32 * 32;
+  float* Bp = reinterpret_cast<float*>(bpart);
+  int* eb = reinterpret_cast<int*>(bpart + al256(4ull * Kp * ldq));
+  unsigned* bmax = reinterpret_cast<unsigned*>(bpart + al256(4ull * Kp * ldq) + al256(4ull * N));
+  const int64_t acc = std::min<int64_t>(leaf_acc_chunk(), Kp);
+  int rc = 0;
+  for (int64_t k0 = 0, p = 0; k0 < K && rc == 0; k0 += panel, ++p) {
+    const int kl = static_cast<int>(std::min(panel, K - k0));
+    rc = split_a_launch(c.A + k0, c.lda, static_cast<int>(M), kl, Ap, Kp, ea, sms, c.stream);
+    SplitOperand sa{Ap, Kp, ea}, sb{};
+    if (rc == 0) {
+      if (c.eb_presplit) {
+        sb = SplitOperand{c.B + k0 * c.ldb, c.ldb, c.eb_presplit + p * c.eb_stride};
+      } else {
+        rc = split_b_launch(c.B + k0 * c.ldb, c.ldb, kl, static_cast<int>(N), Bp, ldq, eb, bmax, c.stream);
+        sb = SplitOperand{Bp, ldq, eb};
+      }
+    }
+    if (rc == 0)
+      rc = x3_gemm(sa, sb, c.C, c.ldc, static_cast<int>(M), static_cast<int>(N), kl,
+                   (k0 > 0 || c.accumulate) ? 1 : 0, static_cast<int>((acc + 31) / 32), npass, env_band, sms, dev,
+                   c.dbg, c.stream);
+  }
+  if (pooled) cudaFreeAsync(scratch, c.stream);
+  return rc;
+}
+
+// variant: 0 = default (env NORTHUP_LEAF=1..5 may override), 1 = v0 (1 CTA), 2 = v1.2 (pair),
 // 3 = v2 (pair, LDG-fed), 4 = v3 (pair, A' in TMEM).
 int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                          int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                          int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream) {
   using namespace leaf;
+  if (variant == 0) variant = default_leaf_variant();
+  if (variant == 5) {
+    if (b_kmajor) return fail(NU_EINVAL, "the leaf takes B row-major (K x N)");
+    LeafCall c{};
+    c.A = A, c.lda = lda, c.B = B, c.ldb = ldb, c.C = C, c.ldc = ldc, c.M = M, c.N = N, c.K = K;
+    c.accumulate = accumulate, c.panel = kc, c.npass = npass, c.dbg = dbg, c.stream = stream;
+    return leaf_run(c);
+  }
   if (M < 0 || N < 0 || K < 0) return fail(NU_EINVAL, "negative dimension");
   if (M == 0 || N == 0) return 0;
   if (K == 0) {

@@ -13,9 +13,10 @@
 namespace nu {
 
 constexpr int kMaxDevices = 64;
-constexpr int64_t kDefaultKChunk = 2048;   // TMEM accumulation length (R20)
-constexpr int kDefaultNpass = 2;            // 2 = TF32 hi.hi + bf16 cross terms (R21), 3 = 3xTF32
-constexpr int kDefaultLeafVariant = 4;      // 1 = v0 1-CTA, 2 = v1.2 TMA-fed pair, 3 = v2 LDG-fed pair, 4 = v3 A' in TMEM
+constexpr int64_t kDefaultKChunk = 2048;   // K panel of one leaf launch / split (R20, R22)
+constexpr int64_t kAccChunk = 256;         // TMEM accumulation length inside a panel (R20)
+constexpr int kDefaultNpass = 3;            // 3 = fp16 hi.hi + hi.lo + lo.hi on the scaled split (R22)
+constexpr int kDefaultLeafVariant = 5;      // 5 = x3 (split operands); 1..4 = round-1 kernels (comparison)
 constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
 constexpr int kRasterBand = 16;            // n-blocks per raster band in the leaf
 constexpr int64_t kPanelChunks = 1;        // leaf K-panel launches, in k_chunks (0 = one launch)
@@ -155,6 +156,28 @@ int region_of(int G, int64_t M, int64_t N, int r, int64_t* r0, int64_t* r1, int6
 int validate_tree(const northup_tree_s* t);
 
 // --------------------------------------------------------------- leaf
+// One leaf call (leaf_host.cu): C (+)= A.B over K, one split + GEMM per K panel.
+struct LeafCall {
+  const float* A;
+  int64_t lda;
+  const float* B;          // raw fp32 (eb_presplit == NULL) or split in place (split.cu layout)
+  int64_t ldb;
+  const int* eb_presplit;  // B's column exponents, [panel p][eb_stride]
+  int64_t eb_stride;
+  float* C;
+  int64_t ldc;
+  int64_t M, N, K;
+  int accumulate;
+  int64_t panel;           // K per launch (0 = kDefaultKChunk)
+  int npass;
+  char* scratch;           // NULL: stream-ordered from the leaf's pool
+  uint64_t scratch_bytes;
+  float* dbg;
+  cudaStream_t stream;
+};
+int leaf_run(const LeafCall& c);
+uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit);
+int64_t leaf_acc_chunk();
 bool leaf_tma_legal(const void* p, int64_t ld);
 int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                      int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,

@@ -1,0 +1,163 @@
+// Operand split of the leaf (R22): every fp32 operand x of one K
+// panel is written as
+//
+//     x = 2^e (hi + lo),   hi = fp16_rn(x 2^-e),   lo = fp16_rn(x 2^-e - hi)
+//
+// with one power-of-two exponent e per ROW of A and per COLUMN of B (over the
+// panel's K range), chosen so that the row's (column's) largest |x| 2^-e lies
+// in [2^14, 2^15): every hi is a normal fp16 (11 significant bits, so any
+// fp16 x fp16 tensor-core product is exact) for elements down to 2^-28 of the
+// row maximum, and x 2^-e - hi is exact in fp32.  The leaf computes
+// hi_a hi_b + hi_a lo_b + lo_a hi_b with three fp16 MMAs per 16 k and scales
+// the accumulator by 2^(e_i + e_j) (exact).  Error per product
+// <= 3 * 2^-22 |a||b| (R22), against the 1e-5 normwise bound of BJ.
+//
+// The split is the fp32 -> fp16 conversion on the HBM -> SMEM edge:
+// it runs once per K panel, and the split operand has exactly the bytes of
+// the fp32 panel (two fp16 per element), so the GEMM's TMA moves what the raw
+// panel would and the split may run in place.
+//
+// Layouts (ld = the fp32 row stride of the buffer, in floats):
+//   A' row i at byte 4 ld i; 32-k stage s occupies the stage's own 128 bytes:
+//      fp16 [64 s + (k % 32)] = hi, [64 s + 32 + (k % 32)] = lo
+//   B' row k at byte 4 ld k: fp16 [n] = hi, [ld + n] = lo
+// Panels are zero-padded to Kp = K rounded up to 32 (rows / columns [K, Kp)
+// must exist in the destination).
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "leaf_common.cuh"
+#include "northup_internal.h"
+
+namespace nu {
+namespace leaf {
+
+// e with amax 2^-e in [2^14, 2^15), clamped so that 2^-e is a normal float
+// (rows of zeros, or maxima outside [2^-112, 2^127), are not normalised).
+__device__ __forceinline__ int split_exponent(float amax) {
+  int E = static_cast<int>((__float_as_uint(amax) >> 23) & 0xFF);
+  if (E == 0) E = 1;
+  const int e = E - 141;
+  return e < -126 ? -126 : (e > 126 ? 126 : e);
+}
+
+__device__ __forceinline__ float pow2(int e) {   // e in [-126, 127]
+  return __uint_as_float(static_cast<uint32_t>(e + 127) << 23);
+}
+
+__device__ __forceinline__ void split1(float x, float s, __half& hi, __half& lo) {
+  const float y = x * s;                        // exact: s is a power of two
+  hi = __float2half_rn(y);
+  lo = __float2half_rn(y - __half2float(hi));   // y - hi is exact in fp32
+}
+
+// One warp per row of A (grid-stride).  Pass 1: row max; pass 2: each 32-k
+// group is read by the warp, then written (the same 128 bytes when in place).
+__global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
+                                                      float* dst, int64_t ldd, int* ea) {
+  const int lane = threadIdx.x & 31;
+  const int warps = (gridDim.x * blockDim.x) >> 5;
+  for (int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M; r += warps) {
+    const float* a = A + static_cast<int64_t>(r) * lda;
+    float m = 0.f;
+    for (int k = lane; k < Kl; k += 32) m = fmaxf(m, fabsf(a[k]));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const int e = split_exponent(m);
+    if (lane == 0) ea[r] = e;
+    const float s = pow2(-e);
+    __half* out = reinterpret_cast<__half*>(dst + static_cast<int64_t>(r) * ldd);
+    for (int k0 = 0; k0 < Kp; k0 += 32) {
+      const int k = k0 + lane;
+      const float x = k < Kl ? a[k] : 0.f;
+      __syncwarp();                              // the group is read before it is overwritten
+      __half hi, lo;
+      split1(x, s, hi, lo);
+      out[2 * k0 + lane] = hi;
+      out[2 * k0 + 32 + lane] = lo;
+      __syncwarp();
+    }
+  }
+}
+
+// Column maxima of B (|x| as uint bits; atomicMax over 256-row slabs).
+__global__ void __launch_bounds__(256) colmax_kernel(const float* B, int64_t ldb, int Kl, int N,
+                                                     unsigned* bmax) {
+  const int n = blockIdx.x * 256 + threadIdx.x;
+  if (n >= N) return;
+  const int k0 = blockIdx.y * 256, k1 = min(Kl, k0 + 256);
+  float m = 0.f;
+  for (int k = k0; k < k1; ++k) m = fmaxf(m, fabsf(B[static_cast<int64_t>(k) * ldb + n]));
+  atomicMax(bmax + n, __float_as_uint(m));
+}
+
+// One CTA per row of B: the row is staged in shared memory before any of it
+// is overwritten (in place, hi lands on the row's first half and lo on its
+// second).  Rows [Kl, Kp) are written as zeros.
+constexpr int kSplitRowMaxN = 49152;   // 192 KiB of fp32 staging
+__global__ void __launch_bounds__(1024) split_b_kernel(const float* B, int64_t ldb, int Kl, int N,
+                                                       const unsigned* bmax, float* dst, int64_t ldd,
+                                                       int* eb) {
+  extern __shared__ float row[];
+  const int k = blockIdx.x;
+  const float* brow = B + static_cast<int64_t>(k) * ldb;
+  for (int n = threadIdx.x; n < N; n += blockDim.x) row[n] = k < Kl ? brow[n] : 0.f;
+  __syncthreads();
+  __half* hi_row = reinterpret_cast<__half*>(dst + static_cast<int64_t>(k) * ldd);
+  __half* lo_row = hi_row + ldd;
+  for (int n = threadIdx.x; n < N; n += blockDim.x) {
+    const int e = split_exponent(__uint_as_float(bmax[n]));
+    if (k == 0) eb[n] = e;
+    __half h, l;
+    split1(row[n], pow2(-e), h, l);
+    hi_row[n] = h;
+    lo_row[n] = l;
+  }
+}
+
+int64_t split_b_max_n() { return kSplitRowMaxN; }
+
+int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64_t ldd, int* ea, int sms,
+                   cudaStream_t s) {
+  if (M <= 0) return 0;
+  const int Kp = (Kl + 31) / 32 * 32;
+  const int grid = static_cast<int>(std::min<int64_t>((M + 7) / 8, 32LL * sms));
+  split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_a launch: %s", cudaGetErrorString(e));
+}
+
+int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64_t ldd, int* eb,
+                   unsigned* bmax, cudaStream_t s) {
+  if (N <= 0) return 0;
+  if (N > split_b_max_n()) return fail(NU_EINVAL, "split_b: N = %d above %lld", N, (long long)split_b_max_n());
+  const int Kp = (Kl + 31) / 32 * 32;
+  cudaError_t e = cudaMemsetAsync(bmax, 0, sizeof(unsigned) * N, s);
+  if (e != cudaSuccess) return fail(NU_ECUDA, "split_b memset: %s", cudaGetErrorString(e));
+  if (Kl > 0) colmax_kernel<<<dim3((N + 255) / 256, (Kl + 255) / 256), 256, 0, s>>>(B, ldb, Kl, N, bmax);
+  static bool configured[kMaxDevices];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!configured[dev]) {
+    e = cudaFuncSetAttribute(split_b_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * kSplitRowMaxN);
+    if (e != cudaSuccess) return fail(NU_ECUDA, "split_b attribute: %s", cudaGetErrorString(e));
+    configured[dev] = true;
+  }
+  const int threads = std::min(1024, std::max(64, (N / 8 + 31) / 32 * 32));
+  split_b_kernel<<<Kp, threads, 4 * static_cast<size_t>(N), s>>>(B, ldb, Kl, N, bmax, dst, ldd, eb);
+  e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_b launch: %s", cudaGetErrorString(e));
+}
+
+void preload_split() {
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, split_a_kernel);
+  cudaFuncGetAttributes(&fa, colmax_kernel);
+  cudaFuncGetAttributes(&fa, split_b_kernel);
+}
+
+}  // namespace leaf
+}  // namespace nu

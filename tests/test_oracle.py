@@ -144,6 +144,50 @@ def test_freivalds_exact_on_integers_and_detects_misplaced_block():
     assert not np.array_equal(x2, y2)
 
 
+def test_freivalds_ratio_scale_pinned_by_planted_row_error():
+    """The normalised ratio |(C r)_i - (A (B r))_i| / (||A_i|| sum_j ||B_j|| |r_j|)
+    (SURVEY §8(c) "Large configs") is pinned to its closed form: a planted
+    row-wide error Delta_ij = eps ||A_i|| ||B_j|| r_j (same sign as r_j, so no
+    cancellation) gives (Delta r)_i = eps ||A_i|| sum_j ||B_j|| |r_j| exactly,
+    i.e. a ratio of eps.  A scale bug (sum ||B_j||^2, a stray factor N, a
+    missing ||A_i||) moves the ratio off eps; the fp32-rounded exact C stays far
+    below TOL, and eps = 2e-5 > TOL = 1e-5 fails the check."""
+    M, N, K = 48, 64, 96
+    A = nugen.fill(M, K, 31, 1)
+    B = nugen.fill(K, N, 31, 2)
+    R = oracle.gemm(A, B)
+    rn, cn = oracle.row_norms(A), oracle.col_norms(B)
+    r = np.where(np.random.default_rng(5).random(N) < 0.5, -1.0, 1.0)
+    C = R.astype(np.float32)
+    e0, _, _ = oracle.freivalds(A, B, C, r)
+    assert e0 < 1e-7                                 # fp32 rounding of the exact result
+    for i, eps in ((5, 2e-5), (40, 3e-6)):
+        bad = R.copy()
+        bad[i, :] += eps * rn[i] * cn * r            # the planted row error, in fp64
+        # compare in fp64 so the planted value is not lost to fp32 rounding
+        e, x, y = oracle.freivalds(A, B, bad.astype(np.float32), r)
+        dx = (bad.astype(np.float32).astype(np.float64) - R) @ r
+        ratio_i = abs(dx[i]) / (rn[i] * float(np.sum(cn * np.abs(r))))
+        assert abs(ratio_i - eps) < 0.05 * eps      # the closed form, through fp32 rounding
+        assert abs(e - ratio_i) < 1e-7               # the oracle reports that row's ratio
+        assert (e > 1e-5) == (eps > 1e-5)            # 2e-5 fails TOL, 3e-6 passes
+
+
+def test_freivalds_integer_exact_detects_single_element():
+    """On integer inputs x = C r and y = A (B r) are exact in fp64, so a single
+    wrong element (off by 1) is detected however large N is (no dilution)."""
+    M, N, K = 40, 300, 50
+    A = nugen.fill(M, K, 32, 1, "int")
+    B = nugen.fill(K, N, 32, 2, "int")
+    C = oracle.gemm(A, B).astype(np.float32)
+    r = np.where(np.random.default_rng(6).random(N) < 0.5, -1.0, 1.0)
+    _, x, y = oracle.freivalds(A, B, C, r)
+    assert np.array_equal(x, y)
+    C[17, 222] += 1.0
+    _, x2, y2 = oracle.freivalds(A, B, C, r)
+    assert np.flatnonzero(x2 != y2).tolist() == [17] and abs(x2[17] - y2[17]) == 1.0
+
+
 @settings(max_examples=25, deadline=None)
 @given(M=st.integers(1, 40), N=st.integers(1, 40), K=st.integers(0, 40),
        bm=st.integers(1, 17), bn=st.integers(1, 17), bk=st.integers(1, 17),
