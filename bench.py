@@ -4,11 +4,13 @@ metric: "out-of-core GEMM TFLOP/s at 1/2/4/8 B200; % slowdown vs in-HBM;
 roofline frac").
 
 One step = one northup_gemm call = one pass of the whole hot path:
-  value : the GEMM with A, B, C already resident in HBM (single-node HBM tree,
-          CS4 — the paper's in-memory baseline, P:353/P:381);
-  e2e   : the same GEMM through the C ABI from pinned HOST buffers
-          (HOST -> HBM (8 GiB cap) -> SMEM/TMEM), every H2D/D2H inside the
-          timed region — the out-of-core number.  slowdown = t_e2e/t_value - 1.
+  value  : the out-of-core GEMM (the metric) through the C ABI from pinned
+           HOST buffers (HOST -> HBM (8 GiB cap) -> SMEM/TMEM), every H2D/D2H
+           inside the step; CUDA events bracketing the synchronous calls;
+  e2e    : the same calls timed by the host clock (planning and issue included);
+  in_hbm : the same GEMM with A, B, C resident in HBM (single-node HBM tree,
+           CS4 — the paper's in-memory baseline).
+  slowdown = t_value / t_in_hbm - 1.
 
 N = 1 runs BASELINE configs[2] (cfg3: 32768^3, 8 GiB HBM cap).  Under torchrun
 (N > 1) every rank runs its C region of configs[3] (cfg4: 65536 x 65536 x
@@ -51,9 +53,6 @@ HOTSPOT = dict(R=32768, C=32768, iters=256, cap=8 * GiB,
                     "HBM (8 GiB cap) -> SMEM, 1 GPU (S§8(f) NEXT-3)")
 HS_FLOPS_PER_UPDATE = 14                 # flops of one cell update as the formula states (5 mul + 9 add/sub)
 FP32_LANES_PER_SM, N_SMS = 128, 148      # B200: 4 SMSPs x 32 fp32 lanes; 148 SMs
-NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25      # B200_PROFILING.md nominal dense ratio
-LEAF_KERNELS = {1: "nu::leaf::sm1::leaf_gemm_1sm_kernel", 2: "nu::leaf::sm2::leaf_gemm_2sm_kernel",
-                3: "nu::leaf::sm3::leaf_gemm_2sm_ldg_kernel", 4: "nu::leaf::sm4::leaf_gemm_2sm_tm_kernel"}
 
 
 def log(*a):
@@ -201,7 +200,8 @@ def cpu_baseline(cfg: dict, a_host, b_host, c_gpu, budget_s: float) -> dict:
     import numpy as np
     import oracle
     M, N, K = cfg["M"], cfg["N"], cfg["K"]
-    cores = oracle.threads()
+    cores = len(os.sched_getaffinity(0))
+    oracle.set_threads(cores)
     rng = np.random.default_rng(12345)
     rows = np.sort(rng.choice(M, size=min(M, cores), replace=False))
     t0 = time.perf_counter()
@@ -219,9 +219,15 @@ def cpu_baseline(cfg: dict, a_host, b_host, c_gpu, budget_s: float) -> dict:
         nrows += len(more)
         done.append((more, ref2))
     flops = 2.0 * nrows * N * K
+    # the same oracle on one core (a single row of C)
+    oracle.set_threads(1)
+    t0 = time.perf_counter()
+    oracle.gemm_rows(a_host, b_host, rows[:1])
+    one = 2.0 * N * K / (time.perf_counter() - t0) / 1e12
+    oracle.set_threads(cores)
     out = {"value": flops / elapsed / 1e12, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
            "sample": f"{nrows} full rows of C ({nrows}x{N}x{K} fp64 triple loop), {elapsed:.1f} s",
-           "seconds": elapsed}
+           "seconds": elapsed, "single_core_value": one, **cpu_facts()}
     if c_gpu is not None:
         cn = oracle.col_norms(b_host)
         worst = 0.0
@@ -231,6 +237,93 @@ def cpu_baseline(cfg: dict, a_host, b_host, c_gpu, budget_s: float) -> dict:
             worst = max(worst, e)
         out["gpu_normwise_err_on_sample"] = worst
         out["gpu_parity_ok"] = bool(worst <= 1e-5)
+    return out
+
+
+# -------------------------------------------------------------- host facts
+def cpu_facts() -> dict:
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    nodes = [d for d in os.listdir("/sys/devices/system/node") if d.startswith("node") and d[4:].isdigit()] \
+        if os.path.isdir("/sys/devices/system/node") else []
+    return {"cpu_model": model, "numa_nodes": len(nodes) or 1, "logical_cpus": os.cpu_count()}
+
+
+def _cpulist(text: str) -> set:
+    cpus = set()
+    for part in text.strip().split(","):
+        if not part:
+            continue
+        if "-" in part:
+            a, b = part.split("-")
+            cpus.update(range(int(a), int(b) + 1))
+        else:
+            cpus.add(int(part))
+    return cpus
+
+
+def bind_to_gpu_numa(dev_index: int) -> dict:
+    """Bind this process (and the threads it starts: the library's per-GPU
+    workers, the generator's OpenMP threads) to the NUMA node of its GPU, so
+    the pinned root strips are first-touched next to the GPU's PCIe link
+    (SURVEY §7 H5).  Returns what was done; a no-op on one-node hosts."""
+    import torch
+    info = {"gpu": dev_index, "numa_node": None, "cpus": None, "bound": False}
+    try:
+        p = torch.cuda.get_device_properties(dev_index)
+        bus = "%04x:%02x:%02x.0" % (p.pci_domain_id, p.pci_bus_id, p.pci_device_id)
+        with open(f"/sys/bus/pci/devices/{bus}/numa_node") as f:
+            node = int(f.read().strip())
+        info["numa_node"] = node
+        if node < 0:
+            return info
+        with open(f"/sys/devices/system/node/node{node}/cpulist") as f:
+            cpus = _cpulist(f.read()) & os.sched_getaffinity(0)
+        if cpus and len(cpus) < len(os.sched_getaffinity(0)):
+            os.sched_setaffinity(0, cpus)
+            info.update(cpus=len(cpus), bound=True)
+    except (OSError, AttributeError, ValueError) as ex:
+        info["error"] = repr(ex)
+    return info
+
+
+def kernel_launches() -> int:
+    import paper_conf_ipps_chey19_b200 as nu
+    f = nu.lib().northup_debug_kernel_launches
+    f.restype = ctypes.c_longlong
+    return int(f())
+
+
+def leaf_kernel_ms(A, B, C, kc: int, stream, reps: int = 2) -> list:
+    """Device time of each GEMM kernel launch of the leaf (CUDA events recorded
+    by the library around the kernel, on `stream`): the dominant kernel."""
+    import torch
+    import paper_conf_ipps_chey19_b200 as nu
+    f = nu.lib().northup_debug_leaf_gemm_events
+    f.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                  ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
+                  ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p]
+    M, K = A.shape
+    N = B.shape[1]
+    nev = 2 * (-(-K // kc)) * (-(-N // 32768))
+    out = []
+    for _ in range(reps):
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(nev)]
+        for e in evs:
+            e.record(stream)            # creates the events on this device
+        handles = (ctypes.c_void_p * nev)(*[e.cuda_event for e in evs])
+        used = ctypes.c_int(0)
+        nu.check(f(A.data_ptr(), A.stride(0), B.data_ptr(), B.stride(0), C.data_ptr(), C.stride(0), M, N, K, kc,
+                   stream.cuda_stream, handles, nev, ctypes.byref(used)))
+        torch.cuda.synchronize()
+        out += [evs[i].elapsed_time(evs[i + 1]) for i in range(0, used.value, 2)]
     return out
 
 
@@ -246,6 +339,8 @@ def run_ours(args, rank: int, world: int, local_rank: int):
         import torch.distributed as dist
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
+    all_cpus = os.sched_getaffinity(0)
+    numa = bind_to_gpu_numa(local_rank) if not args.no_numa_bind else {"bound": False, "disabled": True}
     name = args.config or ("cfg3" if world == 1 else "cfg4")
     cfg = dict(CONFIGS[name])
     if args.quick:
@@ -257,7 +352,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     kc = args.k_chunk
     if cfg["block"]:
         # a fixed block (cfg1's 64 x 64 x 64) fixes the K-panel sequence: the in-HBM
-        # reference accumulates in the same chunks, so the two stay bitwise comparable
+        # reference runs the same panels, so the two stay bitwise comparable
         kc = cfg["block"][2]
 
     # --- the out-of-core tree: HOST root -> HBM (cap) -> SMEM/TMEM leaf.  N > 1:
@@ -280,9 +375,9 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     nugen.fill(m, K, seed, nugen.MAT_A, "uniform", out=a, i0=r0, ncols=K)
     nugen.fill(K, n, seed, nugen.MAT_B, "uniform", out=b, j0=c0, ncols=N)
     log(f"[rank {rank}] {name} region {m}x{n}x{K}: inputs generated in pinned host memory "
-        f"in {time.perf_counter() - tg:.1f} s")
+        f"in {time.perf_counter() - tg:.1f} s (NUMA {numa})")
 
-    # --- the in-HBM tree (value): same GEMM, operands resident in HBM
+    # --- the in-HBM tree (CS4): the same GEMM with A, B, C resident in HBM
     th = nu.hbm_tree(local_rank)
     th.finalize()
     Ad = torch.from_numpy(a).to(dev)
@@ -327,45 +422,78 @@ def run_ours(args, rank: int, world: int, local_rank: int):
         if dist is not None:
             dist.barrier()
 
+    def max_over_ranks(x: float) -> float:
+        if dist is None:
+            return x
+        v = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(v, op=dist.ReduceOp.MAX)
+        return float(v.item())
+
     def timed(fn, steps, warmup):
+        """Device time (CUDA events on the torch stream bracketing synchronous
+        calls, barrier + synchronize on both sides, max over ranks) and host
+        wall time (perf_counter around the same calls, max over ranks)."""
         for _ in range(warmup):
             fn()
         barrier()
         evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        w0 = time.perf_counter()
         evs[0].record(stream)
         for i in range(steps):
             fn()
             evs[i + 1].record(stream)
         barrier()
+        wall = (time.perf_counter() - w0) * 1e3
         per = [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
-        total = evs[0].elapsed_time(evs[-1])
-        if dist is not None:
-            x = torch.tensor([total], dtype=torch.float64, device=dev)
-            dist.all_reduce(x, op=dist.ReduceOp.MAX)
-            total = float(x.item())
-        return total, per
+        return max_over_ranks(evs[0].elapsed_time(evs[-1])), max_over_ranks(wall), per
 
-    # value: in-HBM (the leaf runs on the current torch stream; one launch/step)
-    def step_hbm():
-        nu.leaf_gemm(Ad, Bd, Cd, k_chunk=kc, stream=stream)
-
-    ooc_stats = {}
-
+    ooc_stats, hbm_stats = {}, {}
     GM, GN = (M, N) if world > 1 else (m, n)
 
     def step_ooc():
         ooc_stats.update(t.gemm(Ab, Bb, Cb, GM, GN, K, ooc_opts))
 
+    def step_hbm():
+        hbm_stats.update(th.gemm(hA, hB, hC, m, n, K, opts))
+
     with ClockSampler(local_rank) as clk:
-        t_hbm, per_hbm = timed(step_hbm, args.steps, args.warmup)
-        t_ooc, per_ooc = timed(step_ooc, args.steps, args.warmup)
-    # BJ configs[1] reference point: the 8192^3 GEMM resident in HBM, same leaf,
-    # timed here (untimed w.r.t. the step) so the out-of-core rate can also be
-    # quoted against it (S§8(d) "relative to cfg2's 8192^3 in-HBM rate")
+        for _ in range(args.warmup):      # warm both trees before either timed region
+            step_ooc()
+        nl0 = kernel_launches()
+        t_ooc, wall_ooc, per_ooc = timed(step_ooc, args.steps, 0)
+        launches_timed = kernel_launches() - nl0
+        plan_ms_ooc = float(ooc_stats.get("t_plan_ms", 0.0))
+        t_hbm, wall_hbm, per_hbm = timed(step_hbm, args.steps, args.warmup)
+        # the dominant kernel, live: events around each GEMM kernel of the in-HBM
+        # leaf on this stream (same operands, same panels)
+        leaf_ms = leaf_kernel_ms(Ad, Bd, Cd, kc, stream, reps=1 if world > 1 else 2)
+    ck = clk.summary()
+    c_hbm = Cd.cpu().numpy()
+    c_ooc = c.copy()
+    bitwise_cross_tier = bool(np.array_equal(c_hbm, c_ooc))
+    # the leaf on device pointers (northup_leaf_gemm) against the CS4 tree: same bits
+    Cd2 = torch.empty_like(Cd)
+    nu.leaf_gemm(Ad, Bd, Cd2, k_chunk=kc, stream=stream)
+    torch.cuda.synchronize(dev)
+    bitwise_tree_vs_leaf = bool(torch.equal(Cd, Cd2))
+    del Cd2
+    # the other splits of the leaf (DESIGN.md R22), in-HBM rate only: npass = 4
+    # adds lo.lo (4 MMAs per 16 k); npass = 1 is hi.hi alone (fails the bound)
+    split_rates = {}
+    if not args.quick or world == 1:
+        for npass in (4, 1):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            nu.leaf_gemm(Ad, Bd, Cd, k_chunk=kc, npass=npass, stream=stream)
+            e0.record(stream)
+            nu.leaf_gemm(Ad, Bd, Cd, k_chunk=kc, npass=npass, stream=stream)
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            split_rates[f"npass{npass}"] = round(2.0 * m * n * K / (e0.elapsed_time(e1) * 1e-3) / 1e12, 3)
+    # BJ configs[1] reference point: the 8192^3 GEMM resident in HBM, same leaf
     A2 = torch.rand((8192, 8192), device=dev) * 2 - 1
     B2 = torch.rand((8192, 8192), device=dev) * 2 - 1
     C2 = torch.empty((8192, 8192), device=dev)
-    t_c2, _ = timed(lambda: nu.leaf_gemm(A2, B2, C2, k_chunk=kc, stream=stream), 5, 3)
+    t_c2, _, _ = timed(lambda: nu.leaf_gemm(A2, B2, C2, k_chunk=kc, stream=stream), 5, 3)
     cfg2_tflops = 2.0 * 8192 ** 3 / (t_c2 / 5 * 1e-3) / 1e12
     del A2, B2, C2
     # staging evidence (untimed): one call in timing mode for per-stream busy
@@ -387,50 +515,41 @@ def run_ours(args, rank: int, world: int, local_rank: int):
         ok = bool(torch.equal(full[r0:r1, c0:c1].cpu(), torch.from_numpy(c)))
         del full
         replicate_ms = (replicate_ms, ok)
-    c_hbm = Cd.cpu().numpy()
-    c_ooc = c.copy()
-    bitwise_cross_tier = bool(np.array_equal(c_hbm, c_ooc))
-    # the single-node HBM tree through the C ABI must give the same bits
-    th.gemm(hA, hB, hC, m, n, K, opts)
-    torch.cuda.synchronize(dev)
-    bitwise_tree_vs_leaf = bool(torch.equal(Cd, torch.from_numpy(c_hbm).to(dev)))
 
     flops_total = 2.0 * M * N * K
-    ms_hbm = t_hbm / args.steps
     ms_ooc = t_ooc / args.steps
-    value = flops_total / (ms_hbm * 1e-3) / 1e12
-    e2e = flops_total / (ms_ooc * 1e-3) / 1e12
+    ms_hbm = t_hbm / args.steps
+    value = flops_total / (ms_ooc * 1e-3) / 1e12
+    in_hbm = flops_total / (ms_hbm * 1e-3) / 1e12
+    e2e = flops_total / (wall_ooc / args.steps * 1e-3) / 1e12
     peaks = measured_peaks()
     # burst peak when the timed region ran at full clocks (a short step, no power
     # cap), the sustained one when the power cap pulled the clocks down
-    ck = clk.summary()
     at_max = bool(ck.get("sm_mhz") and ck.get("sm_max_mhz") and ck["sm_mhz"] >= 0.95 * ck["sm_max_mhz"])
     peak_kind = "burst" if at_max else "sustained"
     p_bf16 = peaks["bf16_burst"] if at_max else peaks["bf16_sustained"]
-    p_tf32 = p_bf16 * NOMINAL_TF32_OVER_BF16
-    # leaf split (R21): per useful MAC one tf32 MAC (hi.hi) + two
-    # bf16 MACs (the cross terms) -> time per useful flop 1/P_tf32 + 2/P_bf16
-    p_eff = 1.0 / (1.0 / p_tf32 + 2.0 / p_bf16)
-    # dominant kernel: the leaf.  One in-HBM step = ceil(K / k_chunk) K-panel
-    # launches on the torch stream (leaf_host.cu), back to back.
+    # leaf split (R22): three fp16 MMAs per useful MAC (hi.hi, hi.lo,
+    # lo.hi); fp16 and bf16 share the dense tensor rate -> P_eff = P_bf16 / 3
+    p_eff = p_bf16 / 3.0
     kc_eff = kc or 2048
-    launches_per_step = -(-K // kc_eff)
-    leaf_ms = statistics.mean(per_hbm) / launches_per_step
-    flops_per_launch = 2.0 * m * n * min(K, kc_eff)
-    achieved = flops_per_launch / (leaf_ms * 1e-3) / 1e12
+    flops_per_launch = 2.0 * m * min(n, 32768) * min(K, kc_eff)
+    kern_ms = statistics.mean(leaf_ms) if leaf_ms else float("nan")
+    achieved = flops_per_launch / (kern_ms * 1e-3) / 1e12
+    launches_per_leaf = -(-K // kc_eff) * (-(-n // 32768))
     traffic = tensor_active = None
     tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
             tj = json.load(f)
-        if (tj.get("M"), tj.get("N"), tj.get("launch_K")) == (m, n, min(K, kc_eff)):
+        if (tj.get("M"), tj.get("N"), tj.get("launch_K")) == (m, min(n, 32768), min(K, kc_eff)):
             traffic = tj.get("dram_bytes")
             tensor_active = tj.get("tensor_pipe_active_pct")
-    clock_ghz = None
+    step_ms_tim = max(1e-9, float(tim.get("t_total_ms", ms_ooc)))
     result = None
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
+            os.sched_setaffinity(0, all_cpus)          # the oracle gets every host core
             cpu = cpu_baseline(dict(cfg, M=m, N=n), a, b, c_ooc, args.cpu_budget)
         result = {
             "metric": METRIC,
@@ -439,15 +558,16 @@ def run_ours(args, rank: int, world: int, local_rank: int):
             "n_gpus": world,
             "steps": args.steps,
             "warmup": args.warmup,
-            "ms_per_step": round(ms_hbm, 3),
+            "ms_per_step": round(ms_ooc, 3),
             "higher_is_better": True,
             "scaling": "strong" if world > 1 else "weak",
             "vs_baseline": None,
-            "dtype": "f32 (tcgen05 split: tf32 hi.hi + bf16 cross terms, fp32 accumulate)",
+            "dtype": "f32 (tcgen05 kind::f16 on a scaled fp16 hi/lo split, 3 MMAs per 16 k, fp32 accumulate)",
             "data": "synthetic (counter-hash uniform [-1,1) fp32, seed = config index)",
             "config": {
                 "workload": f"{name}: {cfg['desc']}" + (" [quick: /4 sizes]" if args.quick else ""),
-                "M": M, "N": N, "K": K, "hbm_cap_bytes": cfg["cap"], "k_chunk": kc or 2048,
+                "M": M, "N": N, "K": K, "hbm_cap_bytes": cfg["cap"], "k_panel": kc or 2048,
+                "tmem_acc_chunk": 256,
                 "region_per_gpu": [m, n, K],
                 "parallelism": f"C subtrees {nu.partition(world, M, N)} over {world} GPU(s)" if world > 1 else "1 GPU",
                 "schedule": {1: "S1", 2: "S2"}.get(ooc_stats.get("schedule"), "auto"),
@@ -456,17 +576,43 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                 "blocks": [ooc_stats.get("bm"), ooc_stats.get("bn"), ooc_stats.get("bk")],
                 "drain_tail_k": ooc_stats.get("tail_k"), "drain_strips": ooc_stats.get("strips"),
                 "hbm_footprint_bytes": ooc_stats.get("hbm_peak_bytes"),
+                "numa": numa,
                 "l2": "inputs (>= 4 GiB each) exceed the 126 MB L2; no flush needed",
+                "value_basis": "out-of-core: northup_gemm from pinned HOST buffers through the tree, every "
+                               "H2D/D2H inside the step; CUDA events on the calling stream bracketing the "
+                               "synchronous calls, max over ranks",
             },
             "e2e": {"value": round(e2e, 3), "unit": "TFLOP/s",
                     "h2d_bytes_per_step": int(ooc_stats.get("bytes_h2d", 0)),
                     "d2h_bytes_per_step": int(ooc_stats.get("bytes_d2h", 0)),
                     "p2p_bytes_per_step": int(ooc_stats.get("bytes_p2p", 0)),
-                    "ms_per_step": round(ms_ooc, 3),
-                    "leaf_launches_per_step": int(ooc_stats.get("leaf_launches", 0))},
+                    "ms_per_step": round(wall_ooc / args.steps, 3),
+                    "leaf_launches_per_step": int(ooc_stats.get("leaf_launches", 0)),
+                    "basis": "the same northup_gemm calls timed by the host clock (planning and issue included)"},
+            "in_hbm": {"value": round(in_hbm, 3), "unit": "TFLOP/s", "ms_per_step": round(ms_hbm, 3),
+                       "basis": "single-node HBM tree (CS4): northup_gemm on operands resident in HBM, same "
+                                "leaf and K-panel sequence (reading R16)",
+                       "split_variants_tflops": split_rates},
             "slowdown_pct_vs_in_hbm": round(100.0 * (ms_ooc / ms_hbm - 1.0), 2),
             "cfg2_in_hbm_tflops": round(cfg2_tflops, 3),
-            "slowdown_pct_vs_cfg2_in_hbm": round(100.0 * (cfg2_tflops / (e2e / world) - 1.0), 2),
+            "slowdown_pct_vs_cfg2_in_hbm": round(100.0 * (cfg2_tflops / (value / world) - 1.0), 2),
+            "runtime_overhead": {
+                "plan_ms": round(plan_ms_ooc, 3),
+                "plan_pct_of_step": round(100.0 * plan_ms_ooc / ms_ooc, 3),
+                "host_vs_device_ms_per_step": round((wall_ooc - t_ooc) / args.steps, 3),
+                "paper": "P:367: runtime overhead below 1 %",
+            },
+            "breakdown": {   # Fig. 7/8 analogue: stream busy shares of one out-of-core step
+                "step_ms": round(step_ms_tim, 3),
+                "compute_pct": round(100.0 * tim.get("t_compute_ms", 0.0) / step_ms_tim, 1),
+                "h2d_pct": round(100.0 * tim.get("t_h2d_ms", 0.0) / step_ms_tim, 1),
+                "d2h_pct": round(100.0 * tim.get("t_d2h_ms", 0.0) / step_ms_tim, 1),
+                "p2p_pct": round(100.0 * tim.get("t_p2p_ms", 0.0) / step_ms_tim, 1),
+                "exposed_transfer_pct": round(100.0 * max(0.0, step_ms_tim - tim.get("t_compute_ms", 0.0))
+                                              / step_ms_tim, 1),
+                "basis": "CUDA events around every op of one untimed call (collect_timing); busy = sum of "
+                         "op durations per stream; exposed = step - compute busy",
+            },
             "staging": {
                 "pcie_measured": pcie,
                 "h2d_busy_gbs": round(tim["bytes_h2d"] / (tim["t_h2d_ms"] * 1e6), 2) if tim.get("t_h2d_ms") else None,
@@ -474,11 +620,6 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                 "h2d_avg_gbs_over_step": round(ooc_stats.get("bytes_h2d", 0) / (ms_ooc * 1e6), 2),
                 "d2h_avg_gbs_over_step": round(ooc_stats.get("bytes_d2h", 0) / (ms_ooc * 1e6), 2),
                 "busy_ms": {k: round(tim.get(k, 0.0), 2) for k in ("t_h2d_ms", "t_compute_ms", "t_d2h_ms", "t_p2p_ms")},
-                # share of the copy time hidden under compute: the part of the step not
-                # covered by leaf kernels is at most the exposed copy time
-                "copy_hidden_pct": round(100.0 * (1.0 - max(0.0, ms_ooc - tim.get("t_compute_ms", 0.0))
-                                                  / max(1e-9, tim.get("t_h2d_ms", 0.0) + tim.get("t_d2h_ms", 0.0))), 1)
-                if tim.get("t_h2d_ms") else None,
                 "basis": "busy = sum of the copy-stream op durations (CUDA events, one untimed call in timing mode)"},
             "e2e_roofline": None,
             "replicate": None if replicate_ms is None else {
@@ -490,31 +631,39 @@ def run_ours(args, rank: int, world: int, local_rank: int):
             "roofline": {"bound": "tensor", "achieved": round(achieved, 3),
                          "peak": round(p_eff, 3), "unit": "TFLOP/s",
                          "frac": round(achieved / p_eff, 4), "traffic": traffic,
-                         "peak_basis": (f"useful-flop ceiling of the split 1/(1/P_tf32 + 2/P_bf16): "
-                                        f"P_bf16 = {peaks['source']} bf16 {peak_kind} "
-                                        f"{p_bf16} TF/s (burst if the timed region's median SM clock "
-                                        f"was >= 0.95 x max, else sustained), P_tf32 = P_bf16 x nominal "
-                                        f"tf32/bf16 {NOMINAL_TF32_OVER_BF16:.3f}"),
-                         "kernel": LEAF_KERNELS.get(nu.lib().northup_debug_leaf_variant(), "?"),
-                         "launch": [m, n, min(K, kc_eff)], "launches_per_step": launches_per_step,
-                         "flops_per_launch": flops_per_launch, "ms_per_launch": round(leaf_ms, 3),
+                         "peak_basis": (f"useful-flop ceiling of the split P_bf16 / 3 (three fp16 MMAs per useful "
+                                        f"MAC; fp16 = bf16 dense rate): P_bf16 = {peaks['source']} bf16 "
+                                        f"{peak_kind} {p_bf16} TF/s (burst if the timed region's median SM clock "
+                                        f"was >= 0.95 x max, else sustained)"),
+                         "kernel": "nu::leaf::x3::leaf_x3_kernel",
+                         "launch": [m, min(n, 32768), min(K, kc_eff)], "launches_per_leaf_call": launches_per_leaf,
+                         "flops_per_launch": flops_per_launch, "ms_per_launch": round(kern_ms, 3),
+                         "launches_timed": len(leaf_ms),
                          "tensor_pipe_active_pct_ncu": tensor_active,
+                         "achieved_basis": "useful flops 2 m n k of one K-panel launch / its CUDA-event duration "
+                                           "(events recorded by the library around each GEMM kernel on the torch "
+                                           "stream, in-HBM operands)",
                          "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "
                                           "(profiles/leaf_traffic.json); algorithmic bytes per launch "
-                                          f"= A/B panel + C read+write = {4 * (m + n) * min(K, kc_eff) + 8 * m * n:.3e}"},
-            "gpu_launches": args.steps * launches_per_step * world + int(ooc_stats.get("leaf_launches", 0)) * args.steps,
+                                          f"= split A/B panel + C write = "
+                                          f"{4 * (m + min(n, 32768)) * min(K, kc_eff) + 4 * m * min(n, 32768):.3e}"},
+            "gpu_launches": launches_timed * world,
+            "gpu_launches_basis": "library kernel launches (northup_debug_kernel_launches) during the timed "
+                                  "out-of-core steps on this rank x ranks",
             "parity": {"bitwise_in_hbm_vs_out_of_core": bitwise_cross_tier,
                        "bitwise_tree_vs_leaf": bitwise_tree_vs_leaf},
             "clocks": ck,
         }
         rl = ooc_roofline(2.0 * m * n * K, int(ooc_stats.get("bytes_h2d", 0)),
                           int(ooc_stats.get("bytes_d2h", 0)), p_eff, pcie)
-        e2e_gpu = 2.0 * m * n * K / (ms_ooc * 1e-3) / 1e12
-        rl.update(achieved=round(e2e_gpu, 3), frac=round(e2e_gpu / rl["peak"], 4),
+        v_gpu = 2.0 * m * n * K / (ms_ooc * 1e-3) / 1e12
+        rl.update(achieved=round(v_gpu, 3), frac=round(v_gpu / rl["peak"], 4),
                   basis="per GPU: out-of-core TF/s of this GPU's region / min(P_eff, BW_e x I_e) (S§8(d))")
         result["e2e_roofline"] = rl
         if cpu is not None:
             result["cpu_baseline"] = {k: cpu[k] for k in ("value", "unit", "cores", "kind", "sample")}
+            for k in ("cpu_model", "numa_nodes", "single_core_value"):
+                result["cpu_baseline"][k] = cpu.get(k)
             result["parity"]["oracle_normwise_err_rows"] = cpu.get("gpu_normwise_err_on_sample")
             result["parity"]["oracle_ok"] = cpu.get("gpu_parity_ok")
     th.destroy()
@@ -685,7 +834,7 @@ def run_reference(args):
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{name}: {cfg['desc']}", "M": M, "N": N, "K": K},
         "cpu_baseline": {"value": round(v, 6), "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{nrows} full rows of C per step ({nrows}x{N}x{K})"},
+                         "sample": f"{nrows} full rows of C per step ({nrows}x{N}x{K})", **cpu_facts()},
         "e2e": {"value": round(v, 6), "unit": "TFLOP/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -711,10 +860,25 @@ def main():
                     help="N>1: every rank loads its whole A/B strips over PCIe (no NVLink sharing)")
     ap.add_argument("--device-mod", type=int, default=0,
                     help="map LOCAL_RANK modulo this many GPUs (multi-rank tests on one GPU)")
+    ap.add_argument("--no-numa-bind", action="store_true", help="do not bind ranks to their GPU's NUMA node")
     args = ap.parse_args()
     if args.warmup < 3:
         log("warning: the timing rules ask for >= 3 warm-up steps")
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # not under torchrun: start one rank per GPU ourselves (same command line)
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+        log("spawning:", " ".join(cmd))
+        sys.exit(subprocess.call(cmd))
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        log(f"error: --gpus {args.gpus} but WORLD_SIZE={world}; run one rank per GPU (torchrun "
+            f"--nproc-per-node {args.gpus}) or drop --gpus")
+        sys.exit(2)
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.device_mod > 0:          # test mode: several ranks share the visible GPUs

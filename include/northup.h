@@ -183,9 +183,10 @@ typedef struct {
   int schedule;         /* NU_SCHED_AUTO / S1 / S2 */
   int replicate_result; /* 1: after the join, gather C into every HBM node's replica
                            buffer (northup_tree_set_replica) — NCCL over NVLink */
-  int64_t k_chunk;      /* TMEM accumulation length in K (0 = library default, 2048) */
-  int npass;            /* leaf split (R19/R21): 0 = default (2); 2 = tf32 hi.hi +
-                           bf16 cross terms; 3 = 3xTF32; 1 = plain TF32 (negative test) */
+  int64_t k_chunk;      /* K panel of one leaf launch and of one operand split (0 = 2048); the
+                           TMEM accumulation inside a panel is 256 (R20) */
+  int npass;            /* leaf split (R22): 0 = default (3); 3 = fp16 hi.hi + hi.lo +
+                           lo.hi on the scaled split; 4 = + lo.lo; 1 = hi.hi only (negative test) */
   int resident;         /* 1: run the plan with operands already resident (in-HBM timing) */
   int collect_timing;   /* 1: record per-stage CUDA-event timings into the stats */
   int64_t a_panel_k;    /* FILE root only: A is stored K-panel-major (R15 preprocessing,
@@ -244,11 +245,13 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
 /* ----------------------------------------------------- the leaf directly */
 /* The SMEM/TMEM leaf on device pointers (CS4 in-HBM reference and tests):
  * C = A.B (accumulate = 0) or C += A.B (accumulate = 1), row-major, on `stream`
- * (a cudaStream_t, NULL = legacy default) of the CURRENT device. A and B need a
- * 16-byte-aligned base and lda, ldb multiples of 4 (TMA); C any alignment.
- * k_chunk = TMEM accumulation length (0 = 2048); npass 0/2 = tf32 hi.hi + bf16
- * cross terms, 3 = 3xTF32, 1 = plain TF32 (negative test).
- * Asynchronous: returns after the launch. */
+ * (a cudaStream_t, NULL = legacy default) of the CURRENT device ("C = AB").
+ * Per K panel of k_chunk (0 = 2048) the operands are split into scaled fp16
+ * hi/lo pairs (R22) in stream-ordered scratch the library owns
+ * ((M + N) x panel x 4 bytes, freed on the stream), then multiplied with
+ * tcgen05 MMAs.  A, B, C any alignment; N <= 49152; npass 0/3 = the product
+ * split, 4 = + lo.lo, 1 = hi.hi only (negative test); other values NU_EINVAL.
+ * Asynchronous: returns after the launches. */
 int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                       int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t k_chunk,
                       int npass, void* stream);

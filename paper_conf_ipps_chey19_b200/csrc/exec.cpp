@@ -265,8 +265,15 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       const float* a = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);
       const float* b = reinterpret_cast<const float*>(c.base[op.b_buf] + op.b_off * 4);
       float* cc = reinterpret_cast<float*>(c.base[op.c_buf] + op.c_off * 4);
-      int rc = leaf_gemm_launch(a, op.lda, b, op.ldb, cc, op.ldc, op.m, op.n, op.k, op.accumulate,
-                                P.kc, P.npass, s);
+      LeafCall lc{};
+      lc.A = a, lc.lda = op.lda, lc.B = b, lc.ldb = op.ldb, lc.C = cc, lc.ldc = op.ldc;
+      lc.M = op.m, lc.N = op.n, lc.K = op.k, lc.accumulate = op.accumulate, lc.panel = P.kc, lc.npass = P.npass;
+      if (wi < static_cast<int>(P.scr_buf.size()) && P.scr_buf[wi] >= 0) {
+        lc.scratch = c.base[P.scr_buf[wi]] + P.scr_off[wi];
+        lc.scratch_bytes = P.scr_bytes[wi];
+      }
+      lc.stream = s;
+      int rc = leaf_run(lc);
       if (rc) return rc;
     } else if (op.op == NU_OP_STENCIL) {
       const float* tin = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);
@@ -921,10 +928,14 @@ int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_bu
           if (e != cudaSuccess) result = cuda_fail(e, "copy");
         } else {
           if (w == slow_w && slow_pct > 0) debug_spin(debug_slow_ns(slow_pct, op.m, op.n, op.k), s);
-          result = leaf_gemm_launch(reinterpret_cast<const float*>(base[op.a_buf] + op.a_off * 4), op.lda,
-                                    reinterpret_cast<const float*>(base[op.b_buf] + op.b_off * 4), op.ldb,
-                                    reinterpret_cast<float*>(base[op.c_buf] + op.c_off * 4), op.ldc, op.m, op.n,
-                                    op.k, op.accumulate, kc, npass, s);
+          LeafCall lc{};
+          lc.A = reinterpret_cast<const float*>(base[op.a_buf] + op.a_off * 4), lc.lda = op.lda;
+          lc.B = reinterpret_cast<const float*>(base[op.b_buf] + op.b_off * 4), lc.ldb = op.ldb;
+          lc.C = reinterpret_cast<float*>(base[op.c_buf] + op.c_off * 4), lc.ldc = op.ldc;
+          lc.M = op.m, lc.N = op.n, lc.K = op.k, lc.accumulate = op.accumulate, lc.panel = kc, lc.npass = npass;
+          lc.scratch = base[3] + (q.arena_bytes - q.scratch_bytes), lc.scratch_bytes = q.scratch_bytes;
+          lc.stream = s;
+          result = leaf_run(lc);
         }
         cudaEvent_t ev;
         e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);

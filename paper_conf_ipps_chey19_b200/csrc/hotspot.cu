@@ -517,6 +517,7 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem4);
     hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY><<<dim3(static_cast<unsigned>(gx4), static_cast<unsigned>(gy4)),
                                              kV4NWX * kV4NWY * 32, smem4, stream>>>(a);
+    count_launches(1);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v4 launch");
   }
@@ -530,6 +531,7 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem3);
     hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY><<<dim3(static_cast<unsigned>(gx3), static_cast<unsigned>(gy3)),
                                              kV3NWX * kV3NWY * 32, smem3, stream>>>(a);
+    count_launches(1);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v3 launch");
   }
@@ -539,6 +541,7 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
     if (gy2 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy2);
     hotspot_kernel_v2<kRPT, kNWX, kNWY><<<dim3(static_cast<unsigned>(gx2), static_cast<unsigned>(gy2)),
                                           kNWX * kNWY * 32, 0, stream>>>(a);
+    count_launches(1);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v2 launch");
   }
@@ -549,6 +552,7 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   cudaFuncSetAttribute(hotspot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        static_cast<int>(3ull * (kTY + 2 * kHotspotMaxIters) * (kTX + 2 * kHotspotMaxIters) * 4));
   hotspot_kernel<<<dim3(static_cast<unsigned>(gx), static_cast<unsigned>(gy)), dim3(kWX, kWY), smem, stream>>>(a);
+  count_launches(1);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel launch");
 }

@@ -454,6 +454,7 @@ int x3_gemm(const SplitOperand& A, const SplitOperand& B, float* C, int64_t ldc,
   const int pairs = sms / 2;
   const int grid = 2 * (tiles < pairs ? tiles : pairs);
   leaf_x3_kernel<<<grid, NUM_THREADS, SMEM_BYTES, stream>>>(tmA, tmB, tmC, p);
+  count_launches(1);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "leaf launch: %s", cudaGetErrorString(e));
 }

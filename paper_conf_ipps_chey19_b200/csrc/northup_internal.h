@@ -16,11 +16,14 @@ constexpr int kMaxDevices = 64;
 constexpr int64_t kDefaultKChunk = 2048;   // K panel of one leaf launch / split (R20, R22)
 constexpr int64_t kAccChunk = 256;         // TMEM accumulation length inside a panel (R20)
 constexpr int kDefaultNpass = 3;            // 3 = fp16 hi.hi + hi.lo + lo.hi on the scaled split (R22)
-constexpr int kDefaultLeafVariant = 5;      // 5 = x3 (split operands); 1..4 = round-1 kernels (comparison)
 constexpr int kSlots = 3;                  // staging ring depth per operand (reading R8)
 constexpr int kRasterBand = 16;            // n-blocks per raster band in the leaf
 constexpr int64_t kPanelChunks = 1;        // leaf K-panel launches, in k_chunks (0 = one launch)
 constexpr int kHotspotMaxIters = 8;        // HotSpot-2D iterations per leaf launch (shared-memory border)
+
+// Kernel launches issued by the library (all devices, all threads): the
+// bench's `gpu_launches` claim (northup_debug_kernel_launches).
+void count_launches(int n);
 
 // Thread-local error message (northup_last_error).  Returns its argument so
 // call sites can write `return fail(NU_EINVAL, "...")`.
@@ -123,6 +126,10 @@ struct Plan {
   int npass = 3;
   bool root_is_device = false;
   bool file_root = false;
+  // Leaf scratch per worker (split operands of one K panel, leaf_scratch_bytes):
+  // the last `scr_bytes` of arena buffer `scr_buf`, at byte offset `scr_off`.
+  std::vector<int> scr_buf;
+  std::vector<uint64_t> scr_off, scr_bytes;
   float hs_coef[5] = {};                // HotSpot-2D plans: cap_1, rx_1, ry_1, rz_1, amb
 };
 
@@ -140,7 +147,8 @@ int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc);
 struct QueueShape {
   int64_t tm = 0, tn = 0, bk = 0;   // tile rows / cols, K panel
   int64_t Tr = 0, Tc = 0;           // tile grid
-  uint64_t arena_bytes = 0;         // per sibling: 2 C-tile buffers + kSlots panel slots
+  uint64_t arena_bytes = 0;         // per sibling: 2 C-tile buffers + kSlots panel slots + leaf scratch
+  uint64_t scratch_bytes = 0;       // the leaf scratch at the end of that arena
 };
 int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M, int64_t N,
                  int64_t K, int64_t kc, int tiles, QueueShape* q);
@@ -174,17 +182,24 @@ struct LeafCall {
   uint64_t scratch_bytes;
   float* dbg;
   cudaStream_t stream;
+  // Debug timing: events recorded around each GEMM kernel (2 per launch, up
+  // to n_events) on `stream`; *events_used returns how many were recorded.
+  cudaEvent_t* events = nullptr;
+  int n_events = 0;
+  int* events_used = nullptr;
 };
 int leaf_run(const LeafCall& c);
 uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit);
+// Scratch of the largest leaf op over an m x n C block (256-B rounded).
+inline uint64_t leaf_scratch(int64_t m, int64_t n, int64_t panel) {
+  return (leaf_scratch_bytes(m, n, panel, false) + 255) / 256 * 256;
+}
+constexpr int64_t kLeafMaxN = 32768;   // columns of B split at a time (leaf_run)
 int64_t leaf_acc_chunk();
 bool leaf_tma_legal(const void* p, int64_t ld);
 int leaf_gemm_launch(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
                      int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
                      int npass, cudaStream_t stream);
-int leaf_gemm_launch_dbg(const float* A, int64_t lda, const float* B, int64_t ldb, float* C,
-                         int64_t ldc, int64_t M, int64_t N, int64_t K, int accumulate, int64_t kc,
-                         int npass, int b_kmajor, float* dbg, int variant, cudaStream_t stream);
 
 // --------------------------------------------------------------- HotSpot-2D
 // The leaf (hotspot.cu): `iters` (<= kHotspotMaxIters) iterations on a window

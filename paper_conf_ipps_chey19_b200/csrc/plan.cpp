@@ -71,6 +71,18 @@ int region_of(int G, int64_t M, int64_t N, int r, int64_t* r0, int64_t* r1, int6
   return 0;
 }
 
+// The leaf scratch of worker w: the last `scr` bytes of its arena buffer.
+static void set_scratch(Plan* P, int w, int buf, uint64_t arena_bytes, uint64_t scr) {
+  if (static_cast<int>(P->scr_buf.size()) <= w) {
+    P->scr_buf.resize(w + 1, -1);
+    P->scr_off.resize(w + 1, 0);
+    P->scr_bytes.resize(w + 1, 0);
+  }
+  P->scr_buf[w] = buf;
+  P->scr_off[w] = arena_bytes - scr;
+  P->scr_bytes[w] = scr;
+}
+
 namespace {
 
 northup_op make_leaf(int worker, int a, int64_t a_off, int64_t lda, int b, int64_t b_off,
@@ -125,7 +137,7 @@ struct S2Shape {
   uint64_t bytes;
 };
 
-uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, int64_t sr) {
+uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, int64_t sr, int64_t kc) {
   const int64_t kmain = K - tail;
   uint64_t e = static_cast<uint64_t>(bm) * pad_ld(bn);                    // C block
   if (kmain > 0)
@@ -134,7 +146,7 @@ uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, i
   if (tail > 0)
     e += static_cast<uint64_t>(tail) * pad_ld(bn) +                          // B tail
          static_cast<uint64_t>(kSlots) * sr * pad_ld(tail);                  // A strips
-  return e * 4;
+  return e * 4 + leaf_scratch(bm, bn, kc);                                   // + leaf scratch
 }
 
 // Predicted time of one S2 block with drain tail K_t: the main
@@ -203,11 +215,11 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
       S2Shape cand{};
       double cand_t = 0;
       for (int64_t tail : tails) {
-        uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr);
+        uint64_t bytes = s2_bytes(bm, bn, bk, K, tail, sr, x.kc);
         int64_t use_bk = bk;
         if (bytes > cap && tail == 0 && bk > x.kc && x.obk <= 0) {   // the minimum panel
           use_bk = x.kc;
-          bytes = s2_bytes(bm, bn, use_bk, K, 0, 0);
+          bytes = s2_bytes(bm, bn, use_bk, K, 0, 0, x.kc);
         }
         if (bytes > cap) continue;
         const double t = s2_time(bm, bn, K, tail, x.a_share, x.b_share);
@@ -250,6 +262,7 @@ struct S2Layout {
 S2Layout layout_s2(Builder& B, const S2Shape& s, int hbm_node, int w, int64_t K) {
   S2Layout L;
   L.arena = B.add_buf(B_ARENA, hbm_node, w, s.bytes);
+  set_scratch(B.P, w, L.arena, s.bytes, leaf_scratch(s.bm, s.bn, B.P->kc));
   L.ldC = pad_ld(s.bn);
   L.ldA = pad_ld(s.bk);
   L.ldBs = pad_ld(s.bn);
@@ -592,7 +605,8 @@ int build_s1(const EdgeCtx& x, northup_stats* st) {
   auto bytes_of = [&](int64_t bm_, int64_t bn_, int64_t bk_) -> uint64_t {
     return 4ull * (2ull * bm_ * pad_ld(K)             // two row shards (next prefetches)
                    + 2ull * bm_ * pad_ld(bn_)         // double-buffered C block
-                   + uint64_t(kSlots) * bk_ * pad_ld(bn_));
+                   + uint64_t(kSlots) * bk_ * pad_ld(bn_)) +
+           leaf_scratch(bm_, bn_, x.kc);
   };
   while (bytes_of(bm, bn, bk) > cap) {
     if (bm > 128 && x.obm <= 0) bm = rup(cdiv(bm, 2), 128);
@@ -601,6 +615,7 @@ int build_s1(const EdgeCtx& x, northup_stats* st) {
   }
   const uint64_t bytes = bytes_of(bm, bn, bk);
   const int arena = B.add_buf(B_ARENA, x.hbm_node, w, bytes);
+  set_scratch(B.P, w, arena, bytes, leaf_scratch(bm, bn, x.kc));
   const int64_t ldAs = pad_ld(K), ldC = pad_ld(bn), ldB = pad_ld(bn);
   int64_t off = 0, offAs[2], offC[2], offB[kSlots];
   for (int i = 0; i < 2; ++i) { offAs[i] = off; off += bm * ldAs; }
@@ -656,9 +671,11 @@ int build_in_hbm(Builder& B, int node, int64_t M, int64_t N, int64_t K, int A, i
   uint64_t bytes = 0;
   if (!a_ok) bytes += 4ull * M * ldA;
   if (!b_ok) bytes += 4ull * K * ldB;
-  int arena = -1;
+  const uint64_t scr = leaf_scratch(M, N, B.P->kc);
+  bytes += scr;
   int64_t offA = 0, offB = a_ok ? 0 : M * ldA;
-  if (bytes) arena = B.add_buf(B_ARENA, node, 0, bytes);
+  const int arena = B.add_buf(B_ARENA, node, 0, bytes);
+  set_scratch(B.P, 0, arena, bytes, scr);
   int a = A, b = Bb;
   int64_t la = K, lb = N, oa = 0, ob = 0;
   if (!a_ok) {
@@ -719,7 +736,8 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
   }
   auto hbm_bytes = [&](int64_t bm, int64_t bn) {
     return 4ull * (uint64_t(bm) * pad_ld(bn) +
-                   uint64_t(kSlots) * (uint64_t(bm) * pad_ld(bk) + uint64_t(bk) * pad_ld(bn)));
+                   uint64_t(kSlots) * (uint64_t(bm) * pad_ld(bk) + uint64_t(bk) * pad_ld(bn))) +
+           leaf_scratch(bm, bn, kc);
   };
   int64_t bm = mmax, bn = nmax;
   while (hbm_bytes(bm, bn) > cap) {
@@ -740,7 +758,10 @@ int build_file_root(Builder& B, const northup_tree_s* t, int staging, const std:
                 (unsigned long long)dcap);
   const int dram = B.add_buf(B_DRAM, staging, -1, 4ull * (R * panel_e + cstage_e));
   std::vector<int> arena(G);
-  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+  for (int w = 0; w < G; ++w) {
+    arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+    set_scratch(B.P, w, arena[w], hbm_bytes(bm, bn), leaf_scratch(bm, bn, kc));
+  }
   const int64_t ldC = pad_ld(bn), ldA = pad_ld(bk), ldB = pad_ld(bn);
   const int64_t offC = 0;
   int64_t offSA[kSlots], offSB[kSlots];
@@ -845,7 +866,8 @@ int build_file_direct(Builder& B, const northup_tree_s* t, const std::vector<int
   auto lda_of = [&](int64_t kk) { return bk4 ? kk : pad_ld(kk); };
   auto hbm_bytes = [&](int64_t bm, int64_t bn) {
     const int64_t ldb = (bn == N && N % 4 == 0) ? bn : pad_ld(bn);
-    return 4ull * (uint64_t(bm) * pad_ld(bn) + uint64_t(kSlots) * (uint64_t(bm) * lda_of(bk) + uint64_t(bk) * ldb));
+    return 4ull * (uint64_t(bm) * pad_ld(bn) + uint64_t(kSlots) * (uint64_t(bm) * lda_of(bk) + uint64_t(bk) * ldb)) +
+           leaf_scratch(bm, bn, kc);
   };
   int64_t bm = mmax, bn = nmax;
   while (hbm_bytes(bm, bn) > cap) {
@@ -855,7 +877,10 @@ int build_file_direct(Builder& B, const northup_tree_s* t, const std::vector<int
   }
   const int64_t ldC = pad_ld(bn), ldBs = (bn == N && N % 4 == 0) ? bn : pad_ld(bn);
   std::vector<int> arena(G);
-  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+  for (int w = 0; w < G; ++w) {
+    arena[w] = B.add_buf(B_ARENA, hbm[w], w, hbm_bytes(bm, bn));
+    set_scratch(B.P, w, arena[w], hbm_bytes(bm, bn), leaf_scratch(bm, bn, kc));
+  }
   st->bm = bm;
   st->bn = bn;
   st->bk = bk;
@@ -927,7 +952,8 @@ int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M
   partition_grid(G, M, N, &Pr, &Pc);
   const int64_t bk = std::min<int64_t>(std::max<int64_t>(kc, 4), rup(K, 4));
   auto bytes = [&](int64_t tm, int64_t tn) {
-    return 4ull * (2ull * tm * pad_ld(tn) + uint64_t(kSlots) * (uint64_t(tm) * pad_ld(bk) + uint64_t(bk) * pad_ld(tn)));
+    return 4ull * (2ull * tm * pad_ld(tn) + uint64_t(kSlots) * (uint64_t(tm) * pad_ld(bk) + uint64_t(bk) * pad_ld(tn))) +
+           leaf_scratch(tm, tn, kc);
   };
   // `tiles` (default 2) tiles per sibling: split each sibling's region, one
   // factor of 2 at a time, in the direction that adds fewer PCIe bytes (every
@@ -947,6 +973,7 @@ int choose_queue(const northup_tree_s* t, const std::vector<int>& hbm, int64_t M
       q->Tr = cdiv(M, tm);
       q->Tc = cdiv(N, tn);
       q->arena_bytes = bytes(tm, tn);
+      q->scratch_bytes = leaf_scratch(tm, tn, kc);
       return 0;
     }
     if (tm <= 8 && tn <= 8)
@@ -1114,7 +1141,10 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     rc = choose_queue(t, hbm, M, N, K, P.kc, o ? o->queue_tiles : 0, &q);
     if (rc) return rc;
     std::vector<int> arena(G);
-    for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, q.arena_bytes);
+    for (int w = 0; w < G; ++w) {
+      arena[w] = B.add_buf(B_ARENA, hbm[w], w, q.arena_bytes);
+      set_scratch(&P, w, arena[w], q.arena_bytes, q.scratch_bytes);
+    }
     auto queues = queue_initial(G, q);
     std::vector<int64_t> pctr(G, 0), done(G, 0);
     for (bool more = true; more;) {

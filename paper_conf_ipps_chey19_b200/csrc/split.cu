@@ -126,6 +126,7 @@ int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64
   const int Kp = (Kl + 31) / 32 * 32;
   const int grid = static_cast<int>(std::min<int64_t>((M + 7) / 8, 32LL * sms));
   split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea);
+  count_launches(1);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_a launch: %s", cudaGetErrorString(e));
 }
@@ -137,7 +138,10 @@ int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64
   const int Kp = (Kl + 31) / 32 * 32;
   cudaError_t e = cudaMemsetAsync(bmax, 0, sizeof(unsigned) * N, s);
   if (e != cudaSuccess) return fail(NU_ECUDA, "split_b memset: %s", cudaGetErrorString(e));
-  if (Kl > 0) colmax_kernel<<<dim3((N + 255) / 256, (Kl + 255) / 256), 256, 0, s>>>(B, ldb, Kl, N, bmax);
+  if (Kl > 0) {
+    colmax_kernel<<<dim3((N + 255) / 256, (Kl + 255) / 256), 256, 0, s>>>(B, ldb, Kl, N, bmax);
+    count_launches(1);
+  }
   static bool configured[kMaxDevices];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -148,6 +152,7 @@ int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64
   }
   const int threads = std::min(1024, std::max(64, (N / 8 + 31) / 32 * 32));
   split_b_kernel<<<Kp, threads, 4 * static_cast<size_t>(N), s>>>(B, ldb, Kl, N, bmax, dst, ldd, eb);
+  count_launches(1);
   e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_b launch: %s", cudaGetErrorString(e));
 }

@@ -11,8 +11,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
 
 
-def run_bench(*args, timeout=600):
+def run_bench(*args, timeout=600, torchrun_env=True):
     env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    if not torchrun_env:
+        for k in ("WORLD_SIZE", "RANK", "LOCAL_RANK"):
+            env.pop(k, None)
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), *args], capture_output=True,
                        text=True, timeout=timeout, cwd=ROOT, env=env)
     assert r.returncode == 0, r.stderr[-2000:]
@@ -36,19 +39,42 @@ def test_ours_quick_json_line():
     d = run_bench("--quick", "--steps", "2", "--warmup", "3", "--cpu-budget", "1")
     assert d["metric"] == METRIC and d["unit"] == "TFLOP/s" and d["n_gpus"] == 1
     assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["e2e"]["unit"] == "TFLOP/s"
+    assert d["in_hbm"]["value"] > 0 and "slowdown_pct_vs_in_hbm" in d
     M, N, K = d["config"]["M"], d["config"]["N"], d["config"]["K"]
     assert d["e2e"]["h2d_bytes_per_step"] >= 4 * (M * K + K * N)        # every A/B byte crosses PCIe
     assert d["e2e"]["d2h_bytes_per_step"] == 4 * M * N
     assert d["gpu_launches"] > 0
     rl = d["roofline"]
-    assert rl["bound"] == "tensor" and 0 < rl["frac"] < 1.1 and rl["peak"] > 0
+    assert rl["bound"] == "tensor" and 0 < rl["frac"] < 1.2 and rl["peak"] > 0
+    assert rl["kernel"] == "nu::leaf::x3::leaf_x3_kernel" and rl["launches_timed"] > 0
     er = d["e2e_roofline"]
-    assert er["bound"] in ("tensor", "pcie_h2d", "pcie_d2h") and 0 < er["frac"] < 1.1
+    assert er["bound"] in ("tensor", "pcie_h2d", "pcie_d2h") and 0 < er["frac"] < 1.2
     assert d["staging"]["pcie_measured"]["h2d_gbs"] > 1
     assert d["parity"]["bitwise_in_hbm_vs_out_of_core"] and d["parity"]["bitwise_tree_vs_leaf"]
     assert d["parity"]["oracle_ok"] and d["cpu_baseline"]["kind"] == "oracle"
+    assert d["cpu_baseline"]["single_core_value"] > 0 and d["cpu_baseline"]["numa_nodes"] >= 1
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
     assert d["cfg2_in_hbm_tflops"] > 0 and "slowdown_pct_vs_cfg2_in_hbm" in d
+    assert 0 <= d["runtime_overhead"]["plan_pct_of_step"] < 100
+    assert 0 < d["breakdown"]["compute_pct"] <= 100
+    assert set(d["in_hbm"]["split_variants_tflops"]) == {"npass4", "npass1"}
+
+
+@pytest.mark.gpu
+def test_ours_spawns_ranks_for_gpus_n():
+    """`python bench.py --gpus 4` outside torchrun starts the 4 ranks itself
+    (here 4 processes share the one GPU: --device-mod 1, gloo)."""
+    d = run_bench("--gpus", "4", "--quick", "--steps", "2", "--warmup", "3", "--device-mod", "1",
+                  "--dist-backend", "gloo", "--no-cpu-baseline", timeout=900, torchrun_env=False)
+    assert d["n_gpus"] == 4 and d["value"] > 0 and d["config"]["workload"].startswith("cfg4")
+
+
+def test_gpus_mismatch_with_world_size_fails_loudly():
+    """--gpus N under a launcher that started a different number of ranks."""
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2"], capture_output=True,
+                       text=True, timeout=120, cwd=ROOT, env=env)
+    assert r.returncode == 2 and "WORLD_SIZE=1" in r.stderr
 
 
 def test_ooc_roofline_terms():

@@ -25,7 +25,7 @@ def file_tree(G, cap=0, staging_cap=0):
     (300, 200, 130, 1, 0, 0, "int"),
     (512, 768, 1024, 1, 0, 256, "uniform"),
     (640, 900, 1500, 2, 0, 512, "uniform"),
-    (1000, 1200, 3000, 2, 6_000_000, 1024, "int"),      # capacity -> several C-block rounds
+    (1000, 1200, 3000, 2, 8_000_000, 1024, "int"),      # capacity -> several C-block rounds
 ])
 def test_file_root_gemm(tmp_path, M, N, K, G, cap, panel, kind):
     A = nugen.fill(M, K, 6, 1, kind)
