@@ -265,6 +265,11 @@ int northup_leaf_gemm(const float* A, int64_t lda, const float* B, int64_t ldb, 
 #define NU_OP_ZERO 2
 #define NU_OP_IO_READ 3  /* file -> DRAM staging (pread), host I/O thread */
 #define NU_OP_IO_WRITE 4 /* DRAM staging -> file (pwrite), host I/O thread */
+#define NU_OP_SPLIT_B 6  /* split a resident B region in place into the leaf's fp16 hi/lo operand
+                            (R22): dst_* = the region (rows = K rows of one panel,
+                            cols = N), c_buf / c_off = its column exponents (ints); a LEAF op
+                            whose src_buf >= 0 reads such a B, exponents at src_buf / src_off,
+                            `rows` = exponents per K panel */
 #define NU_OP_STENCIL 5  /* HotSpot-2D leaf (northup_hotspot): a_* = temperature in, b_* = power,
                             c_* = temperature out, all shaped like the m x n window; k = iterations;
                             src_off / dst_off = the window's grid row / column; rows x cols = grid */

@@ -24,6 +24,7 @@ NU_FILE, NU_HOST, NU_HBM, NU_SMEM = 0, 1, 2, 3
 NU_PROC_NONE, NU_PROC_SM100 = 0, 1
 NU_SCHED_AUTO, NU_SCHED_S1, NU_SCHED_S2, NU_SCHED_QUEUE = 0, 1, 2, 3
 NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO, NU_OP_IO_READ, NU_OP_IO_WRITE, NU_OP_STENCIL = 0, 1, 2, 3, 4, 5
+NU_OP_SPLIT_B = 6
 STREAM_NAMES = {0: "h2d", 1: "compute", 2: "d2h", 3: "io", 4: "d2d"}
 STATUS_NAMES = {0: "NU_OK", -1: "NU_EINVAL", -2: "NU_ENOMEM", -3: "NU_EIO", -4: "NU_ECUDA",
                 -5: "NU_ENCCL", -6: "NU_ESTATE", -7: "NU_ENOTSUP"}

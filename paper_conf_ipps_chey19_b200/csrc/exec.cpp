@@ -268,12 +268,25 @@ static int run_worker(RunCtx& c, int wi, double* busy, cudaGraphExec_t* capture_
       LeafCall lc{};
       lc.A = a, lc.lda = op.lda, lc.B = b, lc.ldb = op.ldb, lc.C = cc, lc.ldc = op.ldc;
       lc.M = op.m, lc.N = op.n, lc.K = op.k, lc.accumulate = op.accumulate, lc.panel = P.kc, lc.npass = P.npass;
+      if (op.src_buf >= 0) {   // B split in place by earlier NU_OP_SPLIT_B ops
+        lc.eb_presplit = reinterpret_cast<const int*>(c.base[op.src_buf] + op.src_off * 4);
+        lc.eb_stride = op.rows;
+      }
       if (wi < static_cast<int>(P.scr_buf.size()) && P.scr_buf[wi] >= 0) {
         lc.scratch = c.base[P.scr_buf[wi]] + P.scr_off[wi];
         lc.scratch_bytes = P.scr_bytes[wi];
       }
       lc.stream = s;
       int rc = leaf_run(lc);
+      if (rc) return rc;
+    } else if (op.op == NU_OP_SPLIT_B) {
+      if (wi >= static_cast<int>(P.scr_buf.size()) || P.scr_buf[wi] < 0)
+        return fail(NU_ESTATE, "split op without a leaf scratch");
+      float* bp = reinterpret_cast<float*>(c.base[op.dst_buf] + op.dst_off * 4);
+      int* eb = reinterpret_cast<int*>(c.base[op.c_buf] + op.c_off * 4);
+      unsigned* bmax = reinterpret_cast<unsigned*>(c.base[P.scr_buf[wi]] + P.scr_off[wi]);
+      int rc = leaf::split_b_launch(bp, op.dst_ld, static_cast<int>(op.rows), static_cast<int>(op.cols), bp,
+                                    op.dst_ld, eb, bmax, s);
       if (rc) return rc;
     } else if (op.op == NU_OP_STENCIL) {
       const float* tin = reinterpret_cast<const float*>(c.base[op.a_buf] + op.a_off * 4);

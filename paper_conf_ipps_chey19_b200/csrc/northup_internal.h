@@ -189,6 +189,11 @@ struct LeafCall {
   int* events_used = nullptr;
 };
 int leaf_run(const LeafCall& c);
+namespace leaf {
+// In-place or out-of-place split of a B panel (split.cu); bmax: N words of scratch.
+int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64_t ldd, int* eb,
+                   unsigned* bmax, cudaStream_t s);
+}  // namespace leaf
 uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit);
 // Scratch of the largest leaf op over an m x n C block (256-B rounded).
 inline uint64_t leaf_scratch(int64_t m, int64_t n, int64_t panel) {

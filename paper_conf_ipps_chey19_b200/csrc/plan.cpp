@@ -28,10 +28,11 @@ namespace nu {
 
 
 // Nominal planning constants: the leaf's useful flop rate on
-// one B200 under its power cap (v3, measured 320-336 TF/s) and the measured
-// PCIe Gen5 x16 per-direction bandwidth.  Only used to size the drain tail.
-static constexpr double kPlanFlops = 320e12;
-static constexpr double kPlanPcie = 52e9;
+// one B200 under its power cap (x3 leaf, measured 390 TF/s in-HBM on 32768^3)
+// and the PCIe Gen5 x16 per-direction bandwidth measured with both directions
+// busy (49-50 GB/s).  Only used to size the drain tail.
+static constexpr double kPlanFlops = 390e12;
+static constexpr double kPlanPcie = 49e9;
 
 int partition_grid(int G, int64_t M, int64_t N, int* Pr, int* Pc) {
   if (G <= 0) return fail(NU_EINVAL, "G must be positive");
@@ -109,6 +110,35 @@ northup_op make_leaf(int worker, int a, int64_t a_off, int64_t lda, int b, int64
   return o;
 }
 
+// In-place split of a resident B region (one K panel: rows x cols at off, ld),
+// column exponents to (ebuf, eoff).  Runs on the compute stream, in order with
+// the leaf ops that use the worker's scratch.
+northup_op make_split_b(int worker, int buf, int64_t off, int64_t ld, int64_t rows, int64_t cols, int ebuf,
+                        int64_t eoff) {
+  northup_op o{};
+  o.op = NU_OP_SPLIT_B;
+  o.worker = worker;
+  o.stream = S_COMP;
+  o.dst_buf = buf;
+  o.dst_off = off;
+  o.dst_ld = ld;
+  o.rows = rows;
+  o.cols = cols;
+  o.c_buf = ebuf;
+  o.c_off = eoff;
+  o.src_buf = o.a_buf = o.b_buf = -1;
+  return o;
+}
+
+// Mark a leaf op as reading a pre-split B (exponents at ebuf/eoff, `stride`
+// per K panel).
+northup_op with_presplit_b(northup_op o, int ebuf, int64_t eoff, int64_t stride) {
+  o.src_buf = ebuf;
+  o.src_off = eoff;
+  o.rows = stride;
+  return o;
+}
+
 struct EdgeCtx {
   Builder* B;
   int worker;
@@ -144,8 +174,9 @@ uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, i
     e += static_cast<uint64_t>(kSlots) *
          (static_cast<uint64_t>(bm) * pad_ld(bk) + static_cast<uint64_t>(bk) * pad_ld(bn));
   if (tail > 0)
-    e += static_cast<uint64_t>(tail) * pad_ld(bn) +                          // B tail
-         static_cast<uint64_t>(kSlots) * sr * pad_ld(tail);                  // A strips
+    e += static_cast<uint64_t>(rup(tail, 32)) * pad_ld(bn) +                 // B tail (split in place)
+         static_cast<uint64_t>(kSlots) * sr * pad_ld(tail) +                 // A strips
+         static_cast<uint64_t>(cdiv(tail, kc)) * pad_ld(bn);                 // B tail column exponents
   return e * 4 + leaf_scratch(bm, bn, kc);                                   // + leaf scratch
 }
 
@@ -256,6 +287,7 @@ struct S2Layout {
   int arena = -1;
   int64_t ldC = 0, ldA = 0, ldBs = 0, ldAt = 0;
   int64_t offC = 0, offBT = 0;
+  int64_t offEB = -1;   // B tail column exponents [panel][ldBs] (ints), when the tail is split in place
   int64_t offSA[kSlots] = {}, offSB[kSlots] = {}, offAT[kSlots] = {};
 };
 
@@ -279,13 +311,46 @@ S2Layout layout_s2(Builder& B, const S2Shape& s, int hbm_node, int w, int64_t K)
   }
   if (s.tail > 0) {
     L.offBT = off;
-    off += s.tail * L.ldBs;
+    off += rup(s.tail, 32) * L.ldBs;
     for (int i = 0; i < kSlots; ++i) {
       L.offAT[i] = off;
       off += s.sr * L.ldAt;
     }
+    if (s.bn <= kLeafMaxN) L.offEB = off;   // wider tails are split by each leaf call instead
+    off += cdiv(s.tail, B.P->kc) * L.ldBs;
   }
   return L;
+}
+
+// The B tail is resident for the whole tail phase and read by every strip's
+// leaf: split each loaded piece (one K panel) once, in place, instead of in
+// every leaf call (R22).  Pieces are bk = k_chunk rows.
+void emit_tail_split(Builder& B, int w, const S2Layout& L, const S2Shape& s, int64_t bn, int64_t kt0,
+                     int64_t kk) {
+  if (L.offEB < 0) return;
+  const int64_t kc = B.P->kc, p = kt0 / kc;
+  for (int64_t k = kt0; k < kt0 + kk; k += kc) {   // a piece is a whole number of panels
+    const int64_t rows = std::min(kc, kt0 + kk - k), pp = k / kc;
+    (void)p;
+    B.emit(make_split_b(w, L.arena, L.offBT + k * L.ldBs, L.ldBs, rows, bn, L.arena, L.offEB + pp * L.ldBs),
+           {{L.arena, L.offBT + k * L.ldBs, L.ldBs, rup(rows, 32), bn, true},
+            {L.arena, L.offEB + pp * L.ldBs, L.ldBs, 1, bn, true}});
+  }
+}
+
+void emit_tail_leaf(Builder& B, int w, const S2Layout& L, const S2Shape& s, int ar, int64_t ao, int64_t lda,
+                    int64_t co, int64_t ldc, int64_t rr, int64_t bn, int acc) {
+  northup_op o = make_leaf(w, ar, ao, lda, L.arena, L.offBT, L.ldBs, ar, co, ldc, rr, bn, s.tail, acc);
+  if (L.offEB >= 0) {
+    o = with_presplit_b(o, L.arena, L.offEB, L.ldBs);
+    B.emit(o, {{ar, ao, lda, rr, s.tail, false},
+               {L.arena, L.offBT, L.ldBs, s.tail, bn, false},
+               {L.arena, L.offEB, L.ldBs, cdiv(s.tail, B.P->kc), bn, false},
+               {ar, co, ldc, rr, bn, true}});
+  } else {
+    B.emit(o, {{ar, ao, lda, rr, s.tail, false}, {L.arena, L.offBT, L.ldBs, s.tail, bn, false},
+               {ar, co, ldc, rr, bn, true}});
+  }
 }
 
 // Rows of the graded drain strips (full strips while more than two remain,
@@ -339,6 +404,7 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
                {{x.Bb, k0 * x.ldb + gc, x.ldb, kk, bn, false},
                 {arena, offBT + (k0 - kmain) * ldBs, ldBs, kk, bn, true}});
         st->bytes_h2d += static_cast<uint64_t>(kk) * bn * 4;
+        emit_tail_split(B, w, L, s, bn, k0 - kmain, kk);
       };
       for (int64_t p = 0; p < npan; ++p, ++panel_it) {
         const int sl = panel_it % kSlots;
@@ -392,11 +458,7 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
                  {{x.A, (gr + r) * x.lda + kmain, x.lda, rr, s.tail, false},
                   {arena, offAT[sl], ldAt, rr, s.tail, true}});
           st->bytes_h2d += static_cast<uint64_t>(rr) * s.tail * 4;
-          B.emit(make_leaf(w, arena, offAT[sl], ldAt, arena, offBT, ldBs, arena, offC + r * ldC, ldC,
-                           rr, bn, s.tail, kmain > 0 ? 1 : 0),
-                 {{arena, offAT[sl], ldAt, rr, s.tail, false},
-                  {arena, offBT, ldBs, s.tail, bn, false},
-                  {arena, offC + r * ldC, ldC, rr, bn, true}});
+          emit_tail_leaf(B, w, L, s, arena, offAT[sl], ldAt, offC + r * ldC, ldC, rr, bn, kmain > 0 ? 1 : 0);
           st->leaf_launches++;
           B.emit(make_copy(w, S_D2H, arena, offC + r * ldC, ldC, x.C, (gr + r) * x.ldc + gc, x.ldc, rr,
                            bn),
@@ -522,6 +584,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
                        [&](const EdgeCtx& x) { return k0 * ldb + x.ac0 + j0; });
         load(sb);
         pull(sb);
+        for (int w = 0; w < G; ++w) emit_tail_split(B, w, L[w], s, bn, k0 - kmain, kk);
       };
       for (int64_t p = 0; p < npan; ++p, ++panel_it) {
         const int sl = panel_it % kSlots;
@@ -569,10 +632,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
           for (int w = 0; w < G; ++w) {
             const int ar = L[w].arena;
             const int64_t co = Y.offC + r * Y.ldC;
-            B.emit(make_leaf(w, ar, Y.offAT[sl], Y.ldAt, ar, Y.offBT, Y.ldBs, ar, co, Y.ldC, rr, bn, s.tail,
-                             kmain > 0 ? 1 : 0),
-                   {{ar, Y.offAT[sl], Y.ldAt, rr, s.tail, false}, {ar, Y.offBT, Y.ldBs, s.tail, bn, false},
-                    {ar, co, Y.ldC, rr, bn, true}});
+            emit_tail_leaf(B, w, L[w], s, ar, Y.offAT[sl], Y.ldAt, co, Y.ldC, rr, bn, kmain > 0 ? 1 : 0);
             st->leaf_launches++;
             const int64_t dst = (xs[w].ar0 + i0 + r) * ldc + xs[w].ac0 + j0;
             B.emit(make_copy(w, S_D2H, ar, co, Y.ldC, x0.C, dst, ldc, rr, bn),

@@ -109,17 +109,30 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
         else:
             mem.append(np.full(b["bytes"] // 4, np.nan))
 
-    def view(buf, off, ld, rows, cols):
-        return np.lib.stride_tricks.as_strided(mem[buf][off:], shape=(rows, cols),
+    # NU_OP_SPLIT_B rewrites a resident B region in place into the leaf's split
+    # form: model that as moving the values to a shadow copy (the raw region
+    # becomes NaN) which only pre-split leaf ops read; a later copy into the
+    # region destroys the split form (NaN in the shadow), as on the GPU.
+    shadow = [np.full(len(x), np.nan) for x in mem]
+
+    def view(buf, off, ld, rows, cols, m=None):
+        m = mem if m is None else m
+        return np.lib.stride_tricks.as_strided(m[buf][off:], shape=(rows, cols),
                                                strides=(ld * 8, 8), writeable=True)
 
     def run(op):
         if op["op"] in (nu.NU_OP_COPY, nu.NU_OP_IO_READ, nu.NU_OP_IO_WRITE):
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
                 view(op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
+            view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], shadow)[...] = np.nan
+        elif op["op"] == nu.NU_OP_SPLIT_B:
+            src = view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])
+            view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], shadow)[...] = src
+            src[...] = np.nan
         elif op["op"] == nu.NU_OP_LEAF:
             a = view(op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
-            b = view(op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"])
+            b = view(op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"],
+                     shadow if op["src_buf"] >= 0 else None)
             c = view(op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])
             prod = a @ b
             c[...] = (c + prod) if op["accumulate"] else prod
@@ -335,7 +348,9 @@ def test_shared_staging_plan_replays_exactly(M, N, K, G, cap, kc):
     assert s["shared_staging"] == 1
     ops = p.ops()
     cross = [o for o in ops for d in o["deps"] if ops[d]["worker"] != o["worker"]]
-    assert cross and all(o["stream"] in (4, 0) for o in cross)   # pulls (and slot reuse by loads)
+    # pulls, slot reuse by loads, and the in-place split of the B tail after the
+    # peers pulled their pieces from it (WAR)
+    assert cross and all(o["stream"] in (4, 0) or o["op"] == nu.NU_OP_SPLIT_B for o in cross)
     for seed in range(4):
         C = simulate(p, A, B, M, N, K, rng=random.Random(seed))
         assert np.array_equal(C, ref), f"order seed {seed} broke a dependency"
@@ -404,8 +419,13 @@ def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
     def mem(w, i):
         return strips[w][bufs[i]["kind"]] if bufs[i]["kind"] < 3 else arenas[i]
 
-    def view(w, buf, off, ld, rows, cols):
-        return np.lib.stride_tricks.as_strided(mem(w, buf)[off:], shape=(rows, cols),
+    shadows = {}
+
+    def view(w, buf, off, ld, rows, cols, shadow=False):
+        base = mem(w, buf)
+        if shadow:
+            base = shadows.setdefault(id(base), np.full(len(base), np.nan))
+        return np.lib.stride_tricks.as_strided(base[off:], shape=(rows, cols),
                                                strides=(ld * 8, 8), writeable=True)
 
     queues = {}
@@ -420,9 +440,14 @@ def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
         if op["op"] == nu.NU_OP_COPY:
             view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
                 view(w, op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
+            view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], True)[...] = np.nan
+        elif op["op"] == nu.NU_OP_SPLIT_B:
+            src = view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])
+            view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], True)[...] = src
+            src[...] = np.nan
         elif op["op"] == nu.NU_OP_LEAF:
             a = view(w, op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
-            b = view(w, op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"])
+            b = view(w, op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"], op["src_buf"] >= 0)
             c = view(w, op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])
             c[...] = (c + a @ b) if op["accumulate"] else a @ b
         done.add(i)
