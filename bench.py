@@ -577,6 +577,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                 "drain_tail_k": ooc_stats.get("tail_k"), "drain_strips": ooc_stats.get("strips"),
                 "hbm_footprint_bytes": ooc_stats.get("hbm_peak_bytes"),
                 "numa": numa,
+                "links_at_finalize": t.link_info(),
                 "l2": "inputs (>= 4 GiB each) exceed the 126 MB L2; no flush needed",
                 "value_basis": "out-of-core: northup_gemm from pinned HOST buffers through the tree, every "
                                "H2D/D2H inside the step; CUDA events on the calling stream bracketing the "

@@ -142,6 +142,22 @@ int northup_get_node_info(northup_tree_t t, int node, northup_node_info* info);
  * NUL-terminated string of at most n bytes; *n_needed (may be NULL) gets the
  * full length + 1. */
 int northup_tree_print(northup_tree_t t, char* buf, size_t n, size_t* n_needed);
+/* errno of the last failed file read / write / fdatasync of any FILE path in
+ * this process (0 for an unexpected end of file); a failed call returns
+ * NU_EIO and northup_last_error() names the operation.  Testing: the env var
+ * NORTHUP_IO_FAULT="<read|write>:<eio|enospc|short|eof>:<n>" makes the n-th
+ * pread (pwrite) of the process fail with EIO / ENOSPC, move half the bytes
+ * (a short transfer, which the library completes) or return 0. */
+int northup_last_io_errno(void);
+/* What finalize measured about the tree's links (exec.cpp): *pcie_gbs = the
+ * slowest local GPU's host->HBM rate with every local link busy in both
+ * directions (64 MiB pinned copies; 0 = not measured: HBM root, no GPU worker,
+ * or NORTHUP_CALIBRATE=0 — the planner then uses its nominal 49 GB/s);
+ * *p2p_ok = 1 when every pair of distinct HBM devices has peer access (else
+ * shared staging, S§8(f) NEXT-1, is not planned); *numa_bound = number of local
+ * workers whose threads are bound to their GPU's NUMA node.  NU_ESTATE before
+ * finalize. */
+int northup_tree_link_info(northup_tree_t t, double* pcie_gbs, int* p2p_ok, int* numa_bound);
 
 /* ---------------------------------------- unified data API (Table I) */
 /* alloc(size, tree_node): pinned portable host memory at a NU_HOST node, a

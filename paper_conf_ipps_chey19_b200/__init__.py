@@ -129,6 +129,7 @@ _SIGS = {
     "northup_get_num_nodes": [_vp, _pint],
     "northup_get_node_info": [_vp, _int, ctypes.POINTER(NodeInfo)],
     "northup_tree_print": [_vp, ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)],
+    "northup_tree_link_info": [_vp, _vp, _vp, _vp],
     "northup_alloc": [_vp, _u64, _int, _vp],
     "northup_tree_set_file_dir": [_vp, ctypes.c_char_p],
     "northup_wrap_host": [_vp, _int, _vp, _u64, _vp],
@@ -185,6 +186,14 @@ def lib() -> ctypes.CDLL:
         L.northup_last_error.restype = ctypes.c_char_p
         _lib = L
     return _lib
+
+
+def last_io_errno() -> int:
+    """northup_last_io_errno: errno of the last failed file I/O (0: end of file)."""
+    f = lib().northup_last_io_errno
+    f.argtypes = []
+    f.restype = ctypes.c_int
+    return int(f())
 
 
 def last_error() -> str:
@@ -413,6 +422,12 @@ class Tree:
 
     def set_file_dir(self, d: str) -> None:
         check(lib().northup_tree_set_file_dir(self.handle, d.encode()))
+
+    def link_info(self) -> dict:
+        """northup_tree_link_info: what finalize measured (PCIe, P2P, NUMA binding)."""
+        g, p, n = ctypes.c_double(), ctypes.c_int(), ctypes.c_int()
+        check(lib().northup_tree_link_info(self.handle, ctypes.byref(g), ctypes.byref(p), ctypes.byref(n)))
+        return {"pcie_gbs": g.value, "p2p_ok": bool(p.value), "numa_bound_workers": n.value}
 
     def finalize(self) -> None:
         check(lib().northup_tree_finalize(self.handle))

@@ -14,7 +14,11 @@
 //                                     issued, then cudaEventSynchronize.
 // All dependencies point backwards in plan order, which every thread follows,
 // so the waits cannot deadlock.
+#include <ctype.h>
 #include <errno.h>
+#include <pthread.h>
+#include <sched.h>
+#include <stdio.h>
 #include <fcntl.h>
 #include <string.h>
 #include <unistd.h>
@@ -22,6 +26,7 @@
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
+#include <memory>
 #include <mutex>
 #include <thread>
 
@@ -44,6 +49,120 @@ struct WorkerState {
 
 namespace nu {
 
+// CPUs of the NUMA node the GPU's PCIe device sits on (empty when the host
+// does not say: one node, or numa_node = -1).
+static std::vector<int> gpu_numa_cpus(int device) {
+  std::vector<int> cpus;
+  char bus[32] = {};
+  if (cudaDeviceGetPCIBusId(bus, sizeof bus, device) != cudaSuccess) {
+    cudaGetLastError();
+    return cpus;
+  }
+  for (char* p = bus; *p; ++p) *p = static_cast<char>(tolower(*p));
+  char path[128];
+  snprintf(path, sizeof path, "/sys/bus/pci/devices/%s/numa_node", bus);
+  FILE* f = fopen(path, "r");
+  int node = -1;
+  if (f) {
+    if (fscanf(f, "%d", &node) != 1) node = -1;
+    fclose(f);
+  }
+  if (node < 0) return cpus;
+  snprintf(path, sizeof path, "/sys/devices/system/node/node%d/cpulist", node);
+  f = fopen(path, "r");
+  if (!f) return cpus;
+  char list[4096] = {};
+  if (fgets(list, sizeof list, f)) {
+    for (char* tok = strtok(list, ",\n"); tok; tok = strtok(nullptr, ",\n")) {
+      int lo = 0, hi = 0;
+      if (sscanf(tok, "%d-%d", &lo, &hi) == 2)
+        for (int c = lo; c <= hi; ++c) cpus.push_back(c);
+      else if (sscanf(tok, "%d", &lo) == 1)
+        cpus.push_back(lo);
+    }
+  }
+  fclose(f);
+  return cpus;
+}
+
+// each worker thread issues its GPU's copies from the CPUs of
+// that GPU's NUMA node (bound at the start of every call).
+void numa_bind_plan(northup_tree_s* t) {
+  t->worker_cpus.assign(t->nodes.size(), {});
+  if (getenv("NORTHUP_NO_NUMA_BIND")) return;
+  for (WorkerState* w : t->workers) t->worker_cpus[w->node] = gpu_numa_cpus(w->device);
+}
+
+void bind_worker_thread(const northup_tree_s* t, int node) {
+  if (node < 0 || node >= static_cast<int>(t->worker_cpus.size()) || t->worker_cpus[node].empty()) return;
+  cpu_set_t set;
+  CPU_ZERO(&set);
+  for (int c : t->worker_cpus[node])
+    if (c >= 0 && c < CPU_SETSIZE) CPU_SET(c, &set);
+  pthread_setaffinity_np(pthread_self(), sizeof set, &set);
+}
+
+// The planner's PCIe term (S§8(d) "BW_e = the concurrently measured per-GPU
+// bandwidth with all links active"): every local GPU copies 64 MiB H2D and
+// 64 MiB D2H at once, twice; the slowest GPU's H2D rate of the second round.
+// Skipped for HBM roots (no host edge) and with NORTHUP_CALIBRATE=0.
+int calibrate_pcie(northup_tree_s* t) {
+  t->pcie_gbs = 0.0;
+  const char* env = getenv("NORTHUP_CALIBRATE");
+  if ((env && env[0] == '0') || t->workers.empty() || t->nodes[0].storage == NU_HBM) return 0;
+  const size_t bytes = 64ull << 20;
+  const size_t W = t->workers.size();
+  std::vector<void*> hin(W, nullptr), hout(W, nullptr), din(W, nullptr), dout(W, nullptr);
+  std::vector<cudaEvent_t> ev(4 * W, nullptr);
+  int rc = 0;
+  for (size_t i = 0; i < W && !rc; ++i) {
+    cudaSetDevice(t->workers[i]->device);
+    if (cudaHostAlloc(&hin[i], bytes, cudaHostAllocPortable) != cudaSuccess ||
+        cudaHostAlloc(&hout[i], bytes, cudaHostAllocPortable) != cudaSuccess ||
+        cudaMalloc(&din[i], bytes) != cudaSuccess || cudaMalloc(&dout[i], bytes) != cudaSuccess)
+      rc = 1;
+    for (int k = 0; k < 4 && !rc; ++k)
+      if (cudaEventCreate(&ev[4 * i + k]) != cudaSuccess) rc = 1;
+  }
+  double worst = 0.0;
+  for (int round = 0; round < 2 && !rc; ++round) {
+    for (size_t i = 0; i < W; ++i) {
+      WorkerState* w = t->workers[i];
+      cudaSetDevice(w->device);
+      cudaEventRecord(ev[4 * i + 0], w->streams[S_H2D]);
+      cudaMemcpyAsync(din[i], hin[i], bytes, cudaMemcpyHostToDevice, w->streams[S_H2D]);
+      cudaEventRecord(ev[4 * i + 1], w->streams[S_H2D]);
+      cudaEventRecord(ev[4 * i + 2], w->streams[S_D2H]);
+      cudaMemcpyAsync(hout[i], dout[i], bytes, cudaMemcpyDeviceToHost, w->streams[S_D2H]);
+      cudaEventRecord(ev[4 * i + 3], w->streams[S_D2H]);
+    }
+    worst = 1e30;
+    for (size_t i = 0; i < W; ++i) {
+      cudaSetDevice(t->workers[i]->device);
+      float ms = 0.f;
+      if (cudaEventSynchronize(ev[4 * i + 1]) != cudaSuccess ||
+          cudaEventElapsedTime(&ms, ev[4 * i + 0], ev[4 * i + 1]) != cudaSuccess || ms <= 0.f) {
+        worst = 0.0;
+        break;
+      }
+      worst = std::min(worst, bytes / (ms * 1e-3) / 1e9);
+      cudaEventSynchronize(ev[4 * i + 3]);
+    }
+  }
+  for (size_t i = 0; i < W; ++i) {
+    cudaSetDevice(t->workers[i]->device);
+    if (hin[i]) cudaFreeHost(hin[i]);
+    if (hout[i]) cudaFreeHost(hout[i]);
+    if (din[i]) cudaFree(din[i]);
+    if (dout[i]) cudaFree(dout[i]);
+    for (int k = 0; k < 4; ++k)
+      if (ev[4 * i + k]) cudaEventDestroy(ev[4 * i + k]);
+  }
+  cudaGetLastError();
+  if (!rc && worst > 1.0 && worst < 1e6) t->pcie_gbs = worst;
+  return 0;   // calibration is best effort: the planner falls back to its constant
+}
+
 int finalize_workers(northup_tree_s* t) {
   int ndev = northup_device_count();
   for (const Node& n : t->nodes) {
@@ -65,9 +184,17 @@ int finalize_workers(northup_tree_s* t) {
     // process's progress (cross-sibling waits), which can close a cycle
     preload_kernels();
   }
-  // Shared staging pulls panels from sibling HBM: enable NVLink P2P between
-  // every pair of distinct devices (without it the copies still work, staged
-  // by the driver).
+  // Shared staging pulls panels from sibling HBM: it is planned only when
+  // every pair of distinct HBM devices (local or in peer processes) has P2P
+  // access; enable it between the local ones.
+  t->p2p_ok = true;
+  for (const Node& a : t->nodes)
+    for (const Node& b : t->nodes) {
+      if (a.storage != NU_HBM || b.storage != NU_HBM || a.phys == b.phys) continue;
+      int can = 0;
+      if (cudaDeviceCanAccessPeer(&can, a.phys, b.phys) != cudaSuccess || !can) t->p2p_ok = false;
+    }
+  cudaGetLastError();
   for (WorkerState* a : t->workers)
     for (WorkerState* b : t->workers) {
       if (a->device == b->device) continue;
@@ -79,7 +206,8 @@ int finalize_workers(northup_tree_s* t) {
       if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
       else if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
     }
-  return 0;
+  numa_bind_plan(t);
+  return calibrate_pcie(t);
 }
 
 void destroy_workers(northup_tree_s* t) {
@@ -412,13 +540,17 @@ static int file_block(const northup_buf_s* f, bool write, char* mem, int64_t mem
         off % 4096 == 0)
       fd = f->direct_fd;
     while (bytes) {
-      ssize_t r = write ? pwrite(fd, p, bytes, static_cast<off_t>(off))
-                        : pread(fd, p, bytes, static_cast<off_t>(off));
+      ssize_t r = pio(fd, p, bytes, off, write);
       if (r < 0) {
         if (errno == EINTR) continue;
-        return fail(NU_EIO, "%s(%s): %s", write ? "pwrite" : "pread", f->path.c_str(), strerror(errno));
+        const int err = errno;
+        note_io_errno(err);
+        return fail(NU_EIO, "%s(%s): %s", write ? "pwrite" : "pread", f->path.c_str(), strerror(err));
       }
-      if (r == 0) return fail(NU_EIO, "%s(%s): short transfer", write ? "pwrite" : "pread", f->path.c_str());
+      if (r == 0) {
+        note_io_errno(0);
+        return fail(NU_EIO, "%s(%s): short transfer", write ? "pwrite" : "pread", f->path.c_str());
+      }
       p += r;
       bytes -= static_cast<uint64_t>(r);
       off += static_cast<uint64_t>(r);
@@ -442,7 +574,7 @@ static int file_block(const northup_buf_s* f, bool write, char* mem, int64_t mem
 // opened at all, transfers bounce through a pinned host buffer.
 namespace {
 struct CuFileApi {
-  bool tried = false, ok = false;
+  bool tried = false, ok = false, timed_out = false;
   struct Err {
     int err;
     int cu_err;
@@ -476,8 +608,34 @@ CuFileApi& cufile() {
   g_cufile.write = reinterpret_cast<ssize_t (*)(void*, const void*, size_t, off_t, off_t)>(dlsym(h, "cuFileWrite"));
   if (!g_cufile.driver_open || !g_cufile.handle_register || !g_cufile.read || !g_cufile.write) return g_cufile;
   if (dbg) fprintf(stderr, "[northup] cuFileDriverOpen ...\n");
-  g_cufile.ok = g_cufile.driver_open().err == 0;
-  if (dbg) fprintf(stderr, "[northup] cuFileDriverOpen -> %s\n", g_cufile.ok ? "ok" : "failed");
+  // Watchdog: cuFileDriverOpen has hung on boxes without nvidia-fs; run it on a
+  // detached thread and give up after NORTHUP_CUFILE_TIMEOUT_S (default 20 s),
+  // falling back to the pinned bounce instead of blocking the caller forever.
+  struct OpenState {
+    std::mutex m;
+    std::condition_variable cv;
+    bool done = false, ok = false;
+  };
+  auto st = std::make_shared<OpenState>();
+  auto open_fn = g_cufile.driver_open;
+  std::thread([st, open_fn] {
+    const bool ok = open_fn().err == 0;
+    std::lock_guard<std::mutex> g(st->m);
+    st->done = true;
+    st->ok = ok;
+    st->cv.notify_all();
+  }).detach();
+  const char* to = getenv("NORTHUP_CUFILE_TIMEOUT_S");
+  const double secs = (to && atof(to) > 0) ? atof(to) : 20.0;
+  {
+    std::unique_lock<std::mutex> lk(st->m);
+    st->cv.wait_for(lk, std::chrono::duration<double>(secs), [&] { return st->done; });
+    g_cufile.ok = st->done && st->ok;
+    g_cufile.timed_out = !st->done;
+  }
+  if (dbg)
+    fprintf(stderr, "[northup] cuFileDriverOpen -> %s\n",
+            g_cufile.ok ? "ok" : (g_cufile.timed_out ? "timed out (pinned bounce)" : "failed"));
   return g_cufile;
 }
 
@@ -679,8 +837,11 @@ static int run_io(RunCtx& c, int queue) {
   // O_SYNC semantics of P:242: C is durable when northup_gemm returns.
   if (queue == S_IOW)
     for (size_t b = 0; b < c.file.size(); ++b)
-      if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0)
-        return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(errno));
+      if (c.file[b] && P.bufs[b].kind == B_USER_C && fdatasync(c.file[b]->fd) != 0) {
+        const int err = errno;
+        note_io_errno(err);
+        return fail(NU_EIO, "fdatasync(%s): %s", c.file[b]->path.c_str(), strerror(err));
+      }
   const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   {
     std::lock_guard<std::mutex> g(c.m);
@@ -798,6 +959,7 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
   std::vector<std::string> errs(W + 2);
   std::vector<std::vector<double>> busy(W, std::vector<double>(S_NUM, 0.0));
   auto worker_body = [&](int wi) {
+    bind_worker_thread(t, P.worker_node[wi]);
     cudaGraphExec_t ge = nullptr;
     rcs[wi] = run_worker(ctx, wi, busy[wi].data(), use_graph ? &ge : nullptr);
     if (use_graph) t->graph_execs[wi] = ge;
@@ -829,6 +991,13 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
     }
     for (auto& x : th) x.join();
   }
+  // report the root cause first: an I/O thread's error (the workers then only
+  // see "aborted: file I/O failed")
+  for (int k : {W, W + 1})
+    if (rcs[k]) {
+      if (use_graph) destroy_graphs(t);
+      return fail(rcs[k], "I/O thread %d: %s", k - W, errs[k].c_str());
+    }
   for (int wi = 0; wi <= W + 1; ++wi)
     if (rcs[wi]) {
       if (use_graph) destroy_graphs(t);
@@ -969,6 +1138,7 @@ int execute_queue(northup_tree_s* t, int64_t M, int64_t N, int64_t K, northup_bu
   std::vector<std::thread> th;
   for (int w = 0; w < G; ++w)
     th.emplace_back([&, w] {
+      bind_worker_thread(t, hbm[w]);
       rcs[w] = body(w);
       if (rcs[w]) errs[w] = northup_last_error();
     });

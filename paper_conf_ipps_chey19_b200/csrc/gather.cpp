@@ -7,8 +7,9 @@
 //   * distinct devices: NCCL (loaded with dlopen, so the library has no link
 //     dependency and shares the process's NCCL when PyTorch already loaded
 //     one) — one ncclBroadcast per region inside a group; row-strip regions
-//     (Pc = 1) broadcast straight into place, 2-D regions through a packed
-//     buffer;
+//     (Pc = 1) broadcast straight into place, 2-D regions one at a time
+//     through a region-sized staging buffer (the idle arena, or a buffer
+//     counted against the node's capacity);
 //   * siblings aliasing one device ("virtual siblings", tests): device copies.
 #include <dlfcn.h>
 #include <nccl.h>
@@ -118,53 +119,80 @@ int gather_replicas(northup_tree_s* t, const Plan& P, northup_buf_s* C, northup_
       if (r != ncclSuccess) return nccl_fail(r, "ncclCommInitAll");
       for (auto c : comms) t->nccl_comms.push_back(c);
     }
-    std::vector<void*> packed(G, nullptr);
     if (Pc > 1) {
+      // 2-D regions are not contiguous in the replica: broadcast one region at
+      // a time through a region-sized staging buffer on every GPU.  The staging
+      // is the node's arena (idle after the join) when it is large enough, else
+      // a buffer counted in the node's `used` (capacity checked) and freed on
+      // every path.
+      int64_t maxe = 0;
+      for (int w = 0; w < G; ++w) maxe = std::max(maxe, (r1[w] - r0[w]) * (c1[w] - c0[w]));
+      const uint64_t need = static_cast<uint64_t>(maxe) * 4;
+      struct Staging {
+        northup_tree_s* t;
+        std::vector<void*> own;     // buffers we allocated (not arenas)
+        std::vector<int> node;
+        ~Staging() {
+          for (size_t w = 0; w < own.size(); ++w)
+            if (own[w]) {
+              cudaSetDevice(t->nodes[node[w]].phys);
+              cudaFree(own[w]);
+            }
+        }
+      } stage{t, std::vector<void*>(G, nullptr), std::vector<int>(P.worker_node.begin(), P.worker_node.end())};
+      std::vector<char*> sbuf(G, nullptr);
+      std::vector<uint64_t> counted(G, 0);
+      struct UsedGuard {
+        northup_tree_s* t;
+        const std::vector<int>& node;
+        std::vector<uint64_t>& counted;
+        ~UsedGuard() {
+          for (size_t w = 0; w < counted.size(); ++w) t->nodes[node[w]].used -= counted[w];
+        }
+      } used_guard{t, stage.node, counted};
       for (int w = 0; w < G; ++w) {
+        Node& hn = t->nodes[P.worker_node[w]];
+        if (hn.arena && hn.arena_bytes >= need) {
+          sbuf[w] = static_cast<char*>(hn.arena);
+          continue;
+        }
+        if (hn.capacity && hn.used + need > hn.capacity)
+          return fail(NU_ENOMEM, "replicate_result: node %d needs %llu B of staging beyond its capacity", hn.id,
+                      (unsigned long long)need);
         cudaSetDevice(dev[w]);
-        cudaError_t e = cudaMalloc(&packed[w], static_cast<size_t>(M) * N * 4);
-        if (e != cudaSuccess) return cuda_fail(e, "replica: packed buffer");
+        cudaError_t e = cudaMalloc(&stage.own[w], need);
+        if (e != cudaSuccess) return cuda_fail(e, "replica: staging buffer");
+        sbuf[w] = static_cast<char*>(stage.own[w]);
+        hn.used += need;
+        counted[w] = need;
       }
-      // pack own region contiguously at the region's packed offset
-      int64_t off = 0;
-      std::vector<int64_t> poff(G);
-      for (int w = 0; w < G; ++w) {
-        poff[w] = off;
-        off += (r1[w] - r0[w]) * (c1[w] - c0[w]);
-      }
-      for (int w = 0; w < G; ++w) {
-        cudaSetDevice(dev[w]);
-        const int64_t m = r1[w] - r0[w], n = c1[w] - c0[w];
-        cudaMemcpy2D(static_cast<char*>(packed[w]) + poff[w] * 4, n * 4,
-                     static_cast<char*>(rep[w]) + (r0[w] * N + c0[w]) * 4, N * 4, n * 4, m,
-                     cudaMemcpyDeviceToDevice);
-      }
-      nccl().GroupStart();
-      for (int root = 0; root < G; ++root)
+      for (int root = 0; root < G; ++root) {
+        const int64_t m = r1[root] - r0[root], n = c1[root] - c0[root];
+        if (m <= 0 || n <= 0) continue;
+        cudaSetDevice(dev[root]);
+        cudaError_t e = cudaMemcpy2D(sbuf[root], n * 4, static_cast<char*>(rep[root]) + (r0[root] * N + c0[root]) * 4,
+                                     N * 4, n * 4, m, cudaMemcpyDeviceToDevice);
+        if (e != cudaSuccess) return cuda_fail(e, "replica: pack region");
+        ncclResult_t r = nccl().GroupStart();
+        if (r != ncclSuccess) return nccl_fail(r, "ncclGroupStart");
+        for (int w = 0; w < G && r == ncclSuccess; ++w)
+          r = nccl().Broadcast(sbuf[w], sbuf[w], static_cast<size_t>(m * n), ncclFloat32, root,
+                               static_cast<ncclComm_t>(t->nccl_comms[w]), 0);
+        ncclResult_t r2 = nccl().GroupEnd();
+        if (r != ncclSuccess) return nccl_fail(r, "ncclBroadcast");
+        if (r2 != ncclSuccess) return nccl_fail(r2, "ncclGroupEnd");
         for (int w = 0; w < G; ++w) {
-          const size_t cnt = static_cast<size_t>((r1[root] - r0[root]) * (c1[root] - c0[root]));
-          char* buf = static_cast<char*>(packed[w]) + poff[root] * 4;
-          ncclResult_t r = nccl().Broadcast(buf, buf, cnt, ncclFloat32, root,
-                                            static_cast<ncclComm_t>(t->nccl_comms[w]), 0);
-          if (r != ncclSuccess) {
-            nccl().GroupEnd();
-            return nccl_fail(r, "ncclBroadcast");
-          }
+          if (w == root) continue;
+          cudaSetDevice(dev[w]);
+          e = cudaMemcpy2DAsync(static_cast<char*>(rep[w]) + (r0[root] * N + c0[root]) * 4, N * 4, sbuf[w], n * 4,
+                                n * 4, m, cudaMemcpyDeviceToDevice, 0);
+          if (e != cudaSuccess) return cuda_fail(e, "replica: unpack region");
         }
-      ncclResult_t r = nccl().GroupEnd();
-      if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd");
-      for (int w = 0; w < G; ++w) {
-        cudaSetDevice(dev[w]);
-        for (int root = 0; root < G; ++root) {
-          if (root == w) continue;
-          const int64_t m = r1[root] - r0[root], n = c1[root] - c0[root];
-          cudaMemcpy2DAsync(static_cast<char*>(rep[w]) + (r0[root] * N + c0[root]) * 4, N * 4,
-                            static_cast<char*>(packed[w]) + poff[root] * 4, n * 4, n * 4, m,
-                            cudaMemcpyDeviceToDevice, 0);
+        for (int w = 0; w < G; ++w) {   // the staging is reused by the next region
+          cudaSetDevice(dev[w]);
+          e = cudaDeviceSynchronize();
+          if (e != cudaSuccess) return cuda_fail(e, "replica: region sync");
         }
-        cudaError_t e = cudaDeviceSynchronize();
-        cudaFree(packed[w]);
-        if (e != cudaSuccess) return cuda_fail(e, "replica: unpack");
       }
     } else {
       nccl().GroupStart();

@@ -3,6 +3,7 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <sys/types.h>
 
 #include <array>
 #include <string>
@@ -24,6 +25,13 @@ constexpr int kHotspotMaxIters = 8;        // HotSpot-2D iterations per leaf lau
 // Kernel launches issued by the library (all devices, all threads): the
 // bench's `gpu_launches` claim (northup_debug_kernel_launches).
 void count_launches(int n);
+
+// Positional file I/O for every FILE path (tree.cpp): pread / pwrite, unless a
+// test armed a fault with NORTHUP_IO_FAULT="<read|write>:<eio|enospc|short|eof>:<n>"
+// (the n-th call of that kind fails with EIO / ENOSPC, moves half the bytes, or
+// returns 0).  The errno of the last failed I/O is kept (northup_last_io_errno).
+ssize_t pio(int fd, void* p, size_t n, uint64_t off, bool write);
+void note_io_errno(int e);
 
 // Thread-local error message (northup_last_error).  Returns its argument so
 // call sites can write `return fail(NU_EINVAL, "...")`.
@@ -97,6 +105,13 @@ struct northup_tree_s {
   std::vector<void*> flag_graveyard;   // outgrown flag buffers (peers may still map them)
   uint32_t gen = 0;                    // generation of the current call (monotonic)
   std::vector<int64_t> peer_key;       // the GEMM the peers were exported/imported for
+  // Set at finalize (exec.cpp): every pair of distinct HBM devices has NVLink/P2P
+  // access (else shared staging is not planned), the per-GPU PCIe bandwidth
+  // measured with every local link busy in both directions (0 = not measured:
+  // the planner's nominal constant), and the CPUs of each worker's NUMA node.
+  bool p2p_ok = true;
+  double pcie_gbs = 0.0;
+  std::vector<std::vector<int>> worker_cpus;   // per HBM node id (empty: no binding)
 };
 
 namespace nu {
@@ -236,6 +251,9 @@ inline long long debug_slow_ns(int pct, int64_t m, int64_t n, int64_t k) {
 int execute_plan(northup_tree_s* t, const Plan& plan, northup_buf_s* a, northup_buf_s* b,
                  northup_buf_s* c, const northup_gemm_opts* o, northup_stats* st);
 int finalize_workers(northup_tree_s* t);
+void numa_bind_plan(northup_tree_s* t);
+void bind_worker_thread(const northup_tree_s* t, int node);
+int calibrate_pcie(northup_tree_s* t);
 int ensure_arena(northup_tree_s* t, int node, uint64_t bytes);
 // Multi-process siblings (peer.cpp)
 std::vector<int64_t> peer_key_of(int64_t M, int64_t N, int64_t K, const northup_gemm_opts* o);

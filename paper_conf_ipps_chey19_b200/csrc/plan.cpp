@@ -155,6 +155,7 @@ struct EdgeCtx {
   // A panel and 1/b_share of each B panel over PCIe, its row / column peers
   // the rest, and pulls the other pieces from them over NVLink.
   int a_share = 1, b_share = 1;
+  double pcie = 0.0;       // B/s per GPU measured at finalize (0: kPlanPcie)
   // Origin of the region in the root buffers' addressing: (r0, c0) for a
   // whole-problem root; (0, 0) with ldb = ldc = region width when the root
   // buffers hold only this sibling's strips (multi-process siblings).
@@ -186,8 +187,9 @@ uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, i
 // their A strips arrive (H2D) and finished C strips leave (D2H).
 // With shared staging only this worker's pieces (1/a_share of A, 1/b_share of
 // B) cross its PCIe link; NVLink pulls are ~20x faster and not modelled.
-static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail, int a_share = 1,
-                      int b_share = 1) {
+static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail, int a_share, int b_share,
+                      double pcie) {
+  const double kPlanPcie = pcie > 0 ? pcie : nu::kPlanPcie;   // measured at finalize when available
   const double fl = 2.0 * bm * bn / kPlanFlops;               // s per unit of K
   const double ea = static_cast<double>(bm) / a_share, eb = static_cast<double>(bn) / b_share;
   const double main_c = fl * (K - tail);
@@ -253,7 +255,7 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
           bytes = s2_bytes(bm, bn, use_bk, K, 0, 0, x.kc);
         }
         if (bytes > cap) continue;
-        const double t = s2_time(bm, bn, K, tail, x.a_share, x.b_share);
+        const double t = s2_time(bm, bn, K, tail, x.a_share, x.b_share, x.pcie);
         if (!have || t <= cand_t * (1.0 + 1e-9)) {
           cand = S2Shape{bm, bn, use_bk, tail, tail > 0 ? sr : 0, bytes};
           cand_t = t;
@@ -332,8 +334,11 @@ void emit_tail_split(Builder& B, int w, const S2Layout& L, const S2Shape& s, int
   for (int64_t k = kt0; k < kt0 + kk; k += kc) {   // a piece is a whole number of panels
     const int64_t rows = std::min(kc, kt0 + kk - k), pp = k / kc;
     (void)p;
+    // the split form of an n-column row occupies hi at elements [0, n/2) and lo
+    // at [ld/2, ld/2 + n/2) of the row: declare the whole row (n < ld for a
+    // ragged last block)
     B.emit(make_split_b(w, L.arena, L.offBT + k * L.ldBs, L.ldBs, rows, bn, L.arena, L.offEB + pp * L.ldBs),
-           {{L.arena, L.offBT + k * L.ldBs, L.ldBs, rup(rows, 32), bn, true},
+           {{L.arena, L.offBT + k * L.ldBs, L.ldBs, rup(rows, 32), L.ldBs, true},
             {L.arena, L.offEB + pp * L.ldBs, L.ldBs, 1, bn, true}});
   }
 }
@@ -344,7 +349,7 @@ void emit_tail_leaf(Builder& B, int w, const S2Layout& L, const S2Shape& s, int 
   if (L.offEB >= 0) {
     o = with_presplit_b(o, L.arena, L.offEB, L.ldBs);
     B.emit(o, {{ar, ao, lda, rr, s.tail, false},
-               {L.arena, L.offBT, L.ldBs, s.tail, bn, false},
+               {L.arena, L.offBT, L.ldBs, s.tail, L.ldBs, false},     // the split rows' full span
                {L.arena, L.offEB, L.ldBs, cdiv(s.tail, B.P->kc), bn, false},
                {ar, co, ldc, rr, bn, true}});
   } else {
@@ -1254,6 +1259,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     x.K = K;
     x.cap = t->nodes[hbm[w]].capacity;
     x.kc = P.kc;
+    x.pcie = t->pcie_gbs * 1e9;
     x.obm = root.bm;
     x.obn = root.bn;
     x.obk = root.bk;
@@ -1273,7 +1279,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   // has a region of the same shape under S2 (opts->shared_staging < 0 disables).
   int Pr = 1, Pc = 1;
   partition_grid(G, M, N, &Pr, &Pc);
-  bool share = G > 1 && !(o && o->shared_staging < 0);
+  bool share = G > 1 && !(o && o->shared_staging < 0) && t->p2p_ok;
   for (int w = 0; w < G && share; ++w)
     share = uses[w] == NU_SCHED_S2 && xs[w].r1 - xs[w].r0 == xs[0].r1 - xs[0].r0 &&
             xs[w].c1 - xs[w].c0 == xs[0].c1 - xs[0].c0 && xs[w].r1 > xs[w].r0 && xs[w].c1 > xs[w].c0;

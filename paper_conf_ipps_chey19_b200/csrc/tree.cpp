@@ -2,6 +2,11 @@
 // printout and the unified data-management API (Table I, P:264-272;
 // Listing 4).
 #include <errno.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <atomic>
 #include <fcntl.h>
 #include <stdarg.h>
 #include <stdio.h>
@@ -13,6 +18,40 @@
 #include <string>
 
 #include "northup_internal.h"
+
+namespace nu {
+static std::atomic<int> g_io_errno{0};
+static std::atomic<long long> g_io_calls[2];
+
+void note_io_errno(int e) { g_io_errno.store(e); }
+
+ssize_t pio(int fd, void* p, size_t n, uint64_t off, bool write) {
+  static const char* spec = getenv("NORTHUP_IO_FAULT");
+  if (spec && *spec) {
+    char op[16] = {}, kind[16] = {};
+    long long nth = 0;
+    if (sscanf(spec, "%15[^:]:%15[^:]:%lld", op, kind, &nth) == 3 && (strcmp(op, "write") == 0) == write) {
+      const long long k = g_io_calls[write ? 1 : 0].fetch_add(1) + 1;
+      if (k == nth) {
+        if (strcmp(kind, "eio") == 0) {
+          errno = EIO;
+          return -1;
+        }
+        if (strcmp(kind, "enospc") == 0) {
+          errno = ENOSPC;
+          return -1;
+        }
+        if (strcmp(kind, "eof") == 0) return 0;
+        if (strcmp(kind, "short") == 0 && n > 1) n /= 2;
+      }
+    }
+  }
+  return write ? pwrite(fd, p, n, static_cast<off_t>(off)) : pread(fd, p, n, static_cast<off_t>(off));
+}
+}  // namespace nu
+
+
+extern "C" int northup_last_io_errno(void);
 
 namespace nu {
 
@@ -299,6 +338,20 @@ static void print_node(const northup_tree_s* t, int id, int depth, std::string& 
   for (int c : n.children) print_node(t, c, depth + 1, out);
 }
 
+int northup_tree_link_info(northup_tree_t t, double* pcie_gbs, int* p2p_ok, int* numa_bound) {
+  using namespace nu;
+  if (!t) return fail(NU_EINVAL, "null tree");
+  if (!t->finalized) return fail(NU_ESTATE, "tree not finalized");
+  if (pcie_gbs) *pcie_gbs = t->pcie_gbs;
+  if (p2p_ok) *p2p_ok = t->p2p_ok ? 1 : 0;
+  if (numa_bound) {
+    int n = 0;
+    for (const auto& c : t->worker_cpus) n += c.empty() ? 0 : 1;
+    *numa_bound = n;
+  }
+  return 0;
+}
+
 int northup_tree_print(northup_tree_t t, char* buf, size_t n, size_t* n_needed) {
   if (!t) return fail(NU_EINVAL, "tree is NULL");
   std::string s;
@@ -495,18 +548,23 @@ int northup_buf_info(northup_buf_t b, int* node, void** ptr, uint64_t* bytes) {
   return 0;
 }
 
+
 // Listing 4: file_write = lseek + write; we use pread/pwrite
 // loops (positional, restartable on short transfers).
 static int file_rw(int fd, void* buf, uint64_t count, uint64_t offset, bool write) {
   uint8_t* p = static_cast<uint8_t*>(buf);
   while (count) {
-    ssize_t r = write ? pwrite(fd, p, count, static_cast<off_t>(offset))
-                      : pread(fd, p, count, static_cast<off_t>(offset));
+    ssize_t r = nu::pio(fd, p, count, offset, write);
     if (r < 0) {
       if (errno == EINTR) continue;
-      return fail(NU_EIO, "%s: %s", write ? "pwrite" : "pread", strerror(errno));
+      const int err = errno;
+      nu::note_io_errno(err);
+      return fail(NU_EIO, "%s: %s", write ? "pwrite" : "pread", strerror(err));
     }
-    if (r == 0) return fail(NU_EIO, "%s: unexpected end of file", write ? "pwrite" : "pread");
+    if (r == 0) {
+      nu::note_io_errno(0);
+      return fail(NU_EIO, "%s: unexpected end of file", write ? "pwrite" : "pread");
+    }
     p += r;
     count -= static_cast<uint64_t>(r);
     offset += static_cast<uint64_t>(r);
@@ -614,3 +672,5 @@ int northup_release(northup_tree_t t, northup_buf_t b) {
 }
 
 }  // extern "C"
+
+extern "C" int northup_last_io_errno(void) { return nu::g_io_errno.load(); }

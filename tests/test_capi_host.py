@@ -86,6 +86,25 @@ def test_partition_grid(G, M, N, grid):
 
 
 # ------------------------------------------------------------ plan simulator
+def split_dead_mask(w_off, w_ld, w_rows, w_cols, so, sld, srows, sn):
+    """Which values of a split region (off so, ld sld, srows x sn columns, split
+    form: hi of column n at row element n/2, lo at sld/2 + n/2) a write of
+    w_rows x w_cols at (w_off, w_ld) destroys."""
+    dead = np.zeros((srows, sn), dtype=bool)
+    if w_off + (w_rows - 1) * w_ld + w_cols <= so or so + srows * sld <= w_off:
+        return dead
+    n = np.arange(sn)
+    for r in range(w_rows):
+        a0, a1 = w_off + r * w_ld, w_off + r * w_ld + w_cols
+        for sr in range(max(0, (a0 - so) // sld), min(srows, (a1 - 1 - so) // sld + 1)):
+            base = so + sr * sld
+            lo_e, hi_e = max(a0, base) - base, min(a1, base + sld) - base
+            if hi_e > lo_e:
+                dead[sr] |= ((n // 2 >= lo_e) & (n // 2 < hi_e)) | \
+                            ((sld // 2 + n // 2 >= lo_e) & (sld // 2 + n // 2 < hi_e))
+    return dead
+
+
 def kpanels(A, P):
     """A (M x K) in the K-panel-major file layout of northup_file_tile_kpanels."""
     M, K = A.shape
@@ -110,25 +129,36 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
             mem.append(np.full(b["bytes"] // 4, np.nan))
 
     # NU_OP_SPLIT_B rewrites a resident B region in place into the leaf's split
-    # form: model that as moving the values to a shadow copy (the raw region
-    # becomes NaN) which only pre-split leaf ops read; a later copy into the
-    # region destroys the split form (NaN in the shadow), as on the GPU.
+    # form: model that as moving the values to a shadow copy (the raw rows
+    # become NaN over their whole leading dimension, as the hi / lo halves
+    # do on the GPU) which only pre-split leaf ops read; a later copy into a
+    # row destroys the split values whose hi (element n/2) or lo (ld/2 + n/2)
+    # bytes it overwrites.
     shadow = [np.full(len(x), np.nan) for x in mem]
+    splits = [[] for _ in mem]            # per buffer: split regions (off, ld, rows, n)
 
     def view(buf, off, ld, rows, cols, m=None):
         m = mem if m is None else m
         return np.lib.stride_tricks.as_strided(m[buf][off:], shape=(rows, cols),
                                                strides=(ld * 8, 8), writeable=True)
 
+    def clobber_split(buf, off, ld, rows, cols):
+        """A write destroys the split values whose hi / lo bytes it covers."""
+        for (so, sld, srows, sn) in splits[buf]:
+            dead = split_dead_mask(off, ld, rows, cols, so, sld, srows, sn)
+            if dead.any():
+                view(buf, so, sld, srows, sn, shadow)[dead] = np.nan
+
     def run(op):
         if op["op"] in (nu.NU_OP_COPY, nu.NU_OP_IO_READ, nu.NU_OP_IO_WRITE):
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
                 view(op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
-            view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], shadow)[...] = np.nan
+            clobber_split(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])
         elif op["op"] == nu.NU_OP_SPLIT_B:
             src = view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], shadow)[...] = src
-            src[...] = np.nan
+            view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["dst_ld"])[...] = np.nan
+            splits[op["dst_buf"]].append((op["dst_off"], op["dst_ld"], op["rows"], op["cols"]))
         elif op["op"] == nu.NU_OP_LEAF:
             a = view(op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
             b = view(op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"],
@@ -333,6 +363,7 @@ def test_random_plans_replay_exactly(M, N, K, G, cap_kib, kc, sched, file_root, 
     (1024, 512, 1000, 8, 0, 128),       # 4 x 2, ragged last K panel
     (600, 600, 700, 4, 1_200_000, 64),  # capacity forces several C blocks per region
     (4096, 8192, 512, 8, 0, 128),       # first-panel sub-block grid (bm, bn >= 4096)
+    (900, 900, 1024, 3, 4 << 20, 512),  # ragged last column block with an in-place split B tail
 ])
 def test_shared_staging_plan_replays_exactly(M, N, K, G, cap, kc):
     """Shared staging: every A/B byte crosses PCIe once per grid row / column
@@ -420,6 +451,7 @@ def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
         return strips[w][bufs[i]["kind"]] if bufs[i]["kind"] < 3 else arenas[i]
 
     shadows = {}
+    splits = {}
 
     def view(w, buf, off, ld, rows, cols, shadow=False):
         base = mem(w, buf)
@@ -440,11 +472,16 @@ def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
         if op["op"] == nu.NU_OP_COPY:
             view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])[...] = \
                 view(w, op["src_buf"], op["src_off"], op["src_ld"], op["rows"], op["cols"]).copy()
-            view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], True)[...] = np.nan
+            for (so, sld, srows, sn) in splits.get(id(mem(w, op["dst_buf"])), []):
+                dead = split_dead_mask(op["dst_off"], op["dst_ld"], op["rows"], op["cols"], so, sld, srows, sn)
+                if dead.any():
+                    view(w, op["dst_buf"], so, sld, srows, sn, True)[dead] = np.nan
         elif op["op"] == nu.NU_OP_SPLIT_B:
             src = view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"])
             view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], True)[...] = src
-            src[...] = np.nan
+            view(w, op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["dst_ld"])[...] = np.nan
+            splits.setdefault(id(mem(w, op["dst_buf"])), []).append(
+                (op["dst_off"], op["dst_ld"], op["rows"], op["cols"]))
         elif op["op"] == nu.NU_OP_LEAF:
             a = view(w, op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
             b = view(w, op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"], op["src_buf"] >= 0)

@@ -118,3 +118,68 @@ def test_file_direct_to_hbm(tmp_path, monkeypatch, M, N, K, G, cap, panel, kind)
         e, _ = oracle.normwise_err(C, ref, oracle.row_norms(A), oracle.col_norms(B))
         assert e <= 1e-5, e
     assert st["bytes_file_write"] == 4 * M * N
+
+
+# ------------------------------------------------------------ I/O fault injection
+# NORTHUP_IO_FAULT="<read|write>:<eio|enospc|short|eof>:<n>" (northup.h) makes the
+# n-th pread / pwrite of the process fail; each case runs in its own process.
+_FAULT_SCRIPT = r'''
+import ctypes, json, sys
+import numpy as np
+sys.path.insert(0, {root!r})
+import nugen, oracle
+import paper_conf_ipps_chey19_b200 as nu
+d = {d!r}
+out = {{}}
+M, N, K = 256, 192, 320
+A = nugen.fill(M, K, 9, 1, "int"); B = nugen.fill(K, N, 9, 2, "int")
+A.tofile(d + "/A.bin"); B.tofile(d + "/B.bin")
+t = nu.Tree(); root = t.add_node(-1, nu.NU_FILE); st = t.add_node(root, nu.NU_HOST)
+h = t.add_node(st, nu.NU_HBM, 0); t.add_node(h, nu.NU_SMEM, 0, 227 * 1024, nu.NU_PROC_SM100)
+t.finalize()
+fa = t.open_file(0, d + "/A.bin", 4 * M * K); fb = t.open_file(0, d + "/B.bin", 4 * K * N)
+fc = t.open_file(0, d + "/C.bin", 4 * M * N)
+try:
+    t.gemm(fa, fb, fc, M, N, K, nu.make_opts(k_chunk=64))
+    C = np.fromfile(d + "/C.bin", dtype=np.float32).reshape(M, N)
+    out["rc"] = 0
+    out["exact"] = bool(np.array_equal(C.astype(np.float64), oracle.gemm(A, B)))
+except nu.NorthupError as e:
+    out["rc"] = e.code
+    out["msg"] = str(e)
+out["errno"] = nu.last_io_errno()
+t.destroy()
+print(json.dumps(out))
+'''
+
+
+def _run_fault(tmp_path, spec):
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ)
+    if spec:
+        env["NORTHUP_IO_FAULT"] = spec
+    r = subprocess.run([sys.executable, "-c", _FAULT_SCRIPT.format(root=root, d=str(tmp_path))],
+                       capture_output=True, text=True, timeout=300, env=env)
+    assert r.returncode == 0, r.stderr[-2000:]
+    return json.loads(r.stdout.strip().splitlines()[-1])
+
+
+@pytest.mark.parametrize("spec,err", [("read:eio:3", 5), ("write:enospc:1", 28), ("read:eof:2", 0)])
+def test_file_io_faults_fail_loudly(tmp_path, spec, err):
+    """An I/O error on the FILE path ends northup_gemm with NU_EIO (no hang,
+    Listing 4's file_read / file_write, P:276-289) and keeps the errno."""
+    out = _run_fault(tmp_path, spec)
+    assert out["rc"] == nu.NU_EIO and out["errno"] == err, out
+    assert ("pread" in out["msg"]) == spec.startswith("read") and ("pwrite" in out["msg"]) == spec.startswith("write")
+
+
+@pytest.mark.parametrize("spec", ["read:short:2", "write:short:1", ""])
+def test_file_short_transfers_are_completed(tmp_path, spec):
+    """pread / pwrite may move fewer bytes than asked: the library loops, so
+    the result is still exact."""
+    out = _run_fault(tmp_path, spec)
+    assert out["rc"] == 0 and out["exact"], out

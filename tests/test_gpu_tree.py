@@ -254,11 +254,27 @@ def test_queue_schedule_matches_static_and_oracle(G, M, N, K, cap, kind):
 def test_queue_schedule_steals_from_a_slow_sibling(monkeypatch):
     """A sibling that is slow to pop (test hook emulating an asymmetric tree,
     Fig. 2) loses tiles to the fast one: steals happen and C is still exact."""
-    # sibling 1 holds its compute stream 30x the nominal leaf time before each
-    # leaf (the hook's nominal rate is 300 TF/s; host issue dominates small tiles)
-    monkeypatch.setenv("NORTHUP_DEBUG_SLOW_SIBLING", "1,3000")
+    # sibling 1 holds its compute stream 500x the nominal leaf time (2mnk at
+    # 300 TF/s, ~1 ms here) before each leaf: the two virtual siblings share one
+    # GPU and one PCIe link, so the delay must exceed a tile's copies to show
+    monkeypatch.setenv("NORTHUP_DEBUG_SLOW_SIBLING", "1,50000")
     M, N, K = 2048, 2048, 1024
     C, a, b, st = run_host(M, N, K, G=2, kind="int", seed=2, k_chunk=512, schedule=nu.NU_SCHED_QUEUE,
                            queue_tiles=8)
     assert st["tasks_stolen"] > 0
     check(C, a, b, "int")
+
+
+def test_finalize_measures_links():
+    """finalize calibrates the planner's PCIe term with every local link busy
+    (S§8(d)), records P2P reachability (shared staging needs it) and binds
+    workers to their GPU's NUMA node when the host reports one."""
+    t, _ = nu.host_tree(2, 1 << 30, devices=[0, 0])     # two virtual siblings on one GPU
+    t.finalize()
+    li = t.link_info()
+    assert 10 < li["pcie_gbs"] < 80 and li["p2p_ok"]
+    t.destroy()
+    th = nu.hbm_tree(0)
+    th.finalize()
+    assert th.link_info()["pcie_gbs"] == 0.0            # no host edge, nothing measured
+    th.destroy()
