@@ -54,23 +54,60 @@ __device__ __forceinline__ void split1(float x, float s, __half& hi, __half& lo)
   lo = __float2half_rn(y - __half2float(hi));   // y - hi is exact in fp32
 }
 
+// hi / lo of four consecutive k (or n) as two 8-byte stores' worth of fp16
+__device__ __forceinline__ void split4(float4 x, float s, uint2& hi, uint2& lo) {
+  __half h[4], l[4];
+  split1(x.x, s, h[0], l[0]);
+  split1(x.y, s, h[1], l[1]);
+  split1(x.z, s, h[2], l[2]);
+  split1(x.w, s, h[3], l[3]);
+  hi = make_uint2(__half_as_ushort(h[0]) | (static_cast<uint32_t>(__half_as_ushort(h[1])) << 16),
+                  __half_as_ushort(h[2]) | (static_cast<uint32_t>(__half_as_ushort(h[3])) << 16));
+  lo = make_uint2(__half_as_ushort(l[0]) | (static_cast<uint32_t>(__half_as_ushort(l[1])) << 16),
+                  __half_as_ushort(l[2]) | (static_cast<uint32_t>(__half_as_ushort(l[3])) << 16));
+}
+
 // One warp per row of A (grid-stride).  Pass 1: row max; pass 2: each 32-k
 // group is read by the warp, then written (the same 128 bytes when in place).
+// vec: A and dst rows 16-B aligned (float4 loads, 128 k per warp step).
 __global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
-                                                      float* dst, int64_t ldd, int* ea) {
+                                                      float* dst, int64_t ldd, int* ea, int vec) {
   const int lane = threadIdx.x & 31;
   const int warps = (gridDim.x * blockDim.x) >> 5;
   for (int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M; r += warps) {
     const float* a = A + static_cast<int64_t>(r) * lda;
     float m = 0.f;
-    for (int k = lane; k < Kl; k += 32) m = fmaxf(m, fabsf(a[k]));
+    if (vec) {
+      const int K4 = Kl & ~3;
+      for (int k = 4 * lane; k < K4; k += 128) {
+        const float4 x = *reinterpret_cast<const float4*>(a + k);
+        m = fmaxf(fmaxf(m, fmaxf(fabsf(x.x), fabsf(x.y))), fmaxf(fabsf(x.z), fabsf(x.w)));
+      }
+      for (int k = K4 + lane; k < Kl; k += 32) m = fmaxf(m, fabsf(a[k]));
+    } else {
+      for (int k = lane; k < Kl; k += 32) m = fmaxf(m, fabsf(a[k]));
+    }
 #pragma unroll
     for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
     const int e = split_exponent(m);
     if (lane == 0) ea[r] = e;
     const float s = pow2(-e);
     __half* out = reinterpret_cast<__half*>(dst + static_cast<int64_t>(r) * ldd);
-    for (int k0 = 0; k0 < Kp; k0 += 32) {
+    int kv = 0;
+    if (vec) {
+      // lane l: k = k0 + 4 l .. +3, i.e. group g = l / 8, positions 4 (l % 8) .. +3
+      for (; kv + 128 <= Kl; kv += 128) {
+        const float4 x = *reinterpret_cast<const float4*>(a + kv + 4 * lane);
+        __syncwarp();                            // the 512 bytes are read before they are overwritten
+        uint2 hi, lo;
+        split4(x, s, hi, lo);
+        const int g = lane >> 3, c = 4 * (lane & 7);
+        *reinterpret_cast<uint2*>(out + 2 * (kv + 32 * g) + c) = hi;
+        *reinterpret_cast<uint2*>(out + 2 * (kv + 32 * g) + 32 + c) = lo;
+        __syncwarp();
+      }
+    }
+    for (int k0 = kv; k0 < Kp; k0 += 32) {
       const int k = k0 + lane;
       const float x = k < Kl ? a[k] : 0.f;
       __syncwarp();                              // the group is read before it is overwritten
@@ -94,13 +131,45 @@ __global__ void __launch_bounds__(256) colmax_kernel(const float* B, int64_t ldb
   atomicMax(bmax + n, __float_as_uint(m));
 }
 
+// Column exponents from the column maxima (once per column, not per element).
+__global__ void __launch_bounds__(256) col_exps_kernel(const unsigned* bmax, int N, int* eb) {
+  const int n = blockIdx.x * 256 + threadIdx.x;
+  if (n < N) eb[n] = split_exponent(__uint_as_float(bmax[n]));
+}
+
+// Out of place: rows [k0, k0 + 8) x 4 columns per thread, float4 loads and
+// 8-byte hi / lo stores (B and dst rows 16-B aligned, N % 4 == 0).
+__global__ void __launch_bounds__(256) split_b_oop_kernel(const float* __restrict__ B, int64_t ldb, int Kl, int Kp,
+                                                          int N, const int* __restrict__ eb,
+                                                          float* __restrict__ dst, int64_t ldd) {
+  const int n = 4 * (blockIdx.x * 256 + threadIdx.x);
+  if (n >= N) return;
+  const float s0 = pow2(-eb[n]), s1 = pow2(-eb[n + 1]), s2 = pow2(-eb[n + 2]), s3 = pow2(-eb[n + 3]);
+  const int k1 = min(Kp, 8 * (blockIdx.y + 1));
+  for (int k = 8 * blockIdx.y; k < k1; ++k) {
+    float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (k < Kl) x = *reinterpret_cast<const float4*>(B + static_cast<int64_t>(k) * ldb + n);
+    __half h[4], l[4];
+    split1(x.x, s0, h[0], l[0]);
+    split1(x.y, s1, h[1], l[1]);
+    split1(x.z, s2, h[2], l[2]);
+    split1(x.w, s3, h[3], l[3]);
+    __half* hi_row = reinterpret_cast<__half*>(dst + static_cast<int64_t>(k) * ldd);
+    *reinterpret_cast<uint2*>(hi_row + n) =
+        make_uint2(__half_as_ushort(h[0]) | (static_cast<uint32_t>(__half_as_ushort(h[1])) << 16),
+                   __half_as_ushort(h[2]) | (static_cast<uint32_t>(__half_as_ushort(h[3])) << 16));
+    *reinterpret_cast<uint2*>(hi_row + ldd + n) =
+        make_uint2(__half_as_ushort(l[0]) | (static_cast<uint32_t>(__half_as_ushort(l[1])) << 16),
+                   __half_as_ushort(l[2]) | (static_cast<uint32_t>(__half_as_ushort(l[3])) << 16));
+  }
+}
+
 // One CTA per row of B: the row is staged in shared memory before any of it
 // is overwritten (in place, hi lands on the row's first half and lo on its
 // second).  Rows [Kl, Kp) are written as zeros.
 constexpr int kSplitRowMaxN = 49152;   // 192 KiB of fp32 staging
 __global__ void __launch_bounds__(1024) split_b_kernel(const float* B, int64_t ldb, int Kl, int N,
-                                                       const unsigned* bmax, float* dst, int64_t ldd,
-                                                       int* eb) {
+                                                       const int* eb, float* dst, int64_t ldd) {
   extern __shared__ float row[];
   const int k = blockIdx.x;
   const float* brow = B + static_cast<int64_t>(k) * ldb;
@@ -109,10 +178,8 @@ __global__ void __launch_bounds__(1024) split_b_kernel(const float* B, int64_t l
   __half* hi_row = reinterpret_cast<__half*>(dst + static_cast<int64_t>(k) * ldd);
   __half* lo_row = hi_row + ldd;
   for (int n = threadIdx.x; n < N; n += blockDim.x) {
-    const int e = split_exponent(__uint_as_float(bmax[n]));
-    if (k == 0) eb[n] = e;
     __half h, l;
-    split1(row[n], pow2(-e), h, l);
+    split1(row[n], pow2(-eb[n]), h, l);
     hi_row[n] = h;
     lo_row[n] = l;
   }
@@ -125,7 +192,9 @@ int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64
   if (M <= 0) return 0;
   const int Kp = (Kl + 31) / 32 * 32;
   const int grid = static_cast<int>(std::min<int64_t>((M + 7) / 8, 32LL * sms));
-  split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea);
+  const int vec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && lda % 4 == 0 &&
+                  (reinterpret_cast<uintptr_t>(dst) % 16 == 0) && ldd % 4 == 0;
+  split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea, vec);
   count_launches(1);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_a launch: %s", cudaGetErrorString(e));
@@ -142,16 +211,24 @@ int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64
     colmax_kernel<<<dim3((N + 255) / 256, (Kl + 255) / 256), 256, 0, s>>>(B, ldb, Kl, N, bmax);
     count_launches(1);
   }
-  static bool configured[kMaxDevices];
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (!configured[dev]) {
-    e = cudaFuncSetAttribute(split_b_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * kSplitRowMaxN);
-    if (e != cudaSuccess) return fail(NU_ECUDA, "split_b attribute: %s", cudaGetErrorString(e));
-    configured[dev] = true;
+  col_exps_kernel<<<(N + 255) / 256, 256, 0, s>>>(bmax, N, eb);
+  count_launches(1);
+  const bool vec = dst != B && N % 4 == 0 && ldb % 4 == 0 && ldd % 4 == 0 &&
+                   reinterpret_cast<uintptr_t>(B) % 16 == 0 && reinterpret_cast<uintptr_t>(dst) % 16 == 0;
+  if (vec) {
+    split_b_oop_kernel<<<dim3((N / 4 + 255) / 256, (Kp + 7) / 8), 256, 0, s>>>(B, ldb, Kl, Kp, N, eb, dst, ldd);
+  } else {
+    static bool configured[kMaxDevices];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!configured[dev]) {
+      e = cudaFuncSetAttribute(split_b_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * kSplitRowMaxN);
+      if (e != cudaSuccess) return fail(NU_ECUDA, "split_b attribute: %s", cudaGetErrorString(e));
+      configured[dev] = true;
+    }
+    const int threads = std::min(1024, std::max(64, (N / 8 + 31) / 32 * 32));
+    split_b_kernel<<<Kp, threads, 4 * static_cast<size_t>(N), s>>>(B, ldb, Kl, N, eb, dst, ldd);
   }
-  const int threads = std::min(1024, std::max(64, (N / 8 + 31) / 32 * 32));
-  split_b_kernel<<<Kp, threads, 4 * static_cast<size_t>(N), s>>>(B, ldb, Kl, N, bmax, dst, ldd, eb);
   count_launches(1);
   e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_b launch: %s", cudaGetErrorString(e));
@@ -162,6 +239,8 @@ void preload_split() {
   cudaFuncGetAttributes(&fa, split_a_kernel);
   cudaFuncGetAttributes(&fa, colmax_kernel);
   cudaFuncGetAttributes(&fa, split_b_kernel);
+  cudaFuncGetAttributes(&fa, split_b_oop_kernel);
+  cudaFuncGetAttributes(&fa, col_exps_kernel);
 }
 
 }  // namespace leaf
