@@ -35,7 +35,7 @@ namespace x3 {
 
 constexpr int BM = 256, BN = 256, BM_CTA = 128, BN_CTA = 128;
 constexpr int KS = 32;                               // real k per stage
-constexpr int STAGES = 5;
+constexpr int STAGES = 6;
 constexpr int A_BYTES = BM_CTA * 2 * KS * 2;         // 16 KiB
 constexpr int B_HALF_BYTES = 2 * KS * 64 * 2;        // 64 rows x 64 n fp16 = 8 KiB
 constexpr int B_BYTES = 2 * B_HALF_BYTES;            // 16 KiB
@@ -44,8 +44,9 @@ constexpr int EPI_WARP0 = 2;
 constexpr int EPI_WARPS = 16;                         // four per TMEM lane quarter, 64 columns each
 constexpr int EPI_THREADS = 32 * EPI_WARPS;
 constexpr int EPI_COLS = 64;                          // tile columns per epilogue thread (its running sum)
-constexpr int BOX_BYTES = 32 * 32 * 4;                // one staging box (32 rows x 32 fp32) per warp
-constexpr int EPI_BYTES = EPI_WARPS * BOX_BYTES;
+constexpr int BOX_BYTES = 32 * 32 * 4;                // one staging box: 32 rows x 32 fp32
+constexpr int EPI_BOXES = EPI_WARPS / 2;               // shared by warps ew and ew + 8, in turn
+constexpr int EPI_BYTES = EPI_BOXES * BOX_BYTES;
 constexpr int NUM_THREADS = 32 * (EPI_WARP0 + EPI_WARPS);
 constexpr int TMEM_COLS = 512;                       // two 256-column accumulators
 constexpr int BAR_BYTES = 256;
@@ -157,6 +158,9 @@ __device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* map, uint32
                    reinterpret_cast<uint64_t>(map)),
                "r"(src), "r"(c0), "r"(c1)
                : "memory");
+}
+__device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 template <int N>
@@ -319,7 +323,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const int q = warp & 3;                                   // TMEM lane quarter
     const int cg = ew >> 2;                                   // 64-column group
     const uint32_t tempty_leader = mapa(bar_tempty, 0);
-    const uint32_t box = smem_u32(epi_base + ew * BOX_BYTES);
+    const uint32_t box = smem_u32(epi_base + (ew % EPI_BOXES) * BOX_BYTES);
     const uint32_t t_row = tmem_base + (static_cast<uint32_t>(32 * q) << 16) + EPI_COLS * cg;
     uint32_t chunk_it = 0;
     for (int t = cid; t < num_tiles; t += nclusters) {
@@ -346,35 +350,48 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       }
       const int er = grow < p.M ? p.ea[grow] : 0;
 #pragma unroll
-      for (int h = 0; h < EPI_COLS / 32; ++h) {
+      for (int h = 0; h < EPI_COLS / 32; ++h) {      // scale by 2^(e_i + e_j), in place
         const int gcol0 = nb * BN + EPI_COLS * cg + 32 * h;
         const int ebl = (gcol0 + lane < p.N) ? p.eb[gcol0 + lane] : 0;
-        float* v = sum + 32 * h;   // scaled in place
 #pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = scale2(v[j], er + __shfl_sync(0xffffffffu, ebl, j));
-        if (p.vec_ok) {
-          if (lane == 0) bulk_wait_read<0>();                 // the box's previous store has read it
-          __syncwarp();
-          const uint32_t rowp = box + lane * 128;
+        for (int j = 0; j < 32; ++j) sum[32 * h + j] = scale2(sum[32 * h + j], er + __shfl_sync(0xffffffffu, ebl, j));
+      }
+      // write the tile: warps ew < 8 first, then warps ew >= 8 reuse their boxes
 #pragma unroll
-          for (int i = 0; i < 8; ++i)
-            sts128(rowp + ((i ^ (lane & 7)) << 4), __float_as_uint(v[4 * i]), __float_as_uint(v[4 * i + 1]),
-                   __float_as_uint(v[4 * i + 2]), __float_as_uint(v[4 * i + 3]));
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) {
-            if (p.accumulate) tma_reduce_add_2d(&tmC, box, gcol0, row0);
-            else tma_store_2d(&tmC, box, gcol0, row0);
-            bulk_commit();
+      for (int turn = 0; turn < 2; ++turn) {
+        if ((ew >> 3) == turn) {
+#pragma unroll
+          for (int h = 0; h < EPI_COLS / 32; ++h) {
+            const int gcol0 = nb * BN + EPI_COLS * cg + 32 * h;
+            const float* v = sum + 32 * h;
+            if (p.vec_ok) {
+              if (lane == 0) bulk_wait_read<0>();             // the box's previous store has read it
+              __syncwarp();
+              const uint32_t rowp = box + lane * 128;
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                sts128(rowp + ((i ^ (lane & 7)) << 4), __float_as_uint(v[4 * i]), __float_as_uint(v[4 * i + 1]),
+                       __float_as_uint(v[4 * i + 2]), __float_as_uint(v[4 * i + 3]));
+              fence_proxy_async_smem();
+              __syncwarp();
+              if (lane == 0) {
+                if (p.accumulate) tma_reduce_add_2d(&tmC, box, gcol0, row0);
+                else tma_store_2d(&tmC, box, gcol0, row0);
+                bulk_commit();
+              }
+            } else if (grow < p.M) {
+              float* dst = p.C + static_cast<int64_t>(grow) * p.ldc + gcol0;
+#pragma unroll
+              for (int j = 0; j < 32; ++j) {
+                if (gcol0 + j >= p.N) continue;
+                dst[j] = p.accumulate ? __fadd_rn(dst[j], v[j]) : v[j];
+              }
+            }
           }
-        } else if (grow < p.M) {
-          float* dst = p.C + static_cast<int64_t>(grow) * p.ldc + gcol0;
-#pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            if (gcol0 + j >= p.N) continue;
-            dst[j] = p.accumulate ? __fadd_rn(dst[j], v[j]) : v[j];
-          }
+          if (lane == 0) bulk_wait_read<0>();                 // boxes free for the other turn
+          __syncwarp();
         }
+        named_bar_sync(2, EPI_THREADS);
       }
     }
     if (lane == 0) bulk_wait_all();

@@ -155,10 +155,11 @@ __global__ void __launch_bounds__(256) split_b_oop_kernel(const float* __restric
     split1(x.z, s2, h[2], l[2]);
     split1(x.w, s3, h[3], l[3]);
     __half* hi_row = reinterpret_cast<__half*>(dst + static_cast<int64_t>(k) * ldd);
+    const int64_t lo_off = ldd;
     *reinterpret_cast<uint2*>(hi_row + n) =
         make_uint2(__half_as_ushort(h[0]) | (static_cast<uint32_t>(__half_as_ushort(h[1])) << 16),
                    __half_as_ushort(h[2]) | (static_cast<uint32_t>(__half_as_ushort(h[3])) << 16));
-    *reinterpret_cast<uint2*>(hi_row + ldd + n) =
+    *reinterpret_cast<uint2*>(hi_row + lo_off + n) =
         make_uint2(__half_as_ushort(l[0]) | (static_cast<uint32_t>(__half_as_ushort(l[1])) << 16),
                    __half_as_ushort(l[2]) | (static_cast<uint32_t>(__half_as_ushort(l[3])) << 16));
   }
