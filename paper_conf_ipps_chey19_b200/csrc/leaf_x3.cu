@@ -36,6 +36,7 @@ namespace x3 {
 constexpr int BM = 256, BN = 256, BM_CTA = 128, BN_CTA = 128;
 constexpr int KS = 32;                               // real k per stage
 constexpr int STAGES = 6;
+
 constexpr int A_BYTES = BM_CTA * 2 * KS * 2;         // 16 KiB
 constexpr int B_HALF_BYTES = 2 * KS * 64 * 2;        // 64 rows x 64 n fp16 = 8 KiB
 constexpr int B_BYTES = 2 * B_HALF_BYTES;            // 16 KiB
