@@ -795,6 +795,134 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     return result
 
 
+# --------------------------------------------------------------- FILE root
+def measure_disk(d: str, nbytes: int = 1 << 30) -> dict:
+    """Sequential O_DIRECT write then read of one file on the bench's file
+    system (GB/s): the disk term of the FILE-root roofline (S§8(d))."""
+    import mmap
+    path = os.path.join(d, "disk_probe.bin")
+    chunk = 64 << 20
+    buf = mmap.mmap(-1, chunk)                      # page-aligned (O_DIRECT)
+    buf.write(os.urandom(1 << 20) * (chunk >> 20))
+    flags = getattr(os, "O_DIRECT", 0)
+    out = {"how": f"O_DIRECT {nbytes >> 20} MiB sequential in {chunk >> 20} MiB requests, fsync before stopping the clock"}
+    fd = os.open(path, os.O_CREAT | os.O_WRONLY | os.O_TRUNC | flags, 0o644)
+    t0 = time.perf_counter()
+    for off in range(0, nbytes, chunk):
+        os.pwrite(fd, buf, off)
+    os.fsync(fd)
+    out["write_gbs"] = round(nbytes / (time.perf_counter() - t0) / 1e9, 3)
+    os.close(fd)
+    fd = os.open(path, os.O_RDONLY | flags)
+    t0 = time.perf_counter()
+    for off in range(0, nbytes, chunk):
+        os.preadv(fd, [buf], off)
+    out["read_gbs"] = round(nbytes / (time.perf_counter() - t0) / 1e9, 3)
+    os.close(fd)
+    os.unlink(path)
+    out["o_direct"] = bool(flags)
+    return out
+
+
+def run_file(args, rank: int, world: int, local_rank: int):
+    """S§8(a) a3 / NEXT-4: the GEMM with A, B, C in files on the box's disk:
+    value = FILE -> HOST staging -> HBM (8 GiB cap) -> SMEM/TMEM; the direct
+    edge FILE -> HBM (pinned bounce, or cuFile with NORTHUP_CUFILE=1) beside it;
+    roofline against the measured disk read / write bandwidth."""
+    import shutil
+    import tempfile
+    import numpy as np
+    import torch
+    import nugen
+    import oracle
+    import paper_conf_ipps_chey19_b200 as nu
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    n = args.file_size or 32768
+    if args.quick:
+        n //= 4
+    M = N = K = n
+    panel = 2048 if K >= 2048 else K
+    base = args.file_dir or os.environ.get("NORTHUP_BENCH_FILE_DIR") or "/tmp"
+    free = shutil.disk_usage(base).free
+    if free < 6 * 4 * n * n:
+        return {"metric": METRIC, "unavailable": f"{base}: {free >> 30} GiB free < {6 * 4 * n * n >> 30} GiB"}
+    d = tempfile.mkdtemp(dir=base, prefix="northup_bench_")
+    try:
+        seed = 4
+        a = nugen.fill(M, K, seed, nugen.MAT_A)
+        b = nugen.fill(K, N, seed, nugen.MAT_B)
+        a.tofile(f"{d}/A.bin")
+        b.tofile(f"{d}/B.bin")
+        t0 = time.perf_counter()
+        nu.file_tile_kpanels(f"{d}/A.bin", f"{d}/A_t.bin", M, K, panel)     # R15, outside the timing
+        pre_s = time.perf_counter() - t0
+        os.unlink(f"{d}/A.bin")
+        disk = measure_disk(d)
+        runs = {}
+        for kind in ("staging", "direct"):
+            t = nu.Tree()
+            root = t.add_node(-1, nu.NU_FILE)
+            parent = t.add_node(root, nu.NU_HOST, -1, 0) if kind == "staging" else root
+            h = t.add_node(parent, nu.NU_HBM, local_rank, 8 * GiB)
+            t.add_node(h, nu.NU_SMEM, local_rank, 227 * 1024, nu.NU_PROC_SM100)
+            t.finalize()
+            fa = t.open_file(0, f"{d}/A_t.bin", 4 * M * K)
+            fb = t.open_file(0, f"{d}/B.bin", 4 * K * N)
+            fc = t.open_file(0, f"{d}/C_{kind}.bin", 4 * M * N)
+            o = nu.make_opts(a_panel_k=panel)
+            for _ in range(max(1, args.warmup)):
+                t.gemm(fa, fb, fc, M, N, K, o)
+            ms, st = [], {}
+            for _ in range(args.steps):
+                t0 = time.perf_counter()
+                st = t.gemm(fa, fb, fc, M, N, K, o)     # synchronous: C durable in its file
+                ms.append((time.perf_counter() - t0) * 1e3)
+            t.destroy()
+            c = np.fromfile(f"{d}/C_{kind}.bin", dtype=np.float32).reshape(M, N)
+            rows = np.arange(0, M, max(1, M // 16))
+            ref = oracle.gemm_rows(a, b, rows)
+            e, _ = oracle.normwise_err(np.ascontiguousarray(c[rows]), ref,
+                                       oracle.row_norms(np.ascontiguousarray(a[rows])), oracle.col_norms(b))
+            runs[kind] = {"ms_per_step": round(statistics.mean(ms), 3),
+                          "tflops": round(2.0 * M * N * K / (statistics.mean(ms) * 1e-3) / 1e12, 3),
+                          "file_read_bytes": int(st["bytes_file_read"]), "file_write_bytes": int(st["bytes_file_write"]),
+                          "io_busy_ms": round(st["t_io_ms"], 1), "file_direct_mode": int(st["file_direct_mode"]),
+                          "normwise_err_16_rows": e}
+        peaks = measured_peaks()
+        p_eff = peaks["bf16_sustained"] / 3.0
+        st = runs["staging"]
+        t_disk = st["file_read_bytes"] / (disk["read_gbs"] * 1e9) + st["file_write_bytes"] / (disk["write_gbs"] * 1e9)
+        disk_term = 2.0 * M * N * K / t_disk / 1e12
+        bound = "disk" if disk_term < p_eff else "tensor"
+        peak = min(disk_term, p_eff)
+        value = st["tflops"]
+        return {
+            "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": st["ms_per_step"], "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32 (tcgen05 kind::f16 on a scaled fp16 hi/lo split, fp32 accumulate)",
+            "data": "synthetic (counter-hash uniform [-1,1) fp32 in files on the box's disk)",
+            "config": {"workload": f"file-root: {M}^3 fp32, FILE (no NVMe on the box: virtio disk, {base}) -> "
+                                   f"HOST staging -> HBM (8 GiB cap) -> SMEM/TMEM, 1 GPU",
+                       "M": M, "N": N, "K": K, "a_layout": f"K-panel-major, panel {panel} (R15)",
+                       "preprocess_s": round(pre_s, 2)},
+            "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+                    "file_read_bytes_per_step": st["file_read_bytes"],
+                    "file_write_bytes_per_step": st["file_write_bytes"],
+                    "basis": "host clock around synchronous northup_gemm calls (C written and fdatasync'ed)"},
+            "runs": runs, "disk": disk,
+            "file_roofline": {"bound": bound, "peak": round(peak, 3), "unit": "TFLOP/s",
+                              "terms": {"tensor": round(p_eff, 3), "disk": round(disk_term, 3)},
+                              "achieved": value, "frac": round(value / peak, 4),
+                              "basis": "min(P_eff, 2MNK / (file bytes read / disk read GB/s + file bytes written "
+                                       "/ disk write GB/s)); read and write share the device"},
+            "parity": {"oracle_ok": all(r["normwise_err_16_rows"] <= 1e-5 for r in runs.values())},
+        }
+    finally:
+        shutil.rmtree(d, ignore_errors=True)
+
+
 # --------------------------------------------------------------- reference
 def run_reference(args):
     """The fp64 CPU oracle as the reference arm (bounded sample per step)."""
@@ -847,7 +975,9 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default=None, choices=sorted(CONFIGS) + ["hotspot"])
+    ap.add_argument("--config", default=None, choices=sorted(CONFIGS) + ["hotspot", "file"])
+    ap.add_argument("--file-size", type=int, default=0, help="--config file: M = N = K (default 32768)")
+    ap.add_argument("--file-dir", default=None, help="--config file: where the A, B, C files go")
     ap.add_argument("--k-chunk", type=int, default=2048)
     ap.add_argument("--quick", action="store_true", help="sizes / 4 (smoke-testing the bench)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -886,7 +1016,7 @@ def main():
         local_rank %= args.device_mod
 
     if args.impl == "reference":
-        if rank == 0 and args.config == "hotspot":
+        if rank == 0 and args.config in ("hotspot", "file"):
             print(json.dumps({"impl": "reference", "unavailable": "the HotSpot-2D oracle is timed as cpu_baseline "
                                                                   "in the ours line (no separate reference arm)"}))
             return
@@ -906,6 +1036,7 @@ def main():
         else:
             dist.init_process_group(args.dist_backend)
     res = run_hotspot(args, rank, world, local_rank) if args.config == "hotspot" else \
+        run_file(args, rank, world, local_rank) if args.config == "file" else \
         run_ours(args, rank, world, local_rank)
     if rank == 0 and res is not None:
         print(json.dumps(res), flush=True)
