@@ -3,11 +3,12 @@
 // of the grid resident in HBM, several iterations per launch.
 //
 // The paper's leaf loads a block and its borders into (block+2)^2 local-memory
-// arrays and does one iteration.  Here a CTA loads its 64 x 64 output
-// tile plus an `iters`-wide border of temperature and power into shared
-// memory once and performs all `iters` iterations there (the valid region
-// shrinks by one cell per iteration on every side that is not a grid edge),
-// so HBM is read once and written once per `iters` iterations.
+// arrays and does one iteration.  Here a CTA loads its tile (128
+// columns x 96 rows, output 112 x 80 at 8 iterations) once, keeps temperature
+// in registers and power in shared memory, and performs all `iters`
+// iterations on chip (the valid region shrinks by one cell per iteration on
+// every side that is not a grid edge), so HBM is read once and written once
+// per `iters` iterations.
 //
 // Arithmetic contract (RH4): every cell update is the fixed fp32
 // sequence (round-to-nearest, fma = one rounding)
@@ -26,10 +27,6 @@
 
 namespace nu {
 namespace hs {
-
-constexpr int kTY = 64, kTX = 64;   // output tile per CTA
-constexpr int kWX = 32, kWY = 16;   // 512 threads as 32 x 16
-constexpr int kThreads = kWX * kWY;
 
 struct Args {
   const float* tin;
@@ -54,401 +51,129 @@ __device__ __forceinline__ float update(float t, float p, float n, float s, floa
   return __fmaf_rn(a.cap_1, d, t);
 }
 
-// 4-byte asynchronous global -> shared copies (LDGSTS): every element of the
-// tile is in flight at once instead of one load per thread per loop trip.
-__device__ __forceinline__ void cp_async4(float* smem, const float* gmem) {
-  const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() {
-  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
-}
-
-__global__ void __launch_bounds__(kThreads) hotspot_kernel(Args a) {
-  extern __shared__ float sm[];
-  const int it = a.iters;
-  const int SX = kTX + 2 * it, SY = kTY + 2 * it;
-  float* cur = sm;
-  float* nxt = sm + SY * SX;
-  float* pwr = sm + 2 * SY * SX;
-  const int tx = threadIdx.x, ty = threadIdx.y;
-
-  const int64_t ty0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * kTY;
-  const int64_t tx0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * kTX;
-  const int64_t ty1 = min(ty0 + kTY, a.vy1), tx1 = min(tx0 + kTX, a.vx1);
-  const int64_t sy0 = max(ty0 - it, int64_t(0)), sy1 = min(ty1 + it, a.wm);
-  const int64_t sx0 = max(tx0 - it, int64_t(0)), sx1 = min(tx1 + it, a.wn);
-  const int hy = static_cast<int>(sy1 - sy0), hx = static_cast<int>(sx1 - sx0);
-
-  // data_down HBM -> SMEM: the tile with its borders (coalesced rows, async)
-  for (int y = ty; y < hy; y += kWY) {
-    const float* trow = a.tin + (sy0 + y) * a.ldt + sx0;
-    const float* prow = a.pw + (sy0 + y) * a.ldp + sx0;
-    for (int x = tx; x < hx; x += kWX) {
-      cp_async4(&cur[y * SX + x], trow + x);
-      cp_async4(&pwr[y * SX + x], prow + x);
-    }
-  }
-  cp_async_wait_all();
-  __syncthreads();
-
-  // sides of the shared-memory region that are grid edges (clamped, never shrink)
-  const bool top = a.gy0 + sy0 == 0, bot = a.gy0 + sy1 == a.R;
-  const bool lef = a.gx0 + sx0 == 0, rig = a.gx0 + sx1 == a.C;
-  for (int k = 1; k <= it; ++k) {
-    const int y0 = top ? 0 : k, y1 = bot ? hy : hy - k;
-    const int x0 = lef ? 0 : k, x1 = rig ? hx : hx - k;
-    for (int y = y0 + ty; y < y1; y += kWY) {
-      const int yn = y > 0 ? y - 1 : 0;            // y == 0 only when `top` (clamp)
-      const int ys = y < hy - 1 ? y + 1 : y;       // y == hy - 1 only when `bot`
-      for (int x = x0 + tx; x < x1; x += kWX) {
-        const int xw = x > 0 ? x - 1 : 0;
-        const int xe = x < hx - 1 ? x + 1 : x;
-        nxt[y * SX + x] = update(cur[y * SX + x], pwr[y * SX + x], cur[yn * SX + x], cur[ys * SX + x],
-                                 cur[y * SX + xe], cur[y * SX + xw], a);
-      }
-    }
-    __syncthreads();
-    float* t = cur;
-    cur = nxt;
-    nxt = t;
-  }
-
-  // data_up SMEM -> HBM: the tile
-  const int oy = static_cast<int>(ty0 - sy0), ox = static_cast<int>(tx0 - sx0);
-  const int ny = static_cast<int>(ty1 - ty0), nx = static_cast<int>(tx1 - tx0);
-  for (int y = ty; y < ny; y += kWY) {
-    float* orow = a.tout + (ty0 + y) * a.ldo + tx0;
-    for (int x = tx; x < nx; x += kWX) orow[x] = cur[(oy + y) * SX + ox + x];
-  }
-}
-
 // ---------------------------------------------------------------------------
-// v2: register-blocked.  A CTA owns a region of RH = NWY*RPT rows x RW = NWX*32
-// columns; thread (lane, warp) keeps RPT consecutive cells of one column (and
-// their power) in registers for all iterations.  Per iteration:
-//   * N/S inside the segment come from registers; across segments each thread
-//     publishes its top and bottom cell in shared memory;
-//   * E/W come from warp shuffles; lanes 0 / 31 take the neighbouring warp's
-//     edge column from shared memory;
-//   * one __syncthreads (the exchange arrays are double-buffered by parity).
-// Grid-edge neighbours are clamped per cell, exactly as in v1, and the update
-// is the same function, so v2 is bitwise equal to v1 (tested).
-template <int RPT, int NWX, int NWY>
-__global__ void __launch_bounds__(NWX * NWY * 32, 1) hotspot_kernel_v2(Args a) {
-  constexpr int RW = NWX * 32, RH = NWY * RPT;
-  __shared__ float tops[2][NWY][RW], bots[2][NWY][RW];
-  __shared__ float colL[2][NWX][RH], colR[2][NWX][RH];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int sx = warp % NWX, gyi = warp / NWX;
-  const int h = a.iters;
-  const int OTY = RH - 2 * h, OTX = RW - 2 * h;
-  const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
-  const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
-  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
-  const int x = sx * 32 + lane;                    // column inside the region
-  const int64_t wx = rx + x;                       // window column
-  const int64_t gcol = a.gx0 + wx;                 // grid column
-  const int r0 = gyi * RPT;                        // first row of this segment
-  const bool xin = wx >= 0 && wx < a.wn;
-
-  float v[RPT], p[RPT];
+// v5: a lane owns 4 consecutive columns x V rows in registers, a warp spans
+// the CTA tile's 128 columns, NW warps stack vertically (tile 128 x NW*V).
+// Per iteration: W/E neighbours of the lane's outer columns come from the
+// adjacent lanes (one shfl.up + one shfl.down per row of 4 cells, inner
+// columns from registers), N/S neighbours from registers inside the run and,
+// for the run's first / last row, from the vertically adjacent warps through
+// a double-buffered shared-memory row (one barrier per iteration); power lives
+// in shared memory (one 16-byte load per row of 4 cells).  Same RH4 sequence
+// per cell, so v5 is bitwise equal to the fp32 emulation (and to the
+// round-1 leaves v1-v4, replaced by this one: DESIGN.md §11).
+template <bool EDGE>
+__device__ __forceinline__ float4 v5_row(const float4 c, const float4 p, const float4 n, const float4 s, float wl,
+                                         float er, const Args& a, bool rtop, bool rbot, int cl, int cr) {
+  float nn[4] = {n.x, n.y, n.z, n.w}, ss[4] = {s.x, s.y, s.z, s.w};
+  const float cc[4] = {c.x, c.y, c.z, c.w}, pp[4] = {p.x, p.y, p.z, p.w};
+  float out[4];
 #pragma unroll
-  for (int r = 0; r < RPT; ++r) {
-    const int64_t wy = ry + r0 + r;
-    const bool in = xin && wy >= 0 && wy < a.wm;
-    v[r] = in ? __ldg(a.tin + wy * a.ldt + wx) : 0.0f;
-    p[r] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
-  }
-  // segment rows r with grid row 0 / R - 1 (clamped neighbours); else out of range
-  const int rtop = static_cast<int>(-(a.gy0 + ry + r0));
-  const int rbot = static_cast<int>(a.R - 1 - (a.gy0 + ry + r0));
-  const bool wclamp = gcol == 0, eclamp = gcol == a.C - 1;
-
-  for (int k = 0; k < h; ++k) {
-    const int b = k & 1;
-    tops[b][gyi][x] = v[0];
-    bots[b][gyi][x] = v[RPT - 1];
-    if (lane == 0) {
-#pragma unroll
-      for (int r = 0; r < RPT; ++r) colL[b][sx][r0 + r] = v[r];
+  for (int j = 0; j < 4; ++j) {
+    float w = j > 0 ? cc[j - 1] : wl;
+    float e = j < 3 ? cc[j + 1] : er;
+    float nj = nn[j], sj = ss[j];
+    if (EDGE) {
+      if (rtop) nj = cc[j];
+      if (rbot) sj = cc[j];
+      if (j == cl) w = cc[j];
+      if (j == cr) e = cc[j];
     }
-    if (lane == 31) {
-#pragma unroll
-      for (int r = 0; r < RPT; ++r) colR[b][sx][r0 + r] = v[r];
-    }
-    __syncthreads();
-    const float n0 = gyi > 0 ? bots[b][gyi - 1][x] : v[0];
-    const float sL = gyi < NWY - 1 ? tops[b][gyi + 1][x] : v[RPT - 1];
-    // in place, top to bottom: `above` keeps the old value of the row above
-    float above = n0;
-#pragma unroll
-    for (int r = 0; r < RPT; ++r) {
-      const float c = v[r];
-      float w = __shfl_up_sync(0xffffffffu, c, 1);
-      float e = __shfl_down_sync(0xffffffffu, c, 1);
-      if (lane == 0) w = sx > 0 ? colR[b][sx - 1][r0 + r] : c;
-      if (lane == 31) e = sx < NWX - 1 ? colL[b][sx + 1][r0 + r] : c;
-      float n = above;
-      float s = r < RPT - 1 ? v[r + 1] : sL;
-      if (r == rtop) n = c;                        // grid-edge clamps (as v1)
-      if (r == rbot) s = c;
-      if (wclamp) w = c;
-      if (eclamp) e = c;
-      v[r] = update(c, p[r], n, s, e, w, a);
-      above = c;
-    }
+    out[j] = update(cc[j], pp[j], nj, sj, e, w, a);
   }
-
-  // the output tile: rows [oy0, oy0 + OTY) x cols [ox0, ox0 + OTX) within the valid region
-  if (wx < ox0 || wx >= min(ox0 + OTX, a.vx1)) return;
-  const int64_t ylo = oy0, yhi = min(oy0 + OTY, a.vy1);
-#pragma unroll
-  for (int r = 0; r < RPT; ++r) {
-    const int64_t wy = ry + r0 + r;
-    if (wy >= ylo && wy < yhi) a.tout[wy * a.ldo + wx] = v[r];
-  }
+  return make_float4(out[0], out[1], out[2], out[3]);
 }
 
-// ---------------------------------------------------------------------------
-// v3: register runs + shared-memory plane.  A CTA owns a region of
-// RH = NWY*V rows x RW = NWX*32 columns (plus a one-cell apron in shared
-// memory).  Thread (lane, warp) keeps V consecutive cells of column
-// x = 32*(warp % NWX) + lane, and their power, in registers for all the
-// launch's iterations.  Per iteration it reads the W/E neighbours of its V
-// cells and the cells above / below its run from the current plane, computes
-// V updates, writes them to the next plane, and the CTA synchronises once
-// (two planes alternate).  CTAs whose region touches no grid edge run the
-// clamp-free body; edge CTAs clamp per cell exactly as v1, so v3 is bitwise
-// equal to v1 (tested).
-template <int V, int NWX, int NWY, bool EDGE>
-__device__ __forceinline__ void v3_iterate(const Args& a, float* __restrict__ pl0, float* __restrict__ pl1,
-                                           float (&v)[V], const float (&p)[V], int x, int r0, int rtop,
-                                           int rbot, bool wclamp, bool eclamp) {
-  constexpr int SW = NWX * 32 + 2;   // plane row stride (apron columns 0 and SW - 1)
-  float* cur = pl0;
-  float* nxt = pl1;
+template <int V, int NW, bool EDGE>
+__device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const float* __restrict__ ps,
+                                           float* __restrict__ hb, int lane, int warp, int rtop, int rbot,
+                                           int cl, int cr) {
+  constexpr int RW = 128;
   for (int k = 0; k < a.iters; ++k) {
-    const float* crow = cur + (r0 + 1) * SW + (x + 1);   // this thread's first cell
-    float above = crow[-SW];
-    const float below = crow[V * SW];
+    float* buf = hb + (k & 1) * (NW * 2 * RW);
+    *reinterpret_cast<float4*>(buf + (warp * 2 + 0) * RW + 4 * lane) = v[0];        // my first row
+    *reinterpret_cast<float4*>(buf + (warp * 2 + 1) * RW + 4 * lane) = v[V - 1];    // my last row
+    __syncthreads();
+    float4 prev = warp > 0 ? *reinterpret_cast<const float4*>(buf + ((warp - 1) * 2 + 1) * RW + 4 * lane) : v[0];
+    const float4 below =
+        warp < NW - 1 ? *reinterpret_cast<const float4*>(buf + ((warp + 1) * 2 + 0) * RW + 4 * lane) : v[V - 1];
 #pragma unroll
     for (int r = 0; r < V; ++r) {
-      const float c = v[r];
-      float n = above;
-      float s = r < V - 1 ? v[r + 1] : below;
-      float w = crow[r * SW - 1];
-      float e = crow[r * SW + 1];
-      if (EDGE) {
-        if (r == rtop) n = c;
-        if (r == rbot) s = c;
-        if (wclamp) w = c;
-        if (eclamp) e = c;
-      }
-      v[r] = update(c, p[r], n, s, e, w, a);
-      nxt[(r0 + 1 + r) * SW + x + 1] = v[r];
-      above = c;
+      const float4 c = v[r];
+      const float4 s = r < V - 1 ? v[r + 1] : below;
+      const float wl = __shfl_up_sync(0xffffffffu, c.w, 1);
+      const float er = __shfl_down_sync(0xffffffffu, c.x, 1);
+      float4 p;   // volatile: read per row, not hoisted into registers for all V rows
+      asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                   : "=f"(p.x), "=f"(p.y), "=f"(p.z), "=f"(p.w)
+                   : "r"(static_cast<unsigned>(__cvta_generic_to_shared(ps + (warp * V + r) * RW + 4 * lane))));
+      v[r] = v5_row<EDGE>(c, p, prev, s, wl, er, a, EDGE && r == rtop, EDGE && r == rbot, cl, cr);
+      prev = c;
     }
-    __syncthreads();
-    float* t = cur;
-    cur = nxt;
-    nxt = t;
   }
 }
 
-#ifndef NU_HS_V3_MINB
-#define NU_HS_V3_MINB 1
-#endif
-template <int V, int NWX, int NWY>
-__global__ void __launch_bounds__(NWX * NWY * 32, NU_HS_V3_MINB) hotspot_kernel_v3(Args a) {
-  constexpr int RW = NWX * 32, RH = NWY * V, SW = RW + 2, SH = RH + 2;
-  extern __shared__ float sm3[];
-  float* pl0 = sm3;
-  float* pl1 = sm3 + SH * SW;
+// 2 CTAs per SM (128 registers): one CTA's loads overlap the other's iterations.
+template <int V, int NW>
+__global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
+  constexpr int RW = 128, RH = NW * V;
+  extern __shared__ float sm5[];
+  float* ps = sm5;                 // power tile RH x RW
+  float* hb = sm5 + RH * RW;       // 2 parities x NW warps x {first, last} row x RW
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int x = (warp % NWX) * 32 + lane, r0 = (warp / NWX) * V;
   const int h = a.iters;
   const int OTY = RH - 2 * h, OTX = RW - 2 * h;
   const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
   const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
-  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
-  const int64_t wx = rx + x;
-  const bool xin = wx >= 0 && wx < a.wn;
-  float v[V], p[V];
+  const int64_t ry = oy0 - h, rx = ox0 - h;        // tile origin (window coordinates)
+  const int r0 = warp * V, x0 = 4 * lane;
+  float4 v[V];
 #pragma unroll
   for (int r = 0; r < V; ++r) {
     const int64_t wy = ry + r0 + r;
-    const bool in = xin && wy >= 0 && wy < a.wm;
-    v[r] = in ? __ldg(a.tin + wy * a.ldt + wx) : 0.0f;
-    p[r] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
-  }
+    const bool yin = wy >= 0 && wy < a.wm;
+    float t[4], p[4];
 #pragma unroll
-  for (int r = 0; r < V; ++r) pl0[(r0 + 1 + r) * SW + x + 1] = v[r];
-  __syncthreads();
-  // does the region touch a grid edge?  (uniform per CTA)
-  const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
-  const bool edge = gy_top <= 0 || gy_top + RH >= a.R || gx_left <= 0 || gx_left + RW >= a.C;
-  if (edge) {
-    const int rtop = static_cast<int>(-(gy_top + r0));
-    const int rbot = static_cast<int>(a.R - 1 - (gy_top + r0));
-    const int64_t gcol = gx_left + x;
-    v3_iterate<V, NWX, NWY, true>(a, pl0, pl1, v, p, x, r0, rtop, rbot, gcol == 0, gcol == a.C - 1);
-  } else {
-    v3_iterate<V, NWX, NWY, false>(a, pl0, pl1, v, p, x, r0, 0, 0, false, false);
-  }
-  // store: recompute the coordinates (keeps them out of the iteration's registers)
-  const int64_t oy = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
-  const int64_t ox = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
-  const int64_t sx = ox - h + x;
-  if (sx < ox || sx >= min(ox + OTX, a.vx1)) return;
-  const int ylo = h - r0, yhi = static_cast<int>(min(oy + OTY, a.vy1) - (oy - h)) - r0;
-  float* out = a.tout + (oy - h + r0) * a.ldo + sx;
-#pragma unroll
-  for (int r = 0; r < V; ++r)
-    if (r >= ylo && r < yhi) out[r * a.ldo] = v[r];
-}
-
-// ---------------------------------------------------------------------------
-// v4: v3 with packed fp32x2 arithmetic (sm_100 FADD2 / FFMA2).  Thread
-// (lane, warp) keeps the same V-cell column run as v3, held as V/2 pairs
-// (row j, row j + V/2) in 64-bit registers, so one packed instruction updates
-// two cells.  The shared-memory planes store the runs in the same pair layout
-// (pair-row j of run `seg` at pair-row seg*V/2 + j + 1), so the W/E neighbour
-// pairs are aligned 8-byte loads and the new pair one 8-byte store.  Each lane
-// of FADD2/FFMA2 is an IEEE round-to-nearest add / fused multiply-add, and
-// amb - t is formed as fma(-1, t, amb) (one rounding of the exact difference),
-// so every cell follows the RH4 sequence bit for bit: v4 equals v1-v3.
-__device__ __forceinline__ float2 update2(float2 t, float2 p, float2 n, float2 s, float2 e, float2 w,
-                                          float2 ry, float2 rx, float2 rz, float2 cap, float2 amb) {
-  const float2 m2 = make_float2(-2.0f, -2.0f), m1 = make_float2(-1.0f, -1.0f);
-  const float2 ay = __ffma2_rn(m2, t, __fadd2_rn(s, n));
-  const float2 ax = __ffma2_rn(m2, t, __fadd2_rn(e, w));
-  float2 d = __ffma2_rn(ay, ry, p);
-  d = __ffma2_rn(ax, rx, d);
-  d = __ffma2_rn(__ffma2_rn(m1, t, amb), rz, d);
-  return __ffma2_rn(cap, d, t);
-}
-
-template <int V, int NWX, int NWY, bool EDGE>
-__device__ __forceinline__ void v4_iterate(const Args& a, float2* __restrict__ pl0, float2* __restrict__ pl1,
-                                           float2 (&v)[V / 2], const float2 (&p)[V / 2], int x, int pr0,
-                                           int rtop, int rbot, bool wclamp, bool eclamp) {
-  constexpr int SW = NWX * 32 + 2, H = V / 2;
-  const float2 ry = make_float2(a.ry_1, a.ry_1), rx = make_float2(a.rx_1, a.rx_1);
-  const float2 rz = make_float2(a.rz_1, a.rz_1), cap = make_float2(a.cap_1, a.cap_1);
-  const float2 amb = make_float2(a.amb, a.amb);
-  float2* cur = pl0;
-  float2* nxt = pl1;
-  for (int k = 0; k < a.iters; ++k) {
-    const float2* crow = cur + pr0 * SW + (x + 1);   // this thread's first pair
-    const float above = crow[-SW].y;                 // row -1 of the run
-    const float below = crow[H * SW].x;              // row V of the run
-    float2 prev = make_float2(above, v[H - 1].x);    // north pair of pair 0
-    const float mid = v[0].y;                        // row H (south of row H - 1), pre-update
-#pragma unroll
-    for (int j = 0; j < H; ++j) {
-      const float2 c = v[j];
-      float2 n = prev;
-      float2 s = j < H - 1 ? v[j + 1] : make_float2(mid, below);
-      float2 w = crow[j * SW - 1];
-      float2 e = crow[j * SW + 1];
-      if (EDGE) {
-        if (j == rtop) n.x = c.x;
-        if (j + H == rtop) n.y = c.y;
-        if (j == rbot) s.x = c.x;
-        if (j + H == rbot) s.y = c.y;
-        if (wclamp) w = c;
-        if (eclamp) e = c;
-      }
-      v[j] = update2(c, p[j], n, s, e, w, ry, rx, rz, cap, amb);
-      nxt[(pr0 + j) * SW + x + 1] = v[j];
-      prev = c;
+    for (int j = 0; j < 4; ++j) {
+      const int64_t wx = rx + x0 + j;
+      const bool in = yin && wx >= 0 && wx < a.wn;
+      t[j] = in ? __ldg(a.tin + wy * a.ldt + wx) : 0.0f;
+      p[j] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
     }
-    __syncthreads();
-    float2* t = cur;
-    cur = nxt;
-    nxt = t;
+    v[r] = make_float4(t[0], t[1], t[2], t[3]);
+    *reinterpret_cast<float4*>(ps + (r0 + r) * RW + x0) = make_float4(p[0], p[1], p[2], p[3]);
   }
-}
-
-#ifndef NU_HS_V4_MINB
-#define NU_HS_V4_MINB 1
-#endif
-template <int V, int NWX, int NWY>
-__global__ void __launch_bounds__(NWX * NWY * 32, NU_HS_V4_MINB) hotspot_kernel_v4(Args a) {
-  constexpr int RW = NWX * 32, RH = NWY * V, H = V / 2, SW = RW + 2, SPR = NWY * H + 2;
-  extern __shared__ float2 sm4[];
-  float2* pl0 = sm4;
-  float2* pl1 = sm4 + SPR * SW;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int seg = warp / NWX;
-  const int x = (warp % NWX) * 32 + lane, r0 = seg * V, pr0 = seg * H + 1;
-  const int h = a.iters;
-  const int OTY = RH - 2 * h, OTX = RW - 2 * h;
-  const int64_t oy0 = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
-  const int64_t ox0 = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
-  const int64_t ry = oy0 - h, rx = ox0 - h;        // region origin (window coordinates)
-  const int64_t wx = rx + x;
-  const bool xin = wx >= 0 && wx < a.wn;
-  float2 v[H], p[H];
-#pragma unroll
-  for (int j = 0; j < H; ++j) {
-    const int64_t wy0 = ry + r0 + j, wy1 = wy0 + H;
-    const bool in0 = xin && wy0 >= 0 && wy0 < a.wm, in1 = xin && wy1 >= 0 && wy1 < a.wm;
-    v[j] = make_float2(in0 ? __ldg(a.tin + wy0 * a.ldt + wx) : 0.0f, in1 ? __ldg(a.tin + wy1 * a.ldt + wx) : 0.0f);
-    p[j] = make_float2(in0 ? __ldg(a.pw + wy0 * a.ldp + wx) : 0.0f, in1 ? __ldg(a.pw + wy1 * a.ldp + wx) : 0.0f);
-  }
-#pragma unroll
-  for (int j = 0; j < H; ++j) pl0[(pr0 + j) * SW + x + 1] = v[j];
-  __syncthreads();
+  // (the first iteration's barrier also orders these power stores)
   const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
   const bool edge = gy_top <= 0 || gy_top + RH >= a.R || gx_left <= 0 || gx_left + RW >= a.C;
   if (edge) {
-    const int rtop = static_cast<int>(-(gy_top + r0));
-    const int rbot = static_cast<int>(a.R - 1 - (gy_top + r0));
-    const int64_t gcol = gx_left + x;
-    v4_iterate<V, NWX, NWY, true>(a, pl0, pl1, v, p, x, pr0, rtop, rbot, gcol == 0, gcol == a.C - 1);
+    const int64_t gx = gx_left + x0;   // grid column of this lane's first cell
+    const int cl = (gx <= 0 && gx > -4) ? static_cast<int>(-gx) : -1;
+    const int cr = (a.C - 1 - gx >= 0 && a.C - 1 - gx < 4) ? static_cast<int>(a.C - 1 - gx) : -1;
+    const int64_t gy = gy_top + r0;    // grid row of this thread's first cell
+    const int rtop = (gy <= 0 && gy > -V) ? static_cast<int>(-gy) : -1;
+    const int rbot = (a.R - 1 - gy >= 0 && a.R - 1 - gy < V) ? static_cast<int>(a.R - 1 - gy) : -1;
+    v5_iterate<V, NW, true>(a, v, ps, hb, lane, warp, rtop, rbot, cl, cr);
   } else {
-    v4_iterate<V, NWX, NWY, false>(a, pl0, pl1, v, p, x, pr0, 0, 0, false, false);
+    v5_iterate<V, NW, false>(a, v, ps, hb, lane, warp, -1, -1, -1, -1);
   }
-  const int64_t oy = a.vy0 + static_cast<int64_t>(blockIdx.y) * OTY;
-  const int64_t ox = a.vx0 + static_cast<int64_t>(blockIdx.x) * OTX;
-  const int64_t sx = ox - h + x;
-  if (sx < ox || sx >= min(ox + OTX, a.vx1)) return;
-  const int ylo = h - r0, yhi = static_cast<int>(min(oy + OTY, a.vy1) - (oy - h)) - r0;
-  float* out = a.tout + (oy - h + r0) * a.ldo + sx;
+  const int64_t oy = oy0, ox = ox0;
+  const int64_t ylo = max(oy, a.vy0), yhi = min(oy + OTY, a.vy1);
+  const int64_t xlo = max(ox, a.vx0), xhi = min(ox + OTX, a.vx1);
 #pragma unroll
-  for (int j = 0; j < H; ++j) {
-    if (j >= ylo && j < yhi) out[j * a.ldo] = v[j].x;
-    if (j + H >= ylo && j + H < yhi) out[(j + H) * a.ldo] = v[j].y;
+  for (int r = 0; r < V; ++r) {
+    const int64_t wy = ry + r0 + r;
+    if (wy < ylo || wy >= yhi) continue;
+    const float t[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t wx = rx + x0 + j;
+      if (wx >= xlo && wx < xhi) a.tout[wy * a.ldo + wx] = t[j];
+    }
   }
 }
 
-#ifndef NU_HS_V3_V
-#define NU_HS_V3_V 16
-#endif
-#ifndef NU_HS_V3_NWY
-#define NU_HS_V3_NWY 8
-#endif
-constexpr int kV3V = NU_HS_V3_V, kV3NWX = 4, kV3NWY = NU_HS_V3_NWY;
-#ifndef NU_HS_V4_NWX
-#define NU_HS_V4_NWX 4
-#endif
-#ifndef NU_HS_V4_NWY
-#define NU_HS_V4_NWY 8
-#endif
-#ifndef NU_HS_V4_V
-#define NU_HS_V4_V 16
-#endif
-constexpr int kV4V = NU_HS_V4_V, kV4NWX = NU_HS_V4_NWX, kV4NWY = NU_HS_V4_NWY;
-
-#ifndef NU_HS_RPT
-#define NU_HS_RPT 32
-#endif
-#ifndef NU_HS_NWY
-#define NU_HS_NWY 3
-#endif
-constexpr int kRPT = NU_HS_RPT, kNWX = 4, kNWY = NU_HS_NWY;   // 96 x 128 region, 384 threads
+constexpr int kV5V = 12, kV5NW = 8;   // V rows per thread (registers), NW warps per CTA
 
 }  // namespace hs
 
@@ -457,17 +182,9 @@ int hotspot_max_iters_per_launch() { return kHotspotMaxIters; }
 void hotspot_preload() {
   using namespace hs;
   cudaFuncAttributes fa;
-  cudaFuncGetAttributes(&fa, hotspot_kernel);
-  cudaFuncGetAttributes(&fa, hotspot_kernel_v2<kRPT, kNWX, kNWY>);
-  cudaFuncGetAttributes(&fa, hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY>);
-  cudaFuncGetAttributes(&fa, hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY>);
+  cudaFuncGetAttributes(&fa, hotspot_kernel_v5<kV5V, kV5NW>);
 }
 
-static int hotspot_variant() {
-  // read per launch (a getenv next to a kernel launch), so tests can switch leaves
-  const char* e = getenv("NORTHUP_HS_LEAF");
-  return (e && e[0] >= '1' && e[0] <= '4') ? e[0] - '0' : 3;   // 1, 2, 3: earlier leaves (DESIGN)
-}
 
 int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, float* tout,
                    int64_t ldo, int64_t wm, int64_t wn, int64_t gy0, int64_t gx0, int64_t R,
@@ -507,54 +224,19 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.ry_1 = coef[2];
   a.rz_1 = coef[3];
   a.amb = coef[4];
-  if (hotspot_variant() == 4) {
-    constexpr int RH = kV4V * kV4NWY, RW = 32 * kV4NWX;
+  {
+    constexpr int RH = kV5V * kV5NW, RW = 128;
     const int oty = RH - 2 * iters, otx = RW - 2 * iters;
-    const int64_t gy4 = (a.vy1 - a.vy0 + oty - 1) / oty, gx4 = (a.vx1 - a.vx0 + otx - 1) / otx;
-    if (gy4 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy4);
-    const int smem4 = 2 * (kV4NWY * kV4V / 2 + 2) * (RW + 2) * 8;
-    cudaFuncSetAttribute(hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY>,
-                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem4);
-    hotspot_kernel_v4<kV4V, kV4NWX, kV4NWY><<<dim3(static_cast<unsigned>(gx4), static_cast<unsigned>(gy4)),
-                                             kV4NWX * kV4NWY * 32, smem4, stream>>>(a);
+    const int64_t gy5 = (a.vy1 - a.vy0 + oty - 1) / oty, gx5 = (a.vx1 - a.vx0 + otx - 1) / otx;
+    if (gy5 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy5);
+    const int smem5 = (RH * RW + 2 * kV5NW * 2 * RW) * 4;
+    cudaFuncSetAttribute(hotspot_kernel_v5<kV5V, kV5NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem5);
+    hotspot_kernel_v5<kV5V, kV5NW><<<dim3(static_cast<unsigned>(gx5), static_cast<unsigned>(gy5)), kV5NW * 32,
+                                     smem5, stream>>>(a);
     count_launches(1);
     cudaError_t e = cudaGetLastError();
-    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v4 launch");
+    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v5 launch");
   }
-  if (hotspot_variant() == 3) {
-    constexpr int RH = kV3V * kV3NWY, RW = 32 * kV3NWX;
-    const int oty = RH - 2 * iters, otx = RW - 2 * iters;
-    const int64_t gy3 = (a.vy1 - a.vy0 + oty - 1) / oty, gx3 = (a.vx1 - a.vx0 + otx - 1) / otx;
-    if (gy3 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy3);
-    const int smem3 = 2 * (RH + 2) * (RW + 2) * 4;
-    cudaFuncSetAttribute(hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY>,
-                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem3);
-    hotspot_kernel_v3<kV3V, kV3NWX, kV3NWY><<<dim3(static_cast<unsigned>(gx3), static_cast<unsigned>(gy3)),
-                                             kV3NWX * kV3NWY * 32, smem3, stream>>>(a);
-    count_launches(1);
-    cudaError_t e = cudaGetLastError();
-    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v3 launch");
-  }
-  if (hotspot_variant() == 2) {
-    const int oty = kRPT * kNWY - 2 * iters, otx = 32 * kNWX - 2 * iters;
-    const int64_t gy2 = (a.vy1 - a.vy0 + oty - 1) / oty, gx2 = (a.vx1 - a.vx0 + otx - 1) / otx;
-    if (gy2 > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy2);
-    hotspot_kernel_v2<kRPT, kNWX, kNWY><<<dim3(static_cast<unsigned>(gx2), static_cast<unsigned>(gy2)),
-                                          kNWX * kNWY * 32, 0, stream>>>(a);
-    count_launches(1);
-    cudaError_t e = cudaGetLastError();
-    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_v2 launch");
-  }
-  const int64_t gy = (a.vy1 - a.vy0 + kTY - 1) / kTY, gx = (a.vx1 - a.vx0 + kTX - 1) / kTX;
-  if (gy > 65535) return fail(NU_EINVAL, "hotspot window too tall (%lld tile rows)", (long long)gy);
-  const size_t smem = 3ull * (kTY + 2 * iters) * (kTX + 2 * iters) * sizeof(float);
-  // per device context; cheap next to a launch
-  cudaFuncSetAttribute(hotspot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       static_cast<int>(3ull * (kTY + 2 * kHotspotMaxIters) * (kTX + 2 * kHotspotMaxIters) * 4));
-  hotspot_kernel<<<dim3(static_cast<unsigned>(gx), static_cast<unsigned>(gy)), dim3(kWX, kWY), smem, stream>>>(a);
-  count_launches(1);
-  cudaError_t e = cudaGetLastError();
-  return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel launch");
 }
 
 }  // namespace nu

@@ -118,14 +118,13 @@ def test_in_hbm_leaf_iters_invariance():
     assert np.array_equal(a, b) and np.array_equal(a, c)
 
 
-@pytest.mark.parametrize("variant", ["1", "2", "3", "4"])
-@pytest.mark.parametrize("R,C,iters", [(700, 900, 8), (129, 131, 3), (1, 257, 5), (300, 2, 7)])
-def test_leaf_variants_bitwise(variant, R, C, iters, monkeypatch):
-    """Every leaf (v1 shared-memory tiles, v2 register shuffles, v3 register
-    runs, v4 packed fp32x2 runs) evaluates RH4's sequence per cell, so each
-    equals the exact fp32 emulation bit for bit — whole grids (edge CTAs) and
-    grids large enough for clamp-free interior CTAs."""
-    monkeypatch.setenv("NORTHUP_HS_LEAF", variant)
+@pytest.mark.parametrize("R,C,iters", [(700, 900, 8), (129, 131, 3), (1, 257, 5), (300, 2, 7), (97, 129, 8),
+                                        (450, 333, 6), (1000, 1200, 8)])
+def test_leaf_bitwise_vs_emulation(R, C, iters):
+    """The leaf (v5: 4 columns x 12 rows per thread, shuffled W/E, shared-memory
+    N/S halo rows) evaluates RH4's sequence per cell, so it equals the exact
+    fp32 emulation bit for bit — whole grids (edge CTAs, tile-size boundaries
+    at 96 / 128 cells) and grids large enough for clamp-free interior CTAs."""
     T, P = grids(R, C, seed=R + 3 * C)
     dev = torch.device("cuda", 0)
     t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
