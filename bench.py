@@ -752,6 +752,7 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     cpu_cells = sum((min(R, y + 32 + iters) - max(0, y - iters)) * (min(C, x + 32 + iters) - max(0, x - iters))
                     for y, x in samples) * iters
     tol = ohs.tolerance(iters, tmax)
+    pcie_gcups = cells / (st_o.get("bytes_h2d", 1) / 53e9) / 1e9
     result = {
         "metric": "out-of-core HotSpot-2D cell updates/s (S§8(f) NEXT-3); % slowdown vs in-HBM; roofline frac",
         "value": round(value, 3), "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
@@ -768,14 +769,19 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
                 "h2d_bytes_per_step": int(st_o.get("bytes_h2d", 0)),
                 "d2h_bytes_per_step": int(st_o.get("bytes_d2h", 0)), "ms_per_step": round(ms_o, 3),
                 "leaf_launches_per_step": int(st_o.get("leaf_launches", 0)),
-                "pcie_roofline_gcups": round(cells / (st_o.get("bytes_h2d", 1) / 53e9) / 1e9, 1)},
+                "pcie_roofline_gcups": round(pcie_gcups, 1)},
         "slowdown_pct_vs_in_hbm": round(100.0 * (ms_o / ms_h - 1.0), 2),
+        "e2e_roofline": {"bound": "pcie_h2d" if pcie_gcups < in_hbm else "alu",
+                         "peak": round(min(pcie_gcups, in_hbm), 1), "unit": "Gcell-updates/s",
+                         "frac": round(value / min(pcie_gcups, in_hbm), 4),
+                         "basis": "min(H2D bytes of the plan at 53 GB/s, the in-HBM rate): T and P windows "
+                                  "cross PCIe once per pass"},
         "paper_context": {"hotspot_ooc_gap_pct": 15, "note": "APU + SSD vs DRAM (PAPER.md P:381); context only"},
         "roofline": {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "TFLOP/s",
                      "frac": round(achieved / peak, 4), "traffic": None,
                      "peak_basis": f"dense fp32 peak: {N_SMS} SMs x {FP32_LANES_PER_SM} lanes x 2 flops (FMA) x "
                                    f"clocks.max.sm {f_max / 1e6:.0f} MHz",
-                     "kernel": "nu::hs::hotspot_kernel_v5", "launch": [R, C, li],
+                     "kernel": "nu::hs::hotspot_kernel_tma", "launch": [R, C, li],
                      "flops_per_launch": flops_per_launch,
                      "flops_basis": f"{HS_FLOPS_PER_UPDATE} flops per useful cell update (the update's "
                                     f"5 multiplies + 9 adds; the kernel issues 3 FADD + 6 FFMA) x R x C x "

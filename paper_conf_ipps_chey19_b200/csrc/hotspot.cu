@@ -3,12 +3,14 @@
 // of the grid resident in HBM, several iterations per launch.
 //
 // The paper's leaf loads a block and its borders into (block+2)^2 local-memory
-// arrays and does one iteration.  Here a CTA loads its tile (128
-// columns x 96 rows, output 112 x 80 at 8 iterations) once, keeps temperature
-// in registers and power in shared memory, and performs all `iters`
-// iterations on chip (the valid region shrinks by one cell per iteration on
-// every side that is not a grid edge), so HBM is read once and written once
-// per `iters` iterations.
+// arrays and does one iteration.  Here a tile (128 x 128 cells, output
+// 112 x 112 at 8 iterations) is loaded once, temperature is kept in registers
+// and power in shared memory, and all `iters` iterations run on chip (the valid
+// region shrinks by one cell per iteration on every side that is not a grid
+// edge), so HBM is read once and written once per `iters` iterations.  The
+// product kernel (hotspot_kernel_tma) is persistent and loads the next tile by
+// TMA while the current one iterates; hotspot_kernel_v5 (128 x 96 tiles, plain
+// loads) serves windows whose base or leading dimension is not 16-byte aligned.
 //
 // Arithmetic contract (RH4): every cell update is the fixed fp32
 // sequence (round-to-nearest, fma = one rounding)
@@ -23,6 +25,9 @@
 #include <stdint.h>
 #include <stdlib.h>
 
+#include <algorithm>
+
+#include "leaf_common.cuh"
 #include "northup_internal.h"
 
 namespace nu {
@@ -62,6 +67,16 @@ __device__ __forceinline__ float update(float t, float p, float n, float s, floa
 // in shared memory (one 16-byte load per row of 4 cells).  Same RH4 sequence
 // per cell, so v5 is bitwise equal to the fp32 emulation (and to the
 // round-1 leaves v1-v4, replaced by this one: DESIGN.md §11).
+// Power row segment from shared memory.  volatile: read where written (one row
+// ahead of its use), not hoisted into registers for all rows of the run.
+__device__ __forceinline__ float4 ld_power(const float* q) {
+  float4 p;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(p.x), "=f"(p.y), "=f"(p.z), "=f"(p.w)
+               : "r"(static_cast<unsigned>(__cvta_generic_to_shared(q))));
+  return p;
+}
+
 template <bool EDGE>
 __device__ __forceinline__ float4 v5_row(const float4 c, const float4 p, const float4 n, const float4 s, float wl,
                                          float er, const Args& a, bool rtop, bool rbot, int cl, int cr) {
@@ -84,29 +99,48 @@ __device__ __forceinline__ float4 v5_row(const float4 c, const float4 p, const f
   return make_float4(out[0], out[1], out[2], out[3]);
 }
 
-template <int V, int NW, bool EDGE>
+// NAMED: synchronise the NW compute warps on named barrier 1 instead of
+// __syncthreads.  The halo buffer's parity continues from `k0` so consecutive
+// iterations, also across tiles, never share a buffer.  (Waiting on the two
+// vertical neighbours' mbarriers instead of a CTA-wide barrier was measured
+// slower: the polling costs more issue slots than the barrier skew.)
+template <int V, int NW, bool EDGE, bool NAMED = false>
 __device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const float* __restrict__ ps,
                                            float* __restrict__ hb, int lane, int warp, int rtop, int rbot,
-                                           int cl, int cr) {
+                                           int cl, int cr, int k0 = 0) {
   constexpr int RW = 128;
   for (int k = 0; k < a.iters; ++k) {
-    float* buf = hb + (k & 1) * (NW * 2 * RW);
+    float* buf = hb + ((k0 + k) & 1) * (NW * 2 * RW);
     *reinterpret_cast<float4*>(buf + (warp * 2 + 0) * RW + 4 * lane) = v[0];        // my first row
     *reinterpret_cast<float4*>(buf + (warp * 2 + 1) * RW + 4 * lane) = v[V - 1];    // my last row
-    __syncthreads();
-    float4 prev = warp > 0 ? *reinterpret_cast<const float4*>(buf + ((warp - 1) * 2 + 1) * RW + 4 * lane) : v[0];
-    const float4 below =
-        warp < NW - 1 ? *reinterpret_cast<const float4*>(buf + ((warp + 1) * 2 + 0) * RW + 4 * lane) : v[V - 1];
+    if (NAMED)
+      asm volatile("bar.sync 1, %0;" ::"n"(NW * 32) : "memory");
+    else
+      __syncthreads();
+    // The tile's top (bottom) warp reads its own row as the northern (southern)
+    // neighbour: a select on the index, no branch.  Those rows lie in the
+    // tile's recomputed margin (never written back) unless they are the grid
+    // edge, where v5_row's clamp replaces the neighbour anyway.
+    const int up = warp > 0 ? (warp - 1) * 2 + 1 : 0, dn = warp < NW - 1 ? (warp + 1) * 2 : (NW - 1) * 2 + 1;
+    float4 prev = *reinterpret_cast<const float4*>(buf + up * RW + 4 * lane);
+    const float4 below = *reinterpret_cast<const float4*>(buf + dn * RW + 4 * lane);
+    // Row r's W/E shuffles and power load are issued one row ahead, so their
+    // latency hides behind row r-1's arithmetic (4 warps per SM sub-partition
+    // are too few to cover it otherwise).
+    float wl_n = __shfl_up_sync(0xffffffffu, v[0].w, 1);
+    float er_n = __shfl_down_sync(0xffffffffu, v[0].x, 1);
+    float4 p_n = ld_power(ps + (warp * V) * RW + 4 * lane);
 #pragma unroll
     for (int r = 0; r < V; ++r) {
       const float4 c = v[r];
       const float4 s = r < V - 1 ? v[r + 1] : below;
-      const float wl = __shfl_up_sync(0xffffffffu, c.w, 1);
-      const float er = __shfl_down_sync(0xffffffffu, c.x, 1);
-      float4 p;   // volatile: read per row, not hoisted into registers for all V rows
-      asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
-                   : "=f"(p.x), "=f"(p.y), "=f"(p.z), "=f"(p.w)
-                   : "r"(static_cast<unsigned>(__cvta_generic_to_shared(ps + (warp * V + r) * RW + 4 * lane))));
+      const float wl = wl_n, er = er_n;
+      const float4 p = p_n;
+      if (r + 1 < V) {
+        wl_n = __shfl_up_sync(0xffffffffu, v[r + 1].w, 1);
+        er_n = __shfl_down_sync(0xffffffffu, v[r + 1].x, 1);
+        p_n = ld_power(ps + (warp * V + r + 1) * RW + 4 * lane);
+      }
       v[r] = v5_row<EDGE>(c, p, prev, s, wl, er, a, EDGE && r == rtop, EDGE && r == rbot, cl, cr);
       prev = c;
     }
@@ -173,6 +207,118 @@ __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// Persistent TMA leaf (the product kernel when the window's base and leading
+// dimensions are 16-byte aligned): one CTA per SM walks the tiles
+// (128 x 128, output 112 x 112 at 8 iterations) with 16 compute warps (a lane
+// owns 4 columns x 8 rows, the v5 scheme above); thread 0 also issues the
+// loads.  While the warps iterate tile i, TMA brings tile i+1's
+// temperature (single buffer, freed as soon as the compute warps have copied
+// it into registers) and power (double buffer) into shared memory, so HBM
+// traffic overlaps the arithmetic instead of alternating with it.  Out-of-window
+// cells are zero-filled by TMA, as v5's predicated loads do.
+constexpr int kPW = 16, kPV = 8, kPRH = kPW * kPV, kPRW = 128;
+constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 64 KiB
+constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 32 KiB
+constexpr int kPSmem = 3 * kPTileBytes + kPHaloFloats * 4 + 64;   // T | P[2] | halo | barriers
+
+__device__ __forceinline__ void tma_load_tile(uint32_t dst, const CUtensorMap* map, int x, int y, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(bar)
+      : "memory");
+}
+
+__global__ void __launch_bounds__(kPW * 32, 1)
+    hotspot_kernel_tma(const __grid_constant__ CUtensorMap mT, const __grid_constant__ CUtensorMap mP, Args a,
+                       int tiles_x, int tiles, int rx0, int sx, bool vec_out) {
+  using namespace nu::leaf;
+  extern __shared__ __align__(128) float smp[];
+  float* tb = smp;                                   // temperature of the next tile
+  float* pb = smp + kPRH * kPRW;                     // power, two tiles
+  float* hb = smp + 3 * kPRH * kPRW;                 // halo rows
+  uint64_t* bars = reinterpret_cast<uint64_t*>(hb + kPHaloFloats);
+  const uint32_t full0 = smem_u32(bars), pempty0 = smem_u32(bars + 2), tempty = smem_u32(bars + 4);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int h = a.iters, OTY = kPRH - 2 * h;
+  // Thread 0 is also the producer: it issues tile j's two TMA loads (T into
+  // the single T buffer, P into P buffer j % 2), both completing on full[j % 2].
+  auto issue = [&](int j, int t) {
+    const int by = t / tiles_x, bx = t - by * tiles_x;
+    const int ry = static_cast<int>(a.vy0) + by * OTY - h, rx = rx0 + bx * sx;
+    const uint32_t fb = full0 + 8 * (j & 1);
+    mbar_arrive_expect_tx(fb, 2 * kPTileBytes);
+    tma_load_tile(smem_u32(tb), &mT, rx, ry, fb);
+    tma_load_tile(smem_u32(pb + (j & 1) * kPRH * kPRW), &mP, rx, ry, fb);
+  };
+  if (threadIdx.x == 0) {
+    mbar_init(full0, 1);
+    mbar_init(full0 + 8, 1);
+    mbar_init(pempty0, kPW);
+    mbar_init(pempty0 + 8, kPW);
+    mbar_init(tempty, kPW);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    prefetch_tmap(&mT);
+    prefetch_tmap(&mP);
+    if (static_cast<int>(blockIdx.x) < tiles) issue(0, blockIdx.x);
+  }
+  __syncthreads();
+  const int r0 = warp * kPV, x0 = 4 * lane;
+  int i = 0;
+  for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
+    const int by = t / tiles_x, bx = t - by * tiles_x;
+    const int64_t oy0 = a.vy0 + static_cast<int64_t>(by) * OTY;
+    const int64_t ry = oy0 - h, rx = rx0 + static_cast<int64_t>(bx) * sx;
+    mbar_wait(full0 + 8 * (i & 1), (i >> 1) & 1);
+    float4 v[kPV];
+#pragma unroll
+    for (int r = 0; r < kPV; ++r) v[r] = *reinterpret_cast<const float4*>(tb + (r0 + r) * kPRW + x0);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(tempty);
+    if (threadIdx.x == 0 && t + static_cast<int>(gridDim.x) < tiles) {
+      mbar_wait(tempty, i & 1);                                        // every warp holds tile i's T
+      if (i >= 1) mbar_wait(pempty0 + 8 * ((i + 1) & 1), ((i - 1) >> 1) & 1);   // tile i-1 done with its P
+      issue(i + 1, t + gridDim.x);
+    }
+    __syncwarp();
+    const float* ps = pb + (i & 1) * kPRH * kPRW;
+    const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
+    const bool edge = gy_top <= 0 || gy_top + kPRH >= a.R || gx_left <= 0 || gx_left + kPRW >= a.C;
+    if (edge) {
+      const int64_t gx = gx_left + x0;
+      const int cl = (gx <= 0 && gx > -4) ? static_cast<int>(-gx) : -1;
+      const int cr = (a.C - 1 - gx >= 0 && a.C - 1 - gx < 4) ? static_cast<int>(a.C - 1 - gx) : -1;
+      const int64_t gy = gy_top + r0;
+      const int rtop = (gy <= 0 && gy > -kPV) ? static_cast<int>(-gy) : -1;
+      const int rbot = (a.R - 1 - gy >= 0 && a.R - 1 - gy < kPV) ? static_cast<int>(a.R - 1 - gy) : -1;
+      v5_iterate<kPV, kPW, true, true>(a, v, ps, hb, lane, warp, rtop, rbot, cl, cr, i * h);
+    } else {
+      v5_iterate<kPV, kPW, false, true>(a, v, ps, hb, lane, warp, -1, -1, -1, -1, i * h);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(pempty0 + 8 * (i & 1));
+    const int64_t ylo = max(oy0, a.vy0), yhi = min(oy0 + OTY, a.vy1);
+    const int64_t xlo = max(rx + h, a.vx0), xhi = min(rx + h + sx, a.vx1);
+    const int64_t wx = rx + x0;
+    const bool full4 = vec_out && wx >= xlo && wx + 4 <= xhi;    // 16-B aligned: rx, ldo, tout
+    float* orow = a.tout + (ry + r0) * a.ldo + wx;
+#pragma unroll
+    for (int r = 0; r < kPV; ++r, orow += a.ldo) {
+      const int64_t wy = ry + r0 + r;
+      if (wy < ylo || wy >= yhi) continue;
+      if (full4) {
+        *reinterpret_cast<float4*>(orow) = v[r];
+      } else {
+        const float tv[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          if (wx + j >= xlo && wx + j < xhi) orow[j] = tv[j];
+      }
+    }
+  }
+}
+
 constexpr int kV5V = 12, kV5NW = 8;   // V rows per thread (registers), NW warps per CTA
 
 }  // namespace hs
@@ -183,6 +329,7 @@ void hotspot_preload() {
   using namespace hs;
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, hotspot_kernel_v5<kV5V, kV5NW>);
+  cudaFuncGetAttributes(&fa, hotspot_kernel_tma);
 }
 
 
@@ -224,6 +371,32 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.ry_1 = coef[2];
   a.rz_1 = coef[3];
   a.amb = coef[4];
+  const bool aligned = (reinterpret_cast<uintptr_t>(tin) & 15) == 0 && (reinterpret_cast<uintptr_t>(pw) & 15) == 0 &&
+                       ldt % 4 == 0 && ldp % 4 == 0 && wm < (1ll << 30) && wn < (1ll << 30);
+  if (aligned) {
+    CUtensorMap mT, mP;
+    int rc = leaf::encode_2d(&mT, tin, wn, wm, ldt, kPRW, kPRH, CU_TENSOR_MAP_SWIZZLE_NONE);
+    if (!rc) rc = leaf::encode_2d(&mP, pw, wn, wm, ldp, kPRW, kPRH, CU_TENSOR_MAP_SWIZZLE_NONE);
+    if (rc) return rc;
+    // TMA reads a box whose first column is 16-byte aligned: tiles start at
+    // multiples of 4 columns and advance by sx (a multiple of 4, <= 128 - 2h)
+    // output columns; tile b owns [rx0 + b sx + h, rx0 + (b + 1) sx + h).
+    const int oty = kPRH - 2 * iters, sx = (kPRW - 2 * iters) / 4 * 4;
+    const int64_t rx0 = (a.vx0 - iters) >= 0 ? (a.vx0 - iters) / 4 * 4 : -((iters - a.vx0 + 3) / 4 * 4);
+    const int64_t ty = (a.vy1 - a.vy0 + oty - 1) / oty, tx = (a.vx1 - (rx0 + iters) + sx - 1) / sx;
+    if (ty * tx >= (1ll << 31)) return fail(NU_EINVAL, "hotspot window too large");
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const int tiles = static_cast<int>(ty * tx);
+    const int grid = std::min(tiles, sms_of(dev));
+    cudaFuncSetAttribute(hotspot_kernel_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, kPSmem);
+    hotspot_kernel_tma<<<grid, kPW * 32, kPSmem, stream>>>(mT, mP, a, static_cast<int>(tx), tiles,
+                                                                   static_cast<int>(rx0), sx,
+                                                                   (reinterpret_cast<uintptr_t>(tout) & 15) == 0 && ldo % 4 == 0);
+    count_launches(1);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_tma launch");
+  }
   {
     constexpr int RH = kV5V * kV5NW, RW = 128;
     const int oty = RH - 2 * iters, otx = RW - 2 * iters;

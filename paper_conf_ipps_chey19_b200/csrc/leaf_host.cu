@@ -165,7 +165,7 @@ int64_t leaf_acc_chunk() {
   return v;
 }
 
-static int sms_of(int dev) {
+int sms_of(int dev) {
   static std::atomic<int> num_sms[kMaxDevices];
   if (num_sms[dev].load() == 0) {
     int n = 0;

@@ -24,6 +24,7 @@ constexpr int kHotspotMaxIters = 8;        // HotSpot-2D iterations per leaf lau
 
 // Kernel launches issued by the library (all devices, all threads): the
 // bench's `gpu_launches` claim (northup_debug_kernel_launches).
+int sms_of(int dev);   // SM count of a device (cached)
 void count_launches(int n);
 
 // Positional file I/O for every FILE path (tree.cpp): pread / pwrite, unless a

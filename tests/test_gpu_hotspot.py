@@ -118,26 +118,44 @@ def test_in_hbm_leaf_iters_invariance():
     assert np.array_equal(a, b) and np.array_equal(a, c)
 
 
+def _on_device(X, dev, layout):
+    """X on the device as a row-major view: "dense" (ld = cols), "padded" (ld a
+    multiple of 4 floats, base 16-B aligned: the persistent TMA kernel) or
+    "offset" (base 4 bytes past an aligned one: the v5 fallback)."""
+    R, C = X.shape
+    if layout == "dense":
+        return torch.from_numpy(np.ascontiguousarray(X)).to(dev)
+    ld = (C + 3) // 4 * 4 + 4
+    buf = torch.full((R + 1, ld + 1), float("nan"), device=dev)
+    flat = buf.view(-1)
+    off = 1 if layout == "offset" else 0
+    v = flat[off:off + R * ld].view(R, ld)[:, :C]
+    v.copy_(torch.from_numpy(np.ascontiguousarray(X)))
+    return v
+
+
+@pytest.mark.parametrize("layout", ["dense", "padded", "offset"])
 @pytest.mark.parametrize("R,C,iters", [(700, 900, 8), (129, 131, 3), (1, 257, 5), (300, 2, 7), (97, 129, 8),
-                                        (450, 333, 6), (1000, 1200, 8)])
-def test_leaf_bitwise_vs_emulation(R, C, iters):
-    """The leaf (v5: 4 columns x 12 rows per thread, shuffled W/E, shared-memory
-    N/S halo rows) evaluates RH4's sequence per cell, so it equals the exact
-    fp32 emulation bit for bit — whole grids (edge CTAs, tile-size boundaries
-    at 96 / 128 cells) and grids large enough for clamp-free interior CTAs."""
+                                        (450, 333, 6), (1000, 1200, 8), (260, 250, 1)])
+def test_leaf_bitwise_vs_emulation(R, C, iters, layout):
+    """The leaf evaluates RH4's sequence per cell, so it equals the exact fp32
+    emulation bit for bit — whole grids (edge tiles, tile-size boundaries at
+    96 / 112 / 128 cells) and grids large enough for clamp-free interior tiles,
+    through the persistent TMA kernel (aligned windows) and the v5 fallback
+    (unaligned base or leading dimension)."""
     T, P = grids(R, C, seed=R + 3 * C)
     dev = torch.device("cuda", 0)
-    t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
-    o = torch.full_like(t, float("nan"))
+    t, p = _on_device(T, dev, layout), _on_device(P, dev, layout)
+    o = _on_device(np.full((R, C), np.nan, np.float32), dev, layout)
     nu.hotspot_leaf(t, p, o, iters)
     full = emulate_fp32(T, P, iters)
     assert np.array_equal(o.cpu().numpy(), full)
     # a sub-window: only its valid region is written, equal to the full-grid evolution
     if R > 2 * iters + 2 and C > 2 * iters + 2:
         y0, y1, x0, x1 = 1, R - 1, 1, C - 1
-        tw = torch.from_numpy(np.ascontiguousarray(T[y0:y1, x0:x1])).to(dev)
-        pw = torch.from_numpy(np.ascontiguousarray(P[y0:y1, x0:x1])).to(dev)
-        ow = torch.full_like(tw, float("nan"))
+        tw = _on_device(T[y0:y1, x0:x1], dev, layout)
+        pw = _on_device(P[y0:y1, x0:x1], dev, layout)
+        ow = _on_device(np.full((y1 - y0, x1 - x0), np.nan, np.float32), dev, layout)
         nu.hotspot_leaf(tw, pw, ow, iters, gy0=y0, gx0=x0, rows=R, cols=C)
         out = ow.cpu().numpy()
         assert np.array_equal(out[iters:-iters, iters:-iters], full[y0 + iters:y1 - iters, x0 + iters:x1 - iters])
