@@ -644,10 +644,12 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                          "achieved_basis": "useful flops 2 m n k of one K-panel launch / its CUDA-event duration "
                                            "(events recorded by the library around each GEMM kernel on the torch "
                                            "stream, in-HBM operands)",
-                         "traffic_basis": "ncu --set full dram__bytes_read+write of one such launch "
-                                          "(profiles/leaf_traffic.json); algorithmic bytes per launch "
-                                          f"= split A/B panel + C write = "
-                                          f"{4 * (m + min(n, 32768)) * min(K, kc_eff) + 4 * m * min(n, 32768):.3e}"},
+                         "traffic_basis": "ncu --set full dram__bytes_read+write of one reduce-add launch "
+                                          "(profiles/leaf_traffic.json); algorithmic bytes of such a launch "
+                                          f"= split A/B panel + C read + C write = "
+                                          f"{4 * (m + min(n, 32768)) * min(K, kc_eff) + 8 * m * min(n, 32768):.3e}"
+                                          + (f" (traffic / algorithmic = {traffic / (4 * (m + min(n, 32768)) * min(K, kc_eff) + 8 * m * min(n, 32768)):.2f})"
+                                             if traffic else "")},
             "gpu_launches": launches_timed * world,
             "gpu_launches_basis": "library kernel launches (northup_debug_kernel_launches) during the timed "
                                   "out-of-core steps on this rank x ranks",

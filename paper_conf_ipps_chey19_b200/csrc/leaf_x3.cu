@@ -9,13 +9,17 @@
 //   * The leader's MMA thread issues per 16 k three kind::f16 MMAs (fp16 in,
 //     fp32 accumulate, M 256 N 256 K 16): hi.hi, hi.lo, lo.hi.
 //   * The tensor core truncates its fp32 accumulator after every MMA (probed,
-//     DESIGN.md R20), so the accumulation runs in TMEM for kAccChunk of K only;
-//     two 256-column accumulators alternate, so the epilogue drains one while
-//     the MMAs fill the other.
-//   * Epilogue (8 warps): tcgen05.ld -> scale by 2^(e_i + e_j) (exact) ->
-//     128-B-swizzled staging box -> TMA store (first chunk) or TMA reduce-add
-//     (C += chunk, an fp32 round-to-nearest add performed in L2).
-//     A C that TMA cannot address (unaligned) is written from registers.
+//     DESIGN.md R20), so the accumulation runs in TMEM for kAccChunk (256) of
+//     K only; two 256-column accumulators alternate, so the epilogue drains
+//     one while the MMAs fill the other.
+//   * Epilogue (16 warps, four per TMEM lane quarter): each thread owns one row
+//     and 64 columns of its CTA's half tile and adds every chunk into a running
+//     sum in registers (fp32 round-to-nearest, ascending K).  At the end
+//     of the panel it scales by 2^(e_i + e_j) (exact) and writes C once through
+//     a 128-B-swizzled 32 x 32 staging box (8 boxes, shared by warps w and
+//     w + 8 in turn): a TMA store, or a TMA reduce-add (C += panel, an fp32 RN
+//     add in L2) when accumulating.  A C that TMA cannot address (unaligned)
+//     is written from registers.
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>

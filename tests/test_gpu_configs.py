@@ -117,3 +117,12 @@ def test_cfg4_one_gpu_sampled():
     assert sampled_check(a, b, c, 4) <= TOL
     assert freivalds_uniform(a, b, c, 4) <= TOL
     t.destroy()
+    # integer inputs: C is exact, so Freivalds with +-1 vectors must match exactly
+    # (a single wrong element of the 2^32 would show: test_oracle pins this)
+    t, a, b, c, st = run_config(M, N, K, 8 * GiB, "int", 4)
+    rng = np.random.default_rng(4)
+    for _ in range(2):
+        r = np.where(rng.random(N) < 0.5, -1.0, 1.0)
+        _, x, y = oracle.freivalds(a, b, c, r)
+        assert np.array_equal(x, y)
+    t.destroy()
