@@ -51,6 +51,7 @@ CONFIGS = {
 HOTSPOT = dict(R=32768, C=32768, iters=256, cap=8 * GiB,
                desc="HotSpot-2D 32768^2 fp32 grid (P:349 32k inputs) x 256 iterations, pinned host -> "
                     "HBM (8 GiB cap) -> SMEM, 1 GPU (S§8(f) NEXT-3)")
+SCHEDULES = {"auto": 0, "s1": 1, "s2": 2, "queue": 3, "s2b": 4}
 HS_FLOPS_PER_UPDATE = 14                 # flops of one cell update as the formula states (5 mul + 9 add/sub)
 FP32_LANES_PER_SM, N_SMS = 128, 148      # B200: 4 SMSPs x 32 fp32 lanes; 148 SMs
 
@@ -387,7 +388,8 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     hB = th.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4)
     hC = th.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4)
     opts = nu.make_opts(k_chunk=kc)
-    ooc_opts = nu.make_opts(k_chunk=kc, shared_staging=-1 if args.no_shared_staging else 0)
+    ooc_opts = nu.make_opts(schedule=SCHEDULES[args.schedule], k_chunk=kc,
+                            shared_staging=-1 if args.no_shared_staging else 0)
     shared_peers = False
     if world > 1 and not args.no_shared_staging:
         # NEXT-1: siblings of a grid row / column share A / B panels over
@@ -414,7 +416,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
         dist.all_gather_object(oks, ok)
         shared_peers = all(oks)
         if not shared_peers:
-            ooc_opts = nu.make_opts(k_chunk=kc, shared_staging=-1)
+            ooc_opts = nu.make_opts(schedule=SCHEDULES[args.schedule], k_chunk=kc, shared_staging=-1)
     stream = torch.cuda.current_stream(dev)
 
     def barrier():
@@ -498,7 +500,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     del A2, B2, C2
     # staging evidence (untimed): one call in timing mode for per-stream busy
     # times, and the link bandwidth this GPU gets for pinned copies
-    tim = t.gemm(Ab, Bb, Cb, GM, GN, K, nu.make_opts(k_chunk=kc, collect_timing=True,
+    tim = t.gemm(Ab, Bb, Cb, GM, GN, K, nu.make_opts(schedule=ooc_opts.schedule, k_chunk=kc, collect_timing=True,
                                                      shared_staging=ooc_opts.shared_staging))
     pcie = measure_pcie(dev)
     replicate_ms = None
@@ -570,7 +572,9 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                 "tmem_acc_chunk": 256,
                 "region_per_gpu": [m, n, K],
                 "parallelism": f"C subtrees {nu.partition(world, M, N)} over {world} GPU(s)" if world > 1 else "1 GPU",
-                "schedule": {1: "S1", 2: "S2"}.get(ooc_stats.get("schedule"), "auto"),
+                "schedule": {1: "S1", 2: "S2 (drain tail)", 3: "queue", 4: "S2B (B-first)"}.get(
+                    ooc_stats.get("schedule"), "auto"),
+                "bfirst_rows": ooc_stats.get("bfirst_rows"),
                 "shared_staging": bool(ooc_stats.get("shared_staging")),
                 "shared_staging_peers": "CUDA IPC (multi-process siblings)" if shared_peers else None,
                 "blocks": [ooc_stats.get("bm"), ooc_stats.get("bn"), ooc_stats.get("bk")],
@@ -988,6 +992,8 @@ def main():
     ap.add_argument("--file-size", type=int, default=0, help="--config file: M = N = K (default 32768)")
     ap.add_argument("--file-dir", default=None, help="--config file: where the A, B, C files go")
     ap.add_argument("--k-chunk", type=int, default=2048)
+    ap.add_argument("--schedule", default="auto", choices=sorted(SCHEDULES),
+                    help="HOST -> HBM schedule (default: the planner's cost model)")
     ap.add_argument("--quick", action="store_true", help="sizes / 4 (smoke-testing the bench)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

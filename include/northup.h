@@ -67,6 +67,12 @@ extern "C" {
                             own queue and, when empty, steals from the head of another's; a tile is
                             an S2 sub-problem (C tile resident, K panels stream, tile drained).
                             HOST root, single process; no shared staging, no graphs. */
+#define NU_SCHED_S2B 4 /* S2's B-first variant: all of B stays resident in HBM (split once,
+                          in place, as its K panels land); rows [0, r1) of the C block are computed
+                          while B streams in, the other rows then run as strips over the full K while
+                          the first rows drain, so C's D2H overlaps compute instead of following it.
+                          NU_SCHED_AUTO picks it over S2 when the cost model predicts a shorter block
+                          time; NU_SCHED_S2 never uses it.  Not with NVLink-shared staging. */
 
 typedef struct northup_tree_s* northup_tree_t;
 typedef struct northup_buf_s* northup_buf_t;
@@ -196,7 +202,7 @@ int northup_release(northup_tree_t t, northup_buf_t b);
 
 /* ------------------------------------------------------- the GEMM (§IV-A) */
 typedef struct {
-  int schedule;         /* NU_SCHED_AUTO / S1 / S2 */
+  int schedule;         /* NU_SCHED_AUTO / S1 / S2 / QUEUE / S2B */
   int replicate_result; /* 1: after the join, gather C into every HBM node's replica
                            buffer (northup_tree_set_replica) — NCCL over NVLink */
   int64_t k_chunk;      /* K panel of one leaf launch and of one operand split (0 = 2048); the
@@ -244,7 +250,7 @@ typedef struct {
   int64_t tasks;         /* NU_SCHED_QUEUE: C tiles */
   int64_t tasks_stolen;  /* NU_SCHED_QUEUE: tiles a sibling took from another sibling's queue */
   int file_direct_mode;  /* FILE root with HBM children (GDS edge): 1 = cuFile, 2 = pinned bounce */
-  int reserved_stat;
+  int bfirst_rows;       /* NU_SCHED_S2B: C rows computed while B streams (r1); 0 otherwise */
 } northup_stats;
 
 /* C = A.B (no alpha/beta; C overwritten — reading R3), A (M x K), B (K x N),

@@ -22,7 +22,7 @@ HEADER = os.path.join(os.path.dirname(_HERE), "include", "northup.h")
 NU_OK, NU_EINVAL, NU_ENOMEM, NU_EIO, NU_ECUDA, NU_ENCCL, NU_ESTATE, NU_ENOTSUP = 0, -1, -2, -3, -4, -5, -6, -7
 NU_FILE, NU_HOST, NU_HBM, NU_SMEM = 0, 1, 2, 3
 NU_PROC_NONE, NU_PROC_SM100 = 0, 1
-NU_SCHED_AUTO, NU_SCHED_S1, NU_SCHED_S2, NU_SCHED_QUEUE = 0, 1, 2, 3
+NU_SCHED_AUTO, NU_SCHED_S1, NU_SCHED_S2, NU_SCHED_QUEUE, NU_SCHED_S2B = 0, 1, 2, 3, 4
 NU_OP_COPY, NU_OP_LEAF, NU_OP_ZERO, NU_OP_IO_READ, NU_OP_IO_WRITE, NU_OP_STENCIL = 0, 1, 2, 3, 4, 5
 NU_OP_SPLIT_B = 6
 STREAM_NAMES = {0: "h2d", 1: "compute", 2: "d2h", 3: "io", 4: "d2d"}
@@ -68,7 +68,7 @@ class Stats(ctypes.Structure):
                 ("shared_staging", ctypes.c_int), ("bytes_p2p", ctypes.c_uint64),
                 ("t_p2p_ms", ctypes.c_double), ("tasks", ctypes.c_int64),
                 ("tasks_stolen", ctypes.c_int64), ("file_direct_mode", ctypes.c_int),
-                ("reserved_stat", ctypes.c_int)]
+                ("bfirst_rows", ctypes.c_int)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -156,6 +156,10 @@ struct EdgeCtx {
   // the rest, and pulls the other pieces from them over NVLink.
   int a_share = 1, b_share = 1;
   double pcie = 0.0;       // B/s per GPU measured at finalize (0: kPlanPcie)
+  // S2's B-first variant: 0 = the cost model picks between it
+  // and the drain-tail schedule, -1 = never (NU_SCHED_S2, shared staging),
+  // 1 = whenever it fits (NU_SCHED_S2B).
+  int bfirst = 0;
   // Origin of the region in the root buffers' addressing: (r0, c0) for a
   // whole-problem root; (0, 0) with ldb = ldc = region width when the root
   // buffers hold only this sibling's strips (multi-process siblings).
@@ -166,6 +170,7 @@ struct EdgeCtx {
 struct S2Shape {
   int64_t bm, bn, bk, tail, sr;
   uint64_t bytes;
+  int64_t r1 = 0;   // > 0: B-first — rows [0, r1) of the block in the main phase (tail = K)
 };
 
 uint64_t s2_bytes(int64_t bm, int64_t bn, int64_t bk, int64_t K, int64_t tail, int64_t sr, int64_t kc) {
@@ -199,6 +204,38 @@ static double s2_time(int64_t bm, int64_t bn, int64_t K, int64_t tail, int a_sha
   const double tail_h = 4.0 * ea * static_cast<double>(tail) / kPlanPcie;
   const double d2h = 4.0 * bm * static_cast<double>(bn) / kPlanPcie;
   return std::max(main_c, main_h) + std::max(std::max(tail_c, tail_h), d2h);
+}
+
+// ------------------------------------------------ S2, B-first variant
+// Under S2 a C row is final only after its last K panel, so C's D2H overlaps
+// only the tail phase (the "structural bound").  The B-first
+// variant keeps ALL of B resident (split once, in place, as it lands): while
+// B's K panels stream in, rows [0, r1) of the block are computed panel by
+// panel (their A panels through kSlots slots); then the other rows run as
+// strips over the full K against the resident B, and the r1 finished rows
+// drain while those strips compute.  Arena (elements):
+//   [C rows r1 x pad(bn)] [kSlots x A slot r1 x pad(bk)] [B K x pad(bn)]
+//   [kSlots x A strip sr x pad(K)] [kSlots x C strip sr x pad(bn)]
+//   [B column exponents: one row of pad(bn) ints per K panel] [leaf scratch]
+uint64_t bfirst_bytes(int64_t r1, int64_t bn, int64_t bk, int64_t K, int64_t sr, int64_t kc) {
+  uint64_t e = static_cast<uint64_t>(r1) * pad_ld(bn) + static_cast<uint64_t>(kSlots) * r1 * pad_ld(bk) +
+               static_cast<uint64_t>(rup(K, 32)) * pad_ld(bn) +
+               static_cast<uint64_t>(kSlots) * sr * (pad_ld(K) + pad_ld(bn)) +
+               static_cast<uint64_t>(cdiv(K, kc)) * pad_ld(bn);
+  return e * 4 + leaf_scratch(std::max(r1, sr), bn, kc);
+}
+
+// Predicted block time (same rates as s2_time): phase 1 = max(compute of r1
+// rows, H2D of B + their A), phase 2 = max(compute of the other rows, H2D of
+// their A, D2H of the whole block), plus the fill before the first leaf (one
+// B panel and a quarter of an A panel).
+static double bfirst_time(int64_t bm, int64_t bn, int64_t K, int64_t r1, int64_t kc, double pcie) {
+  const double bw = pcie > 0 ? pcie : nu::kPlanPcie;
+  const double fl = 2.0 * static_cast<double>(bn) * K / kPlanFlops;   // s per C row
+  const double row_h = 4.0 * K / bw;                                   // A row, s
+  const double p1 = std::max(fl * r1, 4.0 * static_cast<double>(bn) * K / bw + row_h * r1);
+  const double p2 = std::max(std::max(fl * (bm - r1), row_h * (bm - r1)), 4.0 * bm * static_cast<double>(bn) / bw);
+  return p1 + p2 + 4.0 * (bn + r1 / 4.0) * kc / bw;
 }
 
 int choose_s2(const EdgeCtx& x, S2Shape* out) {
@@ -262,6 +299,35 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
           have = true;
         }
       }
+      if (have && x.bfirst >= 0) {
+        // compare with the B-first variant, both with their pipeline fill (the
+        // drain-tail schedule computes its first panel on a 4 x 4 sub-grid)
+        const double bw = x.pcie > 0 ? x.pcie : kPlanPcie;
+        double best_b = cand_t + 4.0 * (bm + bn) / 4.0 * bk / bw;
+        if (x.bfirst > 0) best_b = 1e300;
+        S2Shape bc{};
+        bool have_b = false;
+        // needs a pre-split B (<= kLeafMaxN columns); by the model only with at
+        // least two K panels and the caller's K panel
+        if (bn <= kLeafMaxN && bm >= 2 && (x.bfirst > 0 || (K > x.kc && x.obk <= 0))) {
+          const int64_t step = std::max<int64_t>(128, rup(cdiv(bm, 64), 128));
+          const int64_t sr2 = std::max<int64_t>(1, std::min<int64_t>(1024, rup(cdiv(bm, 32), 128)));
+          for (int64_t r1 = std::min(step, bm - 1); r1 < bm; r1 += step) {
+            const uint64_t bytes = bfirst_bytes(r1, bn, x.kc, K, sr2, x.kc);
+            if (bytes > cap) break;
+            const double t = bfirst_time(bm, bn, K, r1, x.kc, x.pcie);
+            if (t < best_b * (1.0 - 1e-9)) {
+              best_b = t;
+              bc = S2Shape{bm, bn, x.kc, K, sr2, bytes, r1};
+              have_b = true;
+            }
+          }
+        }
+        if (have_b) {
+          cand = bc;
+          cand_t = best_b;
+        }
+      }
       if (!have) continue;
       const double tot = cand_t * static_cast<double>(cdiv(m, bm) * cdiv(n, bn));
       const bool better = !found || h2d < best_h2d || (h2d == best_h2d && tot < best_t * (1.0 - 1e-9)) ||
@@ -291,11 +357,28 @@ struct S2Layout {
   int64_t offC = 0, offBT = 0;
   int64_t offEB = -1;   // B tail column exponents [panel][ldBs] (ints), when the tail is split in place
   int64_t offSA[kSlots] = {}, offSB[kSlots] = {}, offAT[kSlots] = {};
+  int64_t offCS[kSlots] = {};   // B-first: C strip slots
 };
 
 S2Layout layout_s2(Builder& B, const S2Shape& s, int hbm_node, int w, int64_t K) {
   S2Layout L;
   L.arena = B.add_buf(B_ARENA, hbm_node, w, s.bytes);
+  if (s.r1 > 0) {   // B-first (see bfirst_bytes)
+    set_scratch(B.P, w, L.arena, s.bytes, leaf_scratch(std::max(s.r1, s.sr), s.bn, B.P->kc));
+    L.ldC = L.ldBs = pad_ld(s.bn);
+    L.ldA = pad_ld(s.bk);
+    L.ldAt = pad_ld(K);
+    int64_t off = 0;
+    L.offC = off;
+    off += s.r1 * L.ldC;
+    for (int i = 0; i < kSlots; ++i, off += s.r1 * L.ldA) L.offSA[i] = off;
+    L.offBT = off;
+    off += rup(K, 32) * L.ldBs;
+    for (int i = 0; i < kSlots; ++i, off += s.sr * L.ldAt) L.offAT[i] = off;
+    for (int i = 0; i < kSlots; ++i, off += s.sr * L.ldC) L.offCS[i] = off;
+    L.offEB = off;
+    return L;
+  }
   set_scratch(B.P, w, L.arena, s.bytes, leaf_scratch(s.bm, s.bn, B.P->kc));
   L.ldC = pad_ld(s.bn);
   L.ldA = pad_ld(s.bk);
@@ -360,9 +443,12 @@ void emit_tail_leaf(Builder& B, int w, const S2Layout& L, const S2Shape& s, int 
 
 // Rows of the graded drain strips (full strips while more than two remain,
 // then halving sizes, so the last D2H is small).
+// Never more than sr rows: a strip must fit its slot.
 static int64_t next_strip(int64_t bm, int64_t r, int64_t sr) {
   const int64_t rem = bm - r;
-  return rem > 2 * sr ? sr : (rem <= 512 ? rem : rup(cdiv(rem, 2), 128));
+  if (rem > 2 * sr) return sr;
+  if (rem <= std::min<int64_t>(512, sr)) return rem;
+  return std::min(sr, rup(cdiv(rem, 2), 128));
 }
 
 void s2_stats(const S2Shape& s, northup_stats* st) {
@@ -371,10 +457,109 @@ void s2_stats(const S2Shape& s, northup_stats* st) {
   st->bk = s.bk;
   st->tail_k = s.tail;
   st->strips = 0;
-  for (int64_t r = 0; s.tail > 0 && r < s.bm; r += next_strip(s.bm, r, s.sr), ++st->strips) {
+  for (int64_t r = s.r1; s.tail > 0 && r < s.bm; r += next_strip(s.bm, r, s.sr), ++st->strips) {
   }
   st->hbm_peak_bytes = s.bytes;
-  st->schedule = NU_SCHED_S2;
+  st->schedule = s.r1 > 0 ? NU_SCHED_S2B : NU_SCHED_S2;
+  st->bfirst_rows = static_cast<int>(s.r1);
+}
+
+// One C block (rows gr.., cols gc.., bm x bn) under the B-first variant.
+static void emit_bfirst_block(const EdgeCtx& x, const S2Shape& s, const S2Layout& L, int64_t gr, int64_t gc,
+                              int64_t bm, int64_t bn, int* panel_it, int* strip_it, northup_stats* st) {
+  Builder& B = *x.B;
+  const int w = x.worker, arena = L.arena;
+  const int64_t K = x.K, kc = B.P->kc, r1 = std::min(s.r1, bm);
+  const int64_t ldC = L.ldC, ldA = L.ldA, ldBs = L.ldBs, ldAt = L.ldAt;
+  const bool presplit = bn <= kLeafMaxN;
+  // ---- phase 1: B's K panels land in the resident B and rows [0, r1) accumulate
+  const int64_t npan = cdiv(K, kc);
+  for (int64_t p = 0; p < npan; ++p, ++*panel_it) {
+    const int sl = *panel_it % kSlots;
+    const int64_t k0 = p * kc, kk = std::min(kc, K - k0);
+    const int64_t boff = L.offBT + k0 * ldBs, eoff = L.offEB + p * ldBs;
+    // Panel 0 gates the pipeline fill: it is computed on a 4 x 4 sub-grid from
+    // the raw B (each leaf splits its piece) and split in place afterwards, so
+    // the first leaf waits for a quarter of the panel instead of all of it.
+    const int64_t gb = (p == 0 && r1 >= 4096 && bn >= 4096) ? 4 : 1;
+    const int64_t sbm = rup(cdiv(r1, gb), 256), sbn = rup(cdiv(bn, gb), 256);
+    for (int64_t jj = 0; jj < bn; jj += sbn) {
+      const int64_t cn = std::min(sbn, bn - jj);
+      B.emit(make_copy(w, S_H2D, x.Bb, k0 * x.ldb + gc + jj, x.ldb, arena, boff + jj, ldBs, kk, cn),
+             {{x.Bb, k0 * x.ldb + gc + jj, x.ldb, kk, cn, false}, {arena, boff + jj, ldBs, kk, cn, true}});
+      st->bytes_h2d += static_cast<uint64_t>(kk) * cn * 4;
+      if (gb == 1 && presplit)   // the whole panel row span is loaded: split it in place
+        B.emit(make_split_b(w, arena, boff, ldBs, kk, bn, arena, eoff),
+               {{arena, boff, ldBs, rup(kk, 32), ldBs, true}, {arena, eoff, ldBs, 1, bn, true}});
+      for (int64_t ii = 0; ii < r1; ii += sbm) {
+        const int64_t rm = std::min(sbm, r1 - ii);
+        if (jj == 0) {
+          B.emit(make_copy(w, S_H2D, x.A, (gr + ii) * x.lda + k0, x.lda, arena, L.offSA[sl] + ii * ldA, ldA, rm,
+                           kk),
+                 {{x.A, (gr + ii) * x.lda + k0, x.lda, rm, kk, false},
+                  {arena, L.offSA[sl] + ii * ldA, ldA, rm, kk, true}});
+          st->bytes_h2d += static_cast<uint64_t>(rm) * kk * 4;
+        }
+        northup_op o = make_leaf(w, arena, L.offSA[sl] + ii * ldA, ldA, arena, boff + jj, ldBs, arena,
+                                 L.offC + ii * ldC + jj, ldC, rm, cn, kk, p > 0 ? 1 : 0);
+        if (gb == 1 && presplit) {
+          o = with_presplit_b(o, arena, eoff, ldBs);
+          B.emit(o, {{arena, L.offSA[sl] + ii * ldA, ldA, rm, kk, false},
+                     {arena, boff, ldBs, kk, ldBs, false},
+                     {arena, eoff, ldBs, 1, bn, false},
+                     {arena, L.offC + ii * ldC + jj, ldC, rm, cn, true}});
+        } else {
+          B.emit(o, {{arena, L.offSA[sl] + ii * ldA, ldA, rm, kk, false},
+                     {arena, boff + jj, ldBs, kk, cn, false},
+                     {arena, L.offC + ii * ldC + jj, ldC, rm, cn, true}});
+        }
+        st->leaf_launches++;
+      }
+    }
+    if (gb > 1 && presplit)   // panel 0 after its sub-grid leaves
+      B.emit(make_split_b(w, arena, boff, ldBs, kk, bn, arena, eoff),
+             {{arena, boff, ldBs, rup(kk, 32), ldBs, true}, {arena, eoff, ldBs, 1, bn, true}});
+  }
+  // ---- phase 2: the other rows as strips over the full K against the resident
+  // B, while rows [0, r1) drain (one piece before each strip's own D2H)
+  int64_t nstrips = 0;
+  for (int64_t r = r1; r < bm; r += next_strip(bm, r, s.sr)) ++nstrips;
+  const int64_t piece = nstrips > 0 ? cdiv(r1, nstrips) : r1;
+  int64_t drained = 0;
+  auto drain_piece = [&]() {
+    const int64_t rr = std::min(piece, r1 - drained);
+    if (rr <= 0) return;
+    B.emit(make_copy(w, S_D2H, arena, L.offC + drained * ldC, ldC, x.C, (gr + drained) * x.ldc + gc, x.ldc, rr, bn),
+           {{arena, L.offC + drained * ldC, ldC, rr, bn, false},
+            {x.C, (gr + drained) * x.ldc + gc, x.ldc, rr, bn, true}});
+    st->bytes_d2h += static_cast<uint64_t>(rr) * bn * 4;
+    drained += rr;
+  };
+  for (int64_t r = r1, rr = 0; r < bm; r += rr, ++*strip_it) {
+    rr = next_strip(bm, r, s.sr);
+    const int sl = *strip_it % kSlots;
+    B.emit(make_copy(w, S_H2D, x.A, (gr + r) * x.lda, x.lda, arena, L.offAT[sl], ldAt, rr, K),
+           {{x.A, (gr + r) * x.lda, x.lda, rr, K, false}, {arena, L.offAT[sl], ldAt, rr, K, true}});
+    st->bytes_h2d += static_cast<uint64_t>(rr) * K * 4;
+    northup_op o = make_leaf(w, arena, L.offAT[sl], ldAt, arena, L.offBT, ldBs, arena, L.offCS[sl], ldC, rr, bn, K, 0);
+    if (presplit) {
+      o = with_presplit_b(o, arena, L.offEB, ldBs);
+      B.emit(o, {{arena, L.offAT[sl], ldAt, rr, K, false},
+                 {arena, L.offBT, ldBs, K, ldBs, false},
+                 {arena, L.offEB, ldBs, cdiv(K, kc), bn, false},
+                 {arena, L.offCS[sl], ldC, rr, bn, true}});
+    } else {
+      B.emit(o, {{arena, L.offAT[sl], ldAt, rr, K, false},
+                 {arena, L.offBT, ldBs, K, bn, false},
+                 {arena, L.offCS[sl], ldC, rr, bn, true}});
+    }
+    st->leaf_launches++;
+    drain_piece();
+    B.emit(make_copy(w, S_D2H, arena, L.offCS[sl], ldC, x.C, (gr + r) * x.ldc + gc, x.ldc, rr, bn),
+           {{arena, L.offCS[sl], ldC, rr, bn, false}, {x.C, (gr + r) * x.ldc + gc, x.ldc, rr, bn, true}});
+    st->bytes_d2h += static_cast<uint64_t>(rr) * bn * 4;
+  }
+  while (drained < r1) drain_piece();
 }
 
 int build_s2(const EdgeCtx& x, northup_stats* st) {
@@ -398,6 +583,10 @@ int build_s2(const EdgeCtx& x, northup_stats* st) {
     for (int64_t j0 = 0; j0 < n; j0 += s.bn) {
       const int64_t bn = std::min(s.bn, n - j0);
       const int64_t gr = x.ar0 + i0, gc = x.ac0 + j0;   // root row/col of the block
+      if (s.r1 > 0) {
+        emit_bfirst_block(x, s, L, gr, gc, bm, bn, &panel_it, &strip_it, st);
+        continue;
+      }
       // ---- main phase: K panels [0, kmain)
       const int64_t npan = kmain > 0 ? cdiv(kmain, s.bk) : 0;
       const int64_t ntail_pieces = s.tail > 0 ? cdiv(s.tail, s.bk) : 0;
@@ -505,6 +694,7 @@ int build_s2_shared(Builder& B, std::vector<EdgeCtx>& xs, int Pr, int Pc, northu
   for (EdgeCtx& x : xs) {
     x.a_share = Pc;
     x.b_share = Pr;
+    x.bfirst = -1;   // the shared plan is emitted in lock step by the drain-tail builder
   }
   S2Shape s{};
   int rc = choose_s2(xs[0], &s);
@@ -1118,7 +1308,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   if (P.kc % 4) return fail(NU_EINVAL, "k_chunk must be a multiple of 4");
   P.npass = o ? o->npass : 0;   // 0 = library default (leaf_host.cu)
   const int sched = o ? o->schedule : NU_SCHED_AUTO;
-  if (sched < NU_SCHED_AUTO || sched > NU_SCHED_QUEUE) return fail(NU_EINVAL, "unknown schedule");
+  if (sched < NU_SCHED_AUTO || sched > NU_SCHED_S2B) return fail(NU_EINVAL, "unknown schedule");
   Builder B;
   B.P = &P;
   const int A = B.add_buf(B_USER_A, 0, -1, 4ull * M * K);
@@ -1264,7 +1454,8 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
     x.obn = root.bn;
     x.obk = root.bk;
     x.sched = sched;
-    int use = sched;
+    x.bfirst = sched == NU_SCHED_S2B ? 1 : sched == NU_SCHED_S2 ? -1 : 0;
+    int use = sched == NU_SCHED_S2B ? NU_SCHED_S2 : sched;
     if (use == NU_SCHED_AUTO) {
       // P:299's row-shard reuse when the caller fixed blocks smaller than the
       // region (cfg1's 64 x 64 blocks); otherwise the C-resident schedule.
@@ -1279,7 +1470,7 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
   // has a region of the same shape under S2 (opts->shared_staging < 0 disables).
   int Pr = 1, Pc = 1;
   partition_grid(G, M, N, &Pr, &Pc);
-  bool share = G > 1 && !(o && o->shared_staging < 0) && t->p2p_ok;
+  bool share = G > 1 && !(o && o->shared_staging < 0) && t->p2p_ok && sched != NU_SCHED_S2B;
   for (int w = 0; w < G && share; ++w)
     share = uses[w] == NU_SCHED_S2 && xs[w].r1 - xs[w].r0 == xs[0].r1 - xs[0].r0 &&
             xs[w].c1 - xs[w].c0 == xs[0].c1 - xs[0].c0 && xs[w].r1 > xs[w].r0 && xs[w].c1 > xs[w].c0;

@@ -139,8 +139,17 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
 
     def view(buf, off, ld, rows, cols, m=None):
         m = mem if m is None else m
+        assert off >= 0 and (rows == 0 or cols == 0 or off + (rows - 1) * ld + cols <= len(m[buf])), \
+            f"op region outside buffer {buf}"
         return np.lib.stride_tricks.as_strided(m[buf][off:], shape=(rows, cols),
                                                strides=(ld * 8, 8), writeable=True)
+
+    # The column exponents a SPLIT_B writes (one int per column, (c_buf, c_off))
+    # are modelled as a tag value; a pre-split leaf requires the tags of every
+    # K panel it reads, so anything overwriting them (or reading them before
+    # the split) poisons its result.
+    EXP_TAG = -12345.0
+    kc = plan.stats().get("bk") or 0
 
     def clobber_split(buf, off, ld, rows, cols):
         """A write destroys the split values whose hi / lo bytes it covers."""
@@ -159,12 +168,18 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["cols"], shadow)[...] = src
             view(op["dst_buf"], op["dst_off"], op["dst_ld"], op["rows"], op["dst_ld"])[...] = np.nan
             splits[op["dst_buf"]].append((op["dst_off"], op["dst_ld"], op["rows"], op["cols"]))
+            view(op["c_buf"], op["c_off"], op["cols"], 1, op["cols"])[...] = EXP_TAG
         elif op["op"] == nu.NU_OP_LEAF:
             a = view(op["a_buf"], op["a_off"], op["lda"], op["m"], op["k"])
             b = view(op["b_buf"], op["b_off"], op["ldb"], op["k"], op["n"],
                      shadow if op["src_buf"] >= 0 else None)
             c = view(op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])
             prod = a @ b
+            if op["src_buf"] >= 0 and kc > 0:
+                for p in range(-(-op["k"] // kc)):
+                    e = view(op["src_buf"], op["src_off"] + p * op["rows"], op["n"], 1, op["n"])
+                    if not (e == EXP_TAG).all():
+                        prod = prod * np.nan
             c[...] = (c + prod) if op["accumulate"] else prod
         else:
             view(op["c_buf"], op["c_off"], op["ldc"], op["m"], op["n"])[...] = 0
@@ -202,6 +217,9 @@ def _plan_case(M, N, K, G=1, cap=0, block=None, sched=nu.NU_SCHED_AUTO, kc=0):
     (400, 520, 1000, 1, 600_000, None, nu.NU_SCHED_S2, 32),       # capacity forces blocks
     (200, 300, 150, 4, 0, (64, 96, 40), nu.NU_SCHED_S1, 0),       # S1 on 4 GPUs
     (1, 1, 1, 1, 0, None, nu.NU_SCHED_AUTO, 0),
+    (700, 300, 520, 1, 0, None, nu.NU_SCHED_S2B, 64),             # B-first: B resident, strips over K
+    (1000, 600, 900, 1, 2_000_000, None, nu.NU_SCHED_S2B, 128),   # B-first under a cap: several blocks
+    (300, 200, 100, 2, 0, None, nu.NU_SCHED_S2B, 32),             # B-first on 2 siblings, ragged
 ])
 def test_plan_simulation_exact(M, N, K, G, cap, block, sched, kc):
     A = nugen.fill(M, K, 3, 1, "int")
@@ -236,10 +254,31 @@ def test_plan_bytes_closed_forms():
     t.destroy()
 
 
+def test_bfirst_plan_bytes_and_shape():
+    """NU_SCHED_S2B: every A and B byte crosses PCIe once and C comes back
+    once (the same closed form as S2); B is split in place once per K panel;
+    the r1 main-phase rows and the strips cover the block."""
+    M, N, K, kc = 4096, 2048, 8192, 512
+    t, p = _plan_case(M, N, K, sched=nu.NU_SCHED_S2B, kc=kc)
+    s = p.stats()
+    assert s["schedule"] == nu.NU_SCHED_S2B and 0 < s["bfirst_rows"] < M and s["tail_k"] == K
+    assert s["bytes_h2d"] == 4 * K * (M + N) and s["bytes_d2h"] == 4 * M * N
+    ops = p.ops()
+    assert sum(op["op"] == nu.NU_OP_SPLIT_B for op in ops) == K // kc
+    t.destroy()
+
+
 def test_cfg3_plan_shape():
-    """cfg3: 32768^3, 8 GiB HBM cap -> C resident, staggered drain, footprint <= cap."""
+    """cfg3: 32768^3, 8 GiB HBM cap -> the cost model picks S2's B-first
+    variant; the drain-tail S2 stays available as NU_SCHED_S2."""
     M = N = K = 32768
     t, p = _plan_case(M, N, K, cap=8 * GiB)
+    s = p.stats()
+    assert s["schedule"] == nu.NU_SCHED_S2B and s["bm"] == M and s["bn"] == N
+    assert 8192 <= s["bfirst_rows"] <= 24576 and s["hbm_peak_bytes"] <= 8 * GiB
+    assert s["bytes_h2d"] == 4 * K * (M + N) and s["bytes_d2h"] == 4 * M * N
+    t.destroy()
+    t, p = _plan_case(M, N, K, cap=8 * GiB, sched=nu.NU_SCHED_S2)
     s = p.stats()
     assert s["schedule"] == nu.NU_SCHED_S2 and s["bm"] == M and s["bn"] == N
     assert 0 < s["tail_k"] < K and s["tail_k"] % 1024 == 0 and s["strips"] >= 8
@@ -327,7 +366,7 @@ from hypothesis import HealthCheck, given, settings, strategies as st
 @settings(max_examples=40, deadline=None, suppress_health_check=[HealthCheck.too_slow])
 @given(M=st.integers(1, 300), N=st.integers(1, 300), K=st.integers(1, 300),
        G=st.sampled_from([1, 2, 3, 4]), cap_kib=st.sampled_from([0, 300, 800, 2000]),
-       kc=st.sampled_from([32, 64, 128]), sched=st.sampled_from([0, 1, 2]),
+       kc=st.sampled_from([32, 64, 128]), sched=st.sampled_from([0, 1, 2, 4]),
        file_root=st.booleans(), panel=st.sampled_from([0, 32, 64]), seed=st.integers(0, 3))
 def test_random_plans_replay_exactly(M, N, K, G, cap_kib, kc, sched, file_root, panel, seed):
     """Any tree shape / capacity / schedule the planner accepts yields an op

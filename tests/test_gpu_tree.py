@@ -79,6 +79,9 @@ def test_cfg1_two_level_tree_64_blocks():
     (640, 900, 1500, 2, 0, 0, 0),                            # 2 siblings, one device
     (500, 700, 333, 4, 0, nu.NU_SCHED_S1, 0),
     (2048, 2048, 12288, 1, 0, nu.NU_SCHED_S2, 1024),         # main phase + drain tail
+    (2048, 1536, 6144, 1, 0, nu.NU_SCHED_S2B, 1024),         # B-first: B resident, strips over K
+    (1000, 1200, 3000, 1, 9_000_000, nu.NU_SCHED_S2B, 512),  # B-first, capacity -> several blocks
+    (700, 520, 900, 2, 0, nu.NU_SCHED_S2B, 128),             # B-first, 2 siblings, ragged
 ])
 @pytest.mark.parametrize("kind", ["uniform", "int"])
 def test_host_root_gemm(M, N, K, G, cap, sched, kc, kind):
@@ -125,6 +128,30 @@ def test_in_hbm_tree_and_cross_tier_bitwise():
     t.destroy()
     check(C_hbm, a, b, "uniform")
     assert np.array_equal(C_hbm, C_ooc)
+
+
+def test_bfirst_bitwise_equals_drain_tail_and_in_hbm():
+    """S2's B-first variant runs the same K-panel sequence per C element as
+    the drain-tail S2 and the in-HBM tree (phase-1 rows panel by panel, strip
+    rows as one leaf call over all panels of the pre-split B), so all three
+    are bitwise equal (reading R20)."""
+    M, N, K, kc = 4096, 3072, 8192, 1024
+    C_b, a, b, st_b = run_host(M, N, K, schedule=nu.NU_SCHED_S2B, k_chunk=kc)
+    assert st_b["schedule"] == nu.NU_SCHED_S2B and 0 < st_b["bfirst_rows"] < M
+    C_s, _, _, st_s = run_host(M, N, K, schedule=nu.NU_SCHED_S2, k_chunk=kc)
+    assert st_s["schedule"] == nu.NU_SCHED_S2
+    check(C_b, a, b, "uniform")
+    assert np.array_equal(C_b, C_s)
+    dev = torch.device("cuda:0")
+    Ad, Bd = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
+    Cd = torch.full((M, N), float("nan"), device=dev)
+    t = nu.hbm_tree(0)
+    t.finalize()
+    t.gemm(t.wrap_device(0, Ad.data_ptr(), Ad.numel() * 4), t.wrap_device(0, Bd.data_ptr(), Bd.numel() * 4),
+           t.wrap_device(0, Cd.data_ptr(), Cd.numel() * 4), M, N, K, nu.make_opts(k_chunk=kc))
+    torch.cuda.synchronize()
+    assert np.array_equal(Cd.cpu().numpy(), C_b)
+    t.destroy()
 
 
 def test_in_hbm_unaligned_operands_staged():
