@@ -307,9 +307,14 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
         if (x.bfirst > 0) best_b = 1e300;
         S2Shape bc{};
         bool have_b = false;
-        // needs a pre-split B (<= kLeafMaxN columns); by the model only with at
-        // least two K panels and the caller's K panel
-        if (bn <= kLeafMaxN && bm >= 2 && (x.bfirst > 0 || (K > x.kc && x.obk <= 0))) {
+        // Needs a pre-split B (<= kLeafMaxN columns).  The model considers it
+        // only for a region that is ONE block, with at least two K panels and
+        // the caller's K panel: with several blocks the drain-tail S2 already
+        // overlaps one block's D2H-bound tail with the next block's H2D-bound
+        // main phase (measured: cfg4 on one GPU 340 vs 334 TF/s, cfg5 94 vs 81),
+        // while B-first blocks serialise on the shared resident B.
+        const bool one_block = bm >= m && bn >= n;
+        if (bn <= kLeafMaxN && bm >= 2 && (x.bfirst > 0 || (one_block && K > x.kc && x.obk <= 0))) {
           const int64_t step = std::max<int64_t>(128, rup(cdiv(bm, 64), 128));
           const int64_t sr2 = std::max<int64_t>(1, std::min<int64_t>(1024, rup(cdiv(bm, 32), 128)));
           for (int64_t r1 = std::min(step, bm - 1); r1 < bm; r1 += step) {
