@@ -156,14 +156,7 @@ uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit
   return s;
 }
 
-int64_t leaf_acc_chunk() {
-  static int64_t v = -1;
-  if (v < 0) {
-    const char* e = getenv("NORTHUP_ACC_CHUNK");
-    v = (e && atoll(e) >= 32) ? atoll(e) / 32 * 32 : kAccChunk;
-  }
-  return v;
-}
+int64_t leaf_acc_chunk() { return kAccChunk; }
 
 int sms_of(int dev) {
   static std::atomic<int> num_sms[kMaxDevices];
@@ -199,11 +192,6 @@ int leaf_run(const LeafCall& c) {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= kMaxDevices) return fail(NU_EINVAL, "device ordinal out of range");
   const int sms = sms_of(dev);
-  static int env_band = -1;
-  if (env_band < 0) {
-    const char* v = getenv("NORTHUP_RASTER_BAND");
-    env_band = (v && atoi(v) > 0) ? atoi(v) : kRasterBand;
-  }
   const int64_t pk = std::min<int64_t>(panel, (K + 31) / 32 * 32);
   const uint64_t need = leaf_scratch_bytes(M, N, pk, c.eb_presplit != nullptr);
   char* scratch = c.scratch;
@@ -247,7 +235,7 @@ int leaf_run(const LeafCall& c) {
       if (rc == 0 && ev) cudaEventRecord(c.events[*c.events_used], c.stream);
       if (rc == 0)
         rc = x3_gemm(sa, sb, c.C + n0, c.ldc, static_cast<int>(M), nn, kl, (k0 > 0 || c.accumulate) ? 1 : 0,
-                     static_cast<int>((acc + 31) / 32), npass, env_band, sms, dev, c.dbg, c.stream);
+                     static_cast<int>((acc + 31) / 32), npass, kRasterBand, sms, dev, c.dbg, c.stream);
       if (rc == 0 && ev) {
         cudaEventRecord(c.events[*c.events_used + 1], c.stream);
         *c.events_used += 2;

@@ -32,25 +32,18 @@ namespace nu {
 namespace {
 
 using PFN_wait32 = int (*)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
-using PFN_write32 = int (*)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
 PFN_wait32 g_wait = nullptr;
-PFN_write32 g_write = nullptr;
 constexpr unsigned kWaitGeq = 0x0;        // CU_STREAM_WAIT_VALUE_GEQ
-constexpr unsigned kWriteDefault = 0x0;   // CU_STREAM_WRITE_VALUE_DEFAULT (fenced)
 constexpr uint32_t kMagic = 0x4e555052;   // "NUPR"
 
 int load_mem_ops() {
-  if (g_wait && g_write) return 0;
+  if (g_wait) return 0;
   void* fw = nullptr;
-  void* fr = nullptr;
-  cudaDriverEntryPointQueryResult q1, q2;
+  cudaDriverEntryPointQueryResult q1;
   cudaError_t e1 = cudaGetDriverEntryPointByVersion("cuStreamWaitValue32", &fw, 12000, cudaEnableDefault, &q1);
-  cudaError_t e2 = cudaGetDriverEntryPointByVersion("cuStreamWriteValue32", &fr, 12000, cudaEnableDefault, &q2);
-  if (e1 != cudaSuccess || e2 != cudaSuccess || q1 != cudaDriverEntryPointSuccess ||
-      q2 != cudaDriverEntryPointSuccess || !fw || !fr)
+  if (e1 != cudaSuccess || q1 != cudaDriverEntryPointSuccess || !fw)
     return fail(NU_ECUDA, "stream memory operations (cuStreamWaitValue32) unavailable");
   g_wait = reinterpret_cast<PFN_wait32>(fw);
-  g_write = reinterpret_cast<PFN_write32>(fr);
   return 0;
 }
 
@@ -94,13 +87,8 @@ int stream_wait_flag(cudaStream_t s, const uint32_t* addr, uint32_t gen) {
 int stream_write_flag(cudaStream_t s, uint32_t* addr, uint32_t gen) {
   // the store into a sibling's flag word: a one-thread kernel with a release store
   // at system scope (valid for any peer-mapped address, including another GPU's
-  // memory over NVLink); NORTHUP_FLAG_MEMOP=1 uses cuStreamWriteValue32 instead
-  static const bool memop = getenv("NORTHUP_FLAG_MEMOP") != nullptr;
-  if (!memop) return flag_store_launch(addr, gen, s);
-  int rc = load_mem_ops();
-  if (rc) return rc;
-  int r = g_write(s, reinterpret_cast<unsigned long long>(addr), gen, kWriteDefault);
-  return r ? fail(NU_ECUDA, "cuStreamWriteValue32 failed (%d)", r) : 0;
+  // memory over NVLink, where a stream memory operation is not guaranteed to be)
+  return flag_store_launch(addr, gen, s);
 }
 
 static void close_peer(northup_tree_s* t, int w) {

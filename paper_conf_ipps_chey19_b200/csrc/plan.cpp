@@ -259,10 +259,6 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
   const int64_t tstep = std::max<int64_t>(x.kc, rup(cdiv(K, 64), x.kc));
   for (int64_t t = tstep; t < K; t += tstep) tails.push_back(t);
   tails.push_back(K);
-  if (const char* ft = getenv("NORTHUP_TAIL_K")) {   // tuning experiments: force the drain tail
-    const int64_t v = atoll(ft);
-    if (v >= 0 && v <= K) tails.assign(1, v);
-  }
   // Among the C-block shapes that fit, pick the fewest H2D bytes: every block
   // streams its A row strip and B column strip once, 4K(bm + bn) per block.
   // For each shape the drain tail minimises the predicted block time (ties:

@@ -1,5 +1,5 @@
 """Small runs of the paths changed late in round 1, for compute-sanitizer (memcheck /
-synccheck): the v3 leaf (product) on ragged shapes, a HOST -> 2 x HBM tree with shared
+synccheck): the product leaf on ragged shapes, a HOST -> 2 x HBM tree with shared
 staging (virtual siblings), the FILE -> HBM edge through the pipelined bounce, a FILE root
 with DRAM staging (two I/O threads), and the HotSpot tree with split first/last blocks."""
 import os, sys, tempfile
