@@ -103,12 +103,21 @@ __device__ __forceinline__ float4 v5_row(const float4 c, const float4 p, const f
 // __syncthreads.  The halo buffer's parity continues from `k0` so consecutive
 // iterations, also across tiles, never share a buffer.  (Waiting on the two
 // vertical neighbours' mbarriers instead of a CTA-wide barrier was measured
-// slower: the polling costs more issue slots than the barrier skew.)
+// slower twice: waiting right after publishing, and split-phase — publish the
+// run's first and last rows first, compute the interior, wait at the next
+// iteration (1507 vs 1674 GCUPS): the mbarrier polling costs more issue slots
+// than the barrier skew it removes.)
 template <int V, int NW, bool EDGE, bool NAMED = false>
 __device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const float* __restrict__ ps,
                                            float* __restrict__ hb, int lane, int warp, int rtop, int rbot,
                                            int cl, int cr, int k0 = 0) {
   constexpr int RW = 128;
+  // The persistent kernel unrolls the iteration loop by two: the new rows then
+  // alternate between two register sets instead of being moved back into the
+  // loop-carried ones (26 moves per iteration; 1584 -> 1674 GCUPS).  v5 has no
+  // registers to spare for it.
+  constexpr int kUnroll = NAMED ? 2 : 1;
+#pragma unroll kUnroll
   for (int k = 0; k < a.iters; ++k) {
     float* buf = hb + ((k0 + k) & 1) * (NW * 2 * RW);
     *reinterpret_cast<float4*>(buf + (warp * 2 + 0) * RW + 4 * lane) = v[0];        // my first row
