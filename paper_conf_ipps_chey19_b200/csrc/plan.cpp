@@ -341,6 +341,37 @@ int choose_s2(const EdgeCtx& x, S2Shape* out) {
       }
     }
   }
+  // Whole-region B-first when the drain-tail S2 needs several C blocks but
+  // all of B fits beside a few strips (tall-skinny regions such as cfg5): one
+  // pass over A with B resident, every C strip drained as soon as it is done,
+  // so H2D (A) and D2H (C) run concurrently from start to end.  The
+  // multi-block drain-tail estimate counts its blocks as pipelined (a block's
+  // tail overlaps the next block's loads) plus half a block's drain at the end.
+  if (found && x.bfirst >= 0 && best.r1 == 0 && (best.bm < m || best.bn < n) && n <= kLeafMaxN && K > x.kc &&
+      x.obk <= 0) {
+    const double bw = x.pcie > 0 ? x.pcie : kPlanPcie;
+    const double nb = static_cast<double>(cdiv(m, best.bm) * cdiv(n, best.bn));
+    const double blk_c = 2.0 * best.bm * best.bn * static_cast<double>(K) / kPlanFlops;
+    const double blk_h = 4.0 * static_cast<double>(best.bm + best.bn) * K / bw;
+    const double blk_d = 4.0 * static_cast<double>(best.bm) * best.bn / bw;
+    const double classic = nb * std::max(blk_c, std::max(blk_h, blk_d)) + blk_d / 2;
+    const int64_t sr2 = std::min<int64_t>(8192, std::max<int64_t>(128, rup(cdiv(m, 128), 128)));
+    const int64_t step = std::max<int64_t>(128, rup(cdiv(m, 64), 128));
+    double best_b = x.bfirst > 0 ? 1e300 : classic;
+    S2Shape bc{};
+    bool have_b = false;
+    for (int64_t r1 = std::min(step, m - 1); r1 < m && r1 > 0; r1 += step) {
+      const uint64_t bytes = bfirst_bytes(r1, n, x.kc, K, sr2, x.kc);
+      if (bytes > cap) break;
+      const double t = bfirst_time(m, n, K, r1, x.kc, x.pcie);
+      if (t < best_b * (1.0 - 1e-9)) {
+        best_b = t;
+        bc = S2Shape{m, n, x.kc, K, sr2, bytes, r1};
+        have_b = true;
+      }
+    }
+    if (have_b) best = bc;
+  }
   if (found) {
     *out = best;
     return 0;
