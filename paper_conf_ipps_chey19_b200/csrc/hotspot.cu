@@ -3,8 +3,8 @@
 // of the grid resident in HBM, several iterations per launch.
 //
 // The paper's leaf loads a block and its borders into (block+2)^2 local-memory
-// arrays and does one iteration.  Here a tile (128 x 128 cells, output
-// 112 x 112 at 8 iterations) is loaded once, temperature is kept in registers
+// arrays and does one iteration.  Here a tile (128 x 132 cells, output
+// 112 x 116 at 8 iterations) is loaded once, temperature is kept in registers
 // and power in shared memory, and all `iters` iterations run on chip (the valid
 // region shrinks by one cell per iteration on every side that is not a grid
 // edge), so HBM is read once and written once per `iters` iterations.  The
@@ -219,16 +219,18 @@ __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
 // ---------------------------------------------------------------------------
 // Persistent TMA leaf (the product kernel when the window's base and leading
 // dimensions are 16-byte aligned): one CTA per SM walks the tiles
-// (128 x 128, output 112 x 112 at 8 iterations) with 16 compute warps (a lane
-// owns 4 columns x 8 rows, the v5 scheme above); thread 0 also issues the
+// (128 columns x 132 rows, output 112 x 116 at 8 iterations) with 12 warps, 3
+// per SM sub-partition (a lane owns 4 columns x 11 rows, the v5 scheme above:
+// measured 1766 GCUPS against 1675 for 16 warps x 8 rows, 1709 for 12 x 10,
+// 1566 for 8 x 16 and 1493 for 10 x 12); thread 0 also issues the
 // loads.  While the warps iterate tile i, TMA brings tile i+1's
 // temperature (single buffer, freed as soon as the compute warps have copied
 // it into registers) and power (double buffer) into shared memory, so HBM
 // traffic overlaps the arithmetic instead of alternating with it.  Out-of-window
 // cells are zero-filled by TMA, as v5's predicated loads do.
-constexpr int kPW = 16, kPV = 8, kPRH = kPW * kPV, kPRW = 128;
-constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 64 KiB
-constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 32 KiB
+constexpr int kPW = 12, kPV = 11, kPRH = kPW * kPV, kPRW = 128;
+constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 66 KiB
+constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 24 KiB
 constexpr int kPSmem = 3 * kPTileBytes + kPHaloFloats * 4 + 64;   // T | P[2] | halo | barriers
 
 __device__ __forceinline__ void tma_load_tile(uint32_t dst, const CUtensorMap* map, int x, int y, uint32_t bar) {

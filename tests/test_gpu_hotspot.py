@@ -140,7 +140,7 @@ def _on_device(X, dev, layout):
 def test_leaf_bitwise_vs_emulation(R, C, iters, layout):
     """The leaf evaluates RH4's sequence per cell, so it equals the exact fp32
     emulation bit for bit — whole grids (edge tiles, tile-size boundaries at
-    96 / 112 / 128 cells) and grids large enough for clamp-free interior tiles,
+    96 / 112 / 116 / 128 / 132 cells) and grids large enough for clamp-free interior tiles,
     through the persistent TMA kernel (aligned windows) and the v5 fallback
     (unaligned base or leading dimension)."""
     T, P = grids(R, C, seed=R + 3 * C)
