@@ -129,6 +129,9 @@ int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64
                    cudaStream_t s);
 int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64_t ldd, int* eb,
                    unsigned* bmax, cudaStream_t s);
+// Both splits of a small panel in one launch (B out of place); see kSplitSmall.
+int split_ab_small_launch(const float* A, int64_t lda, int M, int Kl, float* adst, int64_t ldda, int* ea,
+                          const float* B, int64_t ldb, int N, float* bdst, int64_t lddb, int* eb, cudaStream_t s);
 int64_t split_b_max_n();
 void preload_split();
 void preload_x3();

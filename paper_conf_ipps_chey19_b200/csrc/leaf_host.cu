@@ -158,6 +158,10 @@ uint64_t leaf_scratch_bytes(int64_t m, int64_t n, int64_t panel, bool b_presplit
 
 int64_t leaf_acc_chunk() { return kAccChunk; }
 
+// Panels with at most this many elements of A and B together take the fused
+// one-launch split (split_ab_small_kernel).
+constexpr int64_t kSplitSmallElems = int64_t(1) << 21;
+
 int sms_of(int dev) {
   static std::atomic<int> num_sms[kMaxDevices];
   if (num_sms[dev].load() == 0) {
@@ -218,12 +222,20 @@ int leaf_run(const LeafCall& c) {
   int rc = 0;
   for (int64_t k0 = 0, p = 0; k0 < K && rc == 0; k0 += panel, ++p) {
     const int kl = static_cast<int>(std::min(panel, K - k0));
-    rc = split_a_launch(c.A + k0, c.lda, static_cast<int>(M), kl, Ap, Kp, ea, sms, c.stream);
+    // small panels (cfg1's 64 x 64 x 64 blocks): both splits in one launch
+    const bool small = !c.eb_presplit && N <= NB && static_cast<int64_t>(kl) * (M + N) <= kSplitSmallElems;
+    if (small)
+      rc = split_ab_small_launch(c.A + k0, c.lda, static_cast<int>(M), kl, Ap, Kp, ea, c.B + k0 * c.ldb, c.ldb,
+                                 static_cast<int>(N), Bp, ldq, eb, c.stream);
+    else
+      rc = split_a_launch(c.A + k0, c.lda, static_cast<int>(M), kl, Ap, Kp, ea, sms, c.stream);
     const SplitOperand sa{Ap, Kp, ea};
     for (int64_t n0 = 0; n0 < N && rc == 0; n0 += NB) {
       const int nn = static_cast<int>(std::min(NB, N - n0));
       SplitOperand sb{};
-      if (c.eb_presplit) {
+      if (small) {
+        sb = SplitOperand{Bp, ldq, eb};
+      } else if (c.eb_presplit) {
         // split layout: column n0's hi sits 2 n0 bytes into the row
         const char* row = reinterpret_cast<const char*>(c.B + k0 * c.ldb) + 2 * n0;
         sb = SplitOperand{reinterpret_cast<const float*>(row), c.ldb, c.eb_presplit + p * c.eb_stride + n0};

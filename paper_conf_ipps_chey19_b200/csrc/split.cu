@@ -70,11 +70,11 @@ __device__ __forceinline__ void split4(float4 x, float s, uint2& hi, uint2& lo) 
 // One warp per row of A (grid-stride).  Pass 1: row max; pass 2: each 32-k
 // group is read by the warp, then written (the same 128 bytes when in place).
 // vec: A and dst rows 16-B aligned (float4 loads, 128 k per warp step).
-__global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
-                                                      float* dst, int64_t ldd, int* ea, int vec) {
+__device__ __forceinline__ void split_a_rows(const float* A, int64_t lda, int M, int Kl, int Kp, float* dst,
+                                             int64_t ldd, int* ea, int vec, int block, int blocks) {
   const int lane = threadIdx.x & 31;
-  const int warps = (gridDim.x * blockDim.x) >> 5;
-  for (int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M; r += warps) {
+  const int warps = (blocks * blockDim.x) >> 5;
+  for (int r = (block * blockDim.x + threadIdx.x) >> 5; r < M; r += warps) {
     const float* a = A + static_cast<int64_t>(r) * lda;
     float m = 0.f;
     if (vec) {
@@ -117,6 +117,51 @@ __global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t ld
       out[2 * k0 + 32 + lane] = lo;
       __syncwarp();
     }
+  }
+}
+
+__global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
+                                                      float* dst, int64_t ldd, int* ea, int vec) {
+  split_a_rows(A, lda, M, Kl, Kp, dst, ldd, ea, vec, blockIdx.x, gridDim.x);
+}
+
+// Small panels (cfg1-like leaf calls): the A split and the whole B split
+// (column maxima, exponents, hi / lo) in ONE launch instead of five.  Blocks
+// [0, ga) split rows of A as split_a_kernel does; each further block takes 32
+// columns of B: lane = column, the 8 warps stride over the panel's rows, a
+// shared-memory max per column, then the split (out of place).
+__global__ void __launch_bounds__(256) split_ab_small_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
+                                                             float* adst, int64_t ldda, int* ea, int avec, int ga,
+                                                             const float* B, int64_t ldb, int N, float* bdst,
+                                                             int64_t lddb, int* eb) {
+  if (static_cast<int>(blockIdx.x) < ga) {
+    split_a_rows(A, lda, M, Kl, Kp, adst, ldda, ea, avec, blockIdx.x, ga);
+    return;
+  }
+  __shared__ float cmax[8][32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int n = (blockIdx.x - ga) * 32 + lane;
+  float m = 0.f;
+  if (n < N)
+    for (int k = warp; k < Kl; k += 8) m = fmaxf(m, fabsf(B[static_cast<int64_t>(k) * ldb + n]));
+  cmax[warp][lane] = m;
+  __syncthreads();
+  if (warp == 0) {
+#pragma unroll
+    for (int w = 1; w < 8; ++w) m = fmaxf(m, cmax[w][lane]);
+    cmax[0][lane] = m;
+  }
+  __syncthreads();
+  if (n >= N) return;
+  const int e = split_exponent(cmax[0][lane]);
+  if (warp == 0) eb[n] = e;
+  const float sc = pow2(-e);
+  for (int k = warp; k < Kp; k += 8) {
+    __half h, l;
+    split1(k < Kl ? B[static_cast<int64_t>(k) * ldb + n] : 0.f, sc, h, l);
+    __half* hi_row = reinterpret_cast<__half*>(bdst + static_cast<int64_t>(k) * lddb);
+    hi_row[n] = h;
+    hi_row[lddb + n] = l;
   }
 }
 
@@ -235,6 +280,20 @@ int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_b launch: %s", cudaGetErrorString(e));
 }
 
+int split_ab_small_launch(const float* A, int64_t lda, int M, int Kl, float* adst, int64_t ldda, int* ea,
+                          const float* B, int64_t ldb, int N, float* bdst, int64_t lddb, int* eb, cudaStream_t s) {
+  const int Kp = (Kl + 31) / 32 * 32;
+  const int ga = M > 0 ? (M + 7) / 8 : 0, gb = (N + 31) / 32;
+  if (ga + gb == 0) return 0;
+  const int avec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && lda % 4 == 0 &&
+                   (reinterpret_cast<uintptr_t>(adst) % 16 == 0) && ldda % 4 == 0;
+  split_ab_small_kernel<<<ga + gb, 256, 0, s>>>(A, lda, M, Kl, Kp, adst, ldda, ea, avec, ga, B, ldb, N, bdst, lddb,
+                                                  eb);
+  count_launches(1);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_ab_small launch: %s", cudaGetErrorString(e));
+}
+
 void preload_split() {
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, split_a_kernel);
@@ -242,6 +301,7 @@ void preload_split() {
   cudaFuncGetAttributes(&fa, split_b_kernel);
   cudaFuncGetAttributes(&fa, split_b_oop_kernel);
   cudaFuncGetAttributes(&fa, col_exps_kernel);
+  cudaFuncGetAttributes(&fa, split_ab_small_kernel);
 }
 
 }  // namespace leaf
