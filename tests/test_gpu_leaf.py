@@ -269,3 +269,17 @@ def test_leaf_adversarial_through_tree(kind, K):
     t.destroy()
     assert st["bytes_h2d"] >= 4 * (M * K + K * N)
     assert normwise(C, A, B) <= TOL / 2
+
+
+def test_leaf_small_panel_fused_split_matches_regular_split():
+    """Small panels (A and B together <= 2^21 elements) take the one-launch
+    fused split; the split is per row of A and per column of B, so a small
+    sub-problem reproduces the matching block of a large (regular-split)
+    product bit for bit."""
+    M, N, K = 2048, 1536, 1024
+    A = nugen.fill(M, K, 27, 1)
+    B = nugen.fill(K, N, 27, 2)
+    big = run_leaf(A, B)
+    small = run_leaf(np.ascontiguousarray(A[:64]), np.ascontiguousarray(B[:, :512]))
+    assert np.array_equal(small, big[:64, :512])
+    assert normwise(small, A[:64], B[:, :512]) <= TOL
