@@ -534,19 +534,22 @@ def simulate_local(plan: nu.Plan, A, B, M, N, K, G, rng):
     return C
 
 
-@pytest.mark.parametrize("M,N,K,G,shared", [(512, 512, 640, 2, 0), (512, 512, 640, 4, 0),
-                                             (1024, 512, 1000, 8, 0), (300, 200, 130, 3, -1),
-                                             (512, 256, 384, 4, -1)])
-def test_multiprocess_sibling_plan_uses_local_strips(M, N, K, G, shared):
+@pytest.mark.parametrize("M,N,K,G,shared,sched", [(512, 512, 640, 2, 0, 0), (512, 512, 640, 4, 0, 0),
+                                                   (1024, 512, 1000, 8, 0, 0), (300, 200, 130, 3, -1, 0),
+                                                   (512, 256, 384, 4, -1, 0), (700, 400, 520, 2, -1, 4)])
+def test_multiprocess_sibling_plan_uses_local_strips(M, N, K, G, shared, sched):
     """northup_tree_set_local: the same plan on every process, each sibling's
     root ops addressing its own strips (region-local leading dimensions);
-    replayed with per-process strips it computes A.B exactly."""
+    replayed with per-process strips it computes A.B exactly (also with S2's
+    B-first variant, which a rank may pick when shared staging is off)."""
     A = nugen.fill(M, K, 7, 1, "int")
     B = nugen.fill(K, N, 7, 2, "int")
     t, hbm = nu.host_tree(G)
     t.set_local(hbm[G - 1])
-    p = t.plan(M, N, K, nu.make_opts(k_chunk=64, shared_staging=shared))
+    p = t.plan(M, N, K, nu.make_opts(schedule=sched, k_chunk=64, shared_staging=shared))
     assert p.stats()["shared_staging"] == (1 if shared == 0 else 0)
+    if sched:
+        assert p.stats()["schedule"] == sched
     for seed in range(3):
         C = simulate_local(p, A, B, M, N, K, G, random.Random(seed))
         assert np.array_equal(C, A.astype(np.float64) @ B.astype(np.float64))
