@@ -223,8 +223,8 @@ def test_replicate_result(G):
     t.destroy()
 
 
-@pytest.mark.parametrize("G,block", [(1, (64, 64, 64)), (2, None)])
-def test_graph_capture_and_replay(G, block):
+@pytest.mark.parametrize("G,block,sched", [(1, (64, 64, 64), 0), (2, None, 0), (1, None, nu.NU_SCHED_S2B)])
+def test_graph_capture_and_replay(G, block, sched):
     """opts.graph: the first call captures each GPU's op list into a CUDA graph,
     identical later calls replay it; results are bitwise the same."""
     M, N, K = 512, 384, 640
@@ -233,7 +233,7 @@ def test_graph_capture_and_replay(G, block):
         t.set_block(0, *block)
     t.finalize()
     p = HostProblem(t, M, N, K, 8, "int")
-    o = nu.make_opts(graph=True, shared_staging=-1)   # shared staging disables graphs
+    o = nu.make_opts(graph=True, shared_staging=-1, schedule=sched, k_chunk=128 if sched else 0)
     st1 = t.gemm(p.A, p.B, p.C, M, N, K, o)
     c1 = p.c.copy()
     p.c[...] = np.nan
