@@ -21,11 +21,11 @@ def fma32(a, b, c):
     return s.astype(np.float32)
 
 
-def emulate_fp32(T, P, iters):
+def emulate_fp32(T, P, iters, k=None):
     """The update in fp32 in the kernel's fixed sequence (test-side check,
     independent of the CUDA code): a = fma(-2, t, s + n), b = fma(-2, t, e + w),
     d = fma(a, ry, p), d = fma(b, rx, d), d = fma(amb - t, rz, d), t' = fma(cap, d, t)."""
-    k = nu.hotspot_coeffs(*T.shape)
+    k = nu.hotspot_coeffs(*T.shape) if k is None else k
     f = np.float32
     cap, rx, ry, rz, amb = f(k.cap_1), f(k.rx_1), f(k.ry_1), f(k.rz_1), f(k.amb)
     t = T.astype(np.float32).copy()

@@ -41,6 +41,26 @@ def test_leaf_whole_grid(R, C, iters):
     assert np.array_equal(out, emulate_fp32(T, P, iters))
 
 
+@pytest.mark.parametrize("R,C,iters", [(130, 70, 8), (300, 516, 5)])
+def test_leaf_caller_coefficients(R, C, iters):
+    """Coefficients other than [18]'s defaults (the library specialises the
+    default set into immediates; any other set is passed as kernel arguments):
+    bitwise equal to the fp32 emulation with the same set, within RH3 of the
+    fp64 oracle."""
+    kc = nu.HotspotCoeffs(1.2, 0.11, 0.09, 1e-4, 75.0)
+    kd = {n: float(getattr(kc, n)) for n in ("cap_1", "rx_1", "ry_1", "rz_1", "amb")}
+    T, P = grids(R, C, seed=5 * R + C)
+    dev = torch.device("cuda", 0)
+    t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+    o = torch.full_like(t, float("nan"))
+    nu.hotspot_leaf(t, p, o, iters, coeffs=kc)
+    out = o.cpu().numpy()
+    assert np.array_equal(out, emulate_fp32(T, P, iters, kc))
+    assert not np.array_equal(out, emulate_fp32(T, P, iters))     # the set really differs
+    ref = hs.run(T, P, iters, kd)
+    assert np.abs(out.astype(np.float64) - ref).max() <= hs.tolerance(iters, np.abs(ref).max())
+
+
 def test_leaf_sub_window_valid_region():
     """A window inside the grid: only the valid region (shrunk by `iters` on
     non-edge sides) is written, and it equals the full-grid evolution."""
