@@ -723,6 +723,9 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     with ClockSampler(local_rank) as clk:
         t_h, per_h = timed(lambda: st_h.update(th.hotspot(hT, hP, hO, R, C, iters)), args.steps, args.warmup)
         t_o, per_o = timed(lambda: st_o.update(t.hotspot(Tb, Pb, Ob, R, C, iters)), args.steps, args.warmup)
+    # Fig. 7/8 analogue (untimed): one out-of-core call in timing mode, per-stream busy time
+    tim = t.hotspot(Tb, Pb, Ob, R, C, iters, nu.hotspot_opts(collect_timing=1))
+    torch.cuda.synchronize(dev)
     o_hbm = Od.cpu().numpy()
     bitwise = bool(np.array_equal(o_hbm, O))
     cells = float(R) * C * iters
@@ -758,7 +761,13 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     cpu_cells = sum((min(R, y + 32 + iters) - max(0, y - iters)) * (min(C, x + 32 + iters) - max(0, x - iters))
                     for y, x in samples) * iters
     tol = ohs.tolerance(iters, tmax)
-    pcie_gcups = cells / (st_o.get("bytes_h2d", 1) / 53e9) / 1e9
+    # the link rates measured in this run with both directions active (as for the GEMM lines):
+    # T and P windows cross H2D once per pass while the finished blocks drain D2H
+    pcie = measure_pcie(dev)
+    t_h2d = st_o.get("bytes_h2d", 0) / (pcie["bidir_h2d_gbs"] * 1e9)
+    t_d2h = st_o.get("bytes_d2h", 0) / (pcie["bidir_d2h_gbs"] * 1e9)
+    pcie_gcups = cells / max(t_h2d, t_d2h, 1e-12) / 1e9
+    pcie_bound = "pcie_h2d" if t_h2d >= t_d2h else "pcie_d2h"
     result = {
         "metric": "out-of-core HotSpot-2D cell updates/s (S§8(f) NEXT-3); % slowdown vs in-HBM; roofline frac",
         "value": round(value, 3), "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
@@ -775,13 +784,22 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
                 "h2d_bytes_per_step": int(st_o.get("bytes_h2d", 0)),
                 "d2h_bytes_per_step": int(st_o.get("bytes_d2h", 0)), "ms_per_step": round(ms_o, 3),
                 "leaf_launches_per_step": int(st_o.get("leaf_launches", 0)),
-                "pcie_roofline_gcups": round(pcie_gcups, 1)},
+                "pcie_roofline_gcups": round(pcie_gcups, 1), "pcie_measured": pcie},
         "slowdown_pct_vs_in_hbm": round(100.0 * (ms_o / ms_h - 1.0), 2),
-        "e2e_roofline": {"bound": "pcie_h2d" if pcie_gcups < in_hbm else "alu",
+        "e2e_roofline": {"bound": pcie_bound if pcie_gcups < in_hbm else "in_hbm",
                          "peak": round(min(pcie_gcups, in_hbm), 1), "unit": "Gcell-updates/s",
                          "frac": round(value / min(pcie_gcups, in_hbm), 4),
-                         "basis": "min(H2D bytes of the plan at 53 GB/s, the in-HBM rate): T and P windows "
-                                  "cross PCIe once per pass"},
+                         "terms": {"pcie_h2d": round(cells / max(t_h2d, 1e-12) / 1e9, 1),
+                                   "pcie_d2h": round(cells / max(t_d2h, 1e-12) / 1e9, 1),
+                                   "in_hbm": round(in_hbm, 1)},
+                         "basis": "min(plan's H2D bytes / BW_h2d, D2H bytes / BW_d2h, the in-HBM rate), BW = "
+                                  "pinned copies measured in this run with both directions active; T and P "
+                                  "windows cross PCIe once per pass"},
+        "breakdown": {k.replace("t_", "").replace("_ms", "_busy_ms"): round(tim.get(k, 0.0), 2)
+                      for k in ("t_h2d_ms", "t_compute_ms", "t_d2h_ms")} | {
+            "h2d_busy_gbs": round(tim["bytes_h2d"] / (tim["t_h2d_ms"] * 1e6), 2) if tim.get("t_h2d_ms") else None,
+            "basis": "CUDA events around every op of one untimed out-of-core call (collect_timing); busy = sum "
+                     "of op durations per stream"},
         "paper_context": {"hotspot_ooc_gap_pct": 15, "note": "APU + SSD vs DRAM (PAPER.md P:381); context only"},
         "roofline": {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "TFLOP/s",
                      "frac": round(achieved / peak, 4), "traffic": None,

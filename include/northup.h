@@ -121,8 +121,12 @@ int northup_tree_set_arena(northup_tree_t t, int node, void* dev_ptr, uint64_t b
 
 /* Register the caller-owned device buffer (M x N fp32, row-major) that
  * receives the whole C on this HBM node when northup_gemm_ex runs with
- * opts->replicate_result (S§8(e): NCCL over NVLink for distinct devices,
- * device copies for siblings aliasing one device).  NULL unregisters. */
+ * opts->replicate_result (S§8(e)).  HOST root, one process: the plan copies
+ * every finished C piece from its sibling's HBM into every replica (peer
+ * device-to-device copies over NVLink, issued as the piece drains, so they
+ * overlap the rest of the GEMM).  Other trees: after the join (NCCL over
+ * NVLink for distinct devices, device copies for siblings aliasing one
+ * device).  NULL unregisters. */
 int northup_tree_set_replica(northup_tree_t t, int node, void* dev_ptr, uint64_t bytes);
 
 /* Validate the tree (P:95 level rule: every path from the root ends in a leaf
@@ -203,8 +207,9 @@ int northup_release(northup_tree_t t, northup_buf_t b);
 /* ------------------------------------------------------- the GEMM (§IV-A) */
 typedef struct {
   int schedule;         /* NU_SCHED_AUTO / S1 / S2 / QUEUE / S2B */
-  int replicate_result; /* 1: after the join, gather C into every HBM node's replica
-                           buffer (northup_tree_set_replica) — NCCL over NVLink */
+  int replicate_result; /* 1: every HBM node's replica buffer (northup_tree_set_replica)
+                           receives the whole C: pushed piece by piece during the call
+                           (HOST root, one process) or gathered after the join */
   int64_t k_chunk;      /* K panel of one leaf launch and of one operand split (0 = 2048); the
                            TMEM accumulation inside a panel is 256 (R20) */
   int npass;            /* leaf split (R22): 0 = default (3); 3 = fp16 hi.hi + hi.lo +
@@ -310,7 +315,8 @@ typedef struct {
 } northup_op;
 
 typedef struct {
-  int kind;       /* 0 = user A, 1 = user B, 2 = user C, 3 = node arena */
+  int kind;       /* 0 = user A, 1 = user B, 2 = user C, 3 = node arena, 4 = DRAM staging,
+                     5 = a sibling's replica of C (replicate_result pushes) */
   int node;       /* tree node the buffer lives at */
   int worker;     /* owning worker for arenas, -1 for user buffers */
   uint64_t bytes; /* size (arena: planned footprint) */

@@ -103,7 +103,8 @@ int northup_gemm_ex(northup_tree_t t, northup_buf_t A, northup_buf_t B, northup_
       rc = execute_queue(t, M, N, K, A, B, C, o, st);   // tiles popped at run time
     else
       rc = execute_plan(t, plan, A, B, C, o, st);
-    if (!rc && o && o->replicate_result) rc = gather_replicas(t, plan, C, st);
+    // replicas: pushed by the plan's own copies, else gathered after the join
+    if (!rc && o && o->replicate_result && !plan.replica_push) rc = gather_replicas(t, plan, C, st);
     cudaSetDevice(prev);
   }
   t->busy = false;

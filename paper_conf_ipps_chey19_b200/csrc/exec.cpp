@@ -887,6 +887,11 @@ int execute_plan(northup_tree_s* t, const Plan& P, northup_buf_s* a, northup_buf
       if (ub->storage == NU_FILE) ctx.file[i] = ub;
       continue;
     }
+    if (pb.kind == B_REPLICA) {   // a sibling's replica of C (peer memory; same process)
+      ctx.base[i] = static_cast<char*>(t->nodes[pb.node].replica);
+      if (!ctx.base[i]) return fail(NU_ESTATE, "replica of node %d was unregistered", pb.node);
+      continue;
+    }
     if (lw >= 0 && pb.worker != lw) {   // a sibling's arena (IPC-mapped, pulls only)
       ctx.base[i] = pb.worker >= 0 && pb.worker < static_cast<int>(t->peers.size())
                         ? t->peers[pb.worker].arena : nullptr;

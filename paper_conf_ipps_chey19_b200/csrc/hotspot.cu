@@ -26,6 +26,9 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <map>
+#include <mutex>
+#include <utility>
 
 #include "leaf_common.cuh"
 #include "northup_internal.h"
@@ -229,9 +232,22 @@ __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
 // traffic overlaps the arithmetic instead of alternating with it.  Out-of-window
 // cells are zero-filled by TMA, as v5's predicated loads do.
 constexpr int kPW = 12, kPV = 11, kPRH = kPW * kPV, kPRW = 128;
+
+// Tile t -> (tile row, tile column), row-major.  CTAs CLAIM tiles in this
+// order from a counter (atomicAdd) instead of taking a static t = c, c + grid,
+// ...: with a static walk, a tile row of grid / 2 tiles (or any width that
+// makes grid ~ a multiple of it) hands one tile column to the same few CTAs,
+// and a column of slower clamped tiles at the grid's west or east edge then
+// stretches the whole launch (measured on the out-of-core plan's edge windows:
+// 0.33 -> 0.52 ms per launch once a window shrinks to 74 tile columns, and a
+// row skew only moved the resonance to 75 columns).
+__device__ __forceinline__ void tile_of(int t, int tiles_x, int& by, int& bx) {
+  by = t / tiles_x;
+  bx = t - by * tiles_x;
+}
 constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 66 KiB
 constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 24 KiB
-constexpr int kPSmem = 3 * kPTileBytes + kPHaloFloats * 4 + 64;   // T | P[2] | halo | barriers
+constexpr int kPSmem = 3 * kPTileBytes + kPHaloFloats * 4 + 64;   // T | P[2] | halo | barriers, tile ids
 
 __device__ __forceinline__ void tma_load_tile(uint32_t dst, const CUtensorMap* map, int x, int y, uint32_t bar) {
   asm volatile(
@@ -243,7 +259,7 @@ __device__ __forceinline__ void tma_load_tile(uint32_t dst, const CUtensorMap* m
 
 __global__ void __launch_bounds__(kPW * 32, 1)
     hotspot_kernel_tma(const __grid_constant__ CUtensorMap mT, const __grid_constant__ CUtensorMap mP, Args a,
-                       int tiles_x, int tiles, int rx0, int sx, bool vec_out) {
+                       int tiles_x, int tiles, int rx0, int sx, bool vec_out, unsigned* ctr) {
   using namespace nu::leaf;
   extern __shared__ __align__(128) float smp[];
   float* tb = smp;                                   // temperature of the next tile
@@ -251,12 +267,14 @@ __global__ void __launch_bounds__(kPW * 32, 1)
   float* hb = smp + 3 * kPRH * kPRW;                 // halo rows
   uint64_t* bars = reinterpret_cast<uint64_t*>(hb + kPHaloFloats);
   const uint32_t full0 = smem_u32(bars), pempty0 = smem_u32(bars + 2), tempty = smem_u32(bars + 4);
+  volatile int* tile_id = reinterpret_cast<volatile int*>(bars + 6);   // [j % 2]: tile of load j, -1 = none
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int h = a.iters, OTY = kPRH - 2 * h;
   // Thread 0 is also the producer: it issues tile j's two TMA loads (T into
   // the single T buffer, P into P buffer j % 2), both completing on full[j % 2].
   auto issue = [&](int j, int t) {
-    const int by = t / tiles_x, bx = t - by * tiles_x;
+    int by, bx;
+    tile_of(t, tiles_x, by, bx);
     const int ry = static_cast<int>(a.vy0) + by * OTY - h, rx = rx0 + bx * sx;
     const uint32_t fb = full0 + 8 * (j & 1);
     mbar_arrive_expect_tx(fb, 2 * kPTileBytes);
@@ -272,25 +290,37 @@ __global__ void __launch_bounds__(kPW * 32, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     prefetch_tmap(&mT);
     prefetch_tmap(&mP);
-    if (static_cast<int>(blockIdx.x) < tiles) issue(0, blockIdx.x);
+    const int t0 = static_cast<int>(atomicAdd(ctr, 1u));
+    tile_id[0] = t0 < tiles ? t0 : -1;
+    if (t0 < tiles) issue(0, t0);
+    else mbar_arrive(full0);                     // nothing to load: release the consumers
   }
   __syncthreads();
   const int r0 = warp * kPV, x0 = 4 * lane;
-  int i = 0;
-  for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
-    const int by = t / tiles_x, bx = t - by * tiles_x;
+  for (int i = 0;; ++i) {
+    mbar_wait(full0 + 8 * (i & 1), (i >> 1) & 1);
+    const int t = tile_id[i & 1];
+    if (t < 0) break;
+    int by, bx;
+    tile_of(t, tiles_x, by, bx);
     const int64_t oy0 = a.vy0 + static_cast<int64_t>(by) * OTY;
     const int64_t ry = oy0 - h, rx = rx0 + static_cast<int64_t>(bx) * sx;
-    mbar_wait(full0 + 8 * (i & 1), (i >> 1) & 1);
     float4 v[kPV];
 #pragma unroll
     for (int r = 0; r < kPV; ++r) v[r] = *reinterpret_cast<const float4*>(tb + (r0 + r) * kPRW + x0);
     __syncwarp();
     if (lane == 0) mbar_arrive(tempty);
-    if (threadIdx.x == 0 && t + static_cast<int>(gridDim.x) < tiles) {
-      mbar_wait(tempty, i & 1);                                        // every warp holds tile i's T
-      if (i >= 1) mbar_wait(pempty0 + 8 * ((i + 1) & 1), ((i - 1) >> 1) & 1);   // tile i-1 done with its P
-      issue(i + 1, t + gridDim.x);
+    if (threadIdx.x == 0) {
+      const int tn = static_cast<int>(atomicAdd(ctr, 1u));
+      if (tn < tiles) {
+        mbar_wait(tempty, i & 1);                                      // every warp holds tile i's T
+        if (i >= 1) mbar_wait(pempty0 + 8 * ((i + 1) & 1), ((i - 1) >> 1) & 1);   // tile i-1 done with its P
+        tile_id[(i + 1) & 1] = tn;
+        issue(i + 1, tn);
+      } else {
+        tile_id[(i + 1) & 1] = -1;
+        mbar_arrive(full0 + 8 * ((i + 1) & 1));
+      }
     }
     __syncwarp();
     const float* ps = pb + (i & 1) * kPRH * kPRW;
@@ -328,9 +358,38 @@ __global__ void __launch_bounds__(kPW * 32, 1)
       }
     }
   }
+  // Every CTA made exactly one failing claim before leaving; the last one out
+  // re-arms the counter for the next launch on this stream.
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(ctr + 1, 1u) == gridDim.x - 1) {
+      ctr[0] = 0;
+      ctr[1] = 0;
+    }
+  }
 }
 
 constexpr int kV5V = 12, kV5NW = 8;   // V rows per thread (registers), NW warps per CTA
+
+// Tile counters of the persistent kernel, one pair per (device, stream): a
+// launch claims tiles from its stream's counter and its last CTA resets it, so
+// launches on one stream (which never overlap) can share it, and launches on
+// different streams (virtual siblings on one device run concurrently) never do.
+static unsigned* tile_counter(int dev, cudaStream_t s) {
+  static std::mutex m;
+  static std::map<std::pair<int, cudaStream_t>, unsigned*> ctrs;
+  std::lock_guard<std::mutex> g(m);
+  auto it = ctrs.find({dev, s});
+  if (it != ctrs.end()) return it->second;
+  unsigned* p = nullptr;
+  if (cudaMalloc(&p, 2 * sizeof(unsigned)) != cudaSuccess) return nullptr;
+  if (cudaMemset(p, 0, 2 * sizeof(unsigned)) != cudaSuccess) {
+    cudaFree(p);
+    return nullptr;
+  }
+  ctrs[{dev, s}] = p;
+  return p;
+}
 
 }  // namespace hs
 
@@ -400,10 +459,12 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
     cudaGetDevice(&dev);
     const int tiles = static_cast<int>(ty * tx);
     const int grid = std::min(tiles, sms_of(dev));
+    unsigned* ctr = tile_counter(dev, stream);
+    if (!ctr) return fail(NU_ECUDA, "hotspot: tile counter allocation failed");
     cudaFuncSetAttribute(hotspot_kernel_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, kPSmem);
     hotspot_kernel_tma<<<grid, kPW * 32, kPSmem, stream>>>(mT, mP, a, static_cast<int>(tx), tiles,
                                                                    static_cast<int>(rx0), sx,
-                                                                   (reinterpret_cast<uintptr_t>(tout) & 15) == 0 && ldo % 4 == 0);
+                                                                   (reinterpret_cast<uintptr_t>(tout) & 15) == 0 && ldo % 4 == 0, ctr);
     count_launches(1);
     cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? 0 : cuda_fail(e, "hotspot_kernel_tma launch");

@@ -122,7 +122,9 @@ namespace nu {
 // file-read and file-write queues of the I/O pseudo-worker (one host thread each)
 enum Stream { S_H2D = 0, S_COMP = 1, S_D2H = 2, S_IO = 3, S_D2D = 4, S_NUM = 5, S_IOW = 5, S_KEYS = 6 };
 inline bool is_io_stream(int s) { return s == S_IO || s == S_IOW; }
-enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3, B_DRAM = 4 };
+// B_REPLICA: the caller's M x N replica of C at an HBM node (replicate_result, pushed
+// region by region as the drains run: see Builder::push_replicas)
+enum BufKind { B_USER_A = 0, B_USER_B = 1, B_USER_C = 2, B_ARENA = 3, B_DRAM = 4, B_REPLICA = 5 };
 
 struct PlanBuf {
   int kind = B_ARENA;
@@ -142,6 +144,7 @@ struct Plan {
   int npass = 3;
   bool root_is_device = false;
   bool file_root = false;
+  bool replica_push = false;          // replicate_result is carried by the plan's own copies
   // Leaf scratch per worker (split operands of one K panel, leaf_scratch_bytes):
   // the last `scr_bytes` of arena buffer `scr_buf`, at byte offset `scr_off`.
   std::vector<int> scr_buf;

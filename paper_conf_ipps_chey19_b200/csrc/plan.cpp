@@ -1455,6 +1455,18 @@ static int build_plan_impl(const northup_tree_s* t, int64_t M, int64_t N, int64_
       if (op.op == NU_OP_COPY) st.copies++;
     return B.overflow ? fail(NU_ENOTSUP, "dependency fan-in above 16") : 0;
   }
+  if (o && o->replicate_result && t->local_node < 0) {
+    // replicate_result in one process: the plan pushes each drained C piece to
+    // every sibling's replica (Builder::push_replicas)
+    for (int w = 0; w < G; ++w) {
+      const Node& n = t->nodes[hbm[w]];
+      if (!n.replica || n.replica_bytes < 4ull * M * N)
+        return fail(NU_EINVAL, "replicate_result: HBM node %d has no M x N replica buffer "
+                               "(northup_tree_set_replica)", n.id);
+    }
+    for (int w = 0; w < G; ++w) B.replica.push_back(B.add_buf(B_REPLICA, hbm[w], w, 4ull * M * N));
+    P.replica_push = true;
+  }
   std::vector<EdgeCtx> xs;
   std::vector<int> uses;
   for (int w = 0; w < G; ++w) {

@@ -36,6 +36,24 @@ inline bool overlaps(const Access& p, int64_t lo, int64_t hi, int64_t off, int64
   return pr < r + rows && r < pr + p.rows && pc < c + cols && c < pc + p.cols;
 }
 
+inline northup_op make_copy(int worker, int stream, int src, int64_t src_off, int64_t src_ld, int dst,
+                     int64_t dst_off, int64_t dst_ld, int64_t rows, int64_t cols) {
+  northup_op o{};
+  o.op = NU_OP_COPY;
+  o.worker = worker;
+  o.stream = stream;
+  o.src_buf = src;
+  o.dst_buf = dst;
+  o.src_off = src_off;
+  o.dst_off = dst_off;
+  o.src_ld = src_ld;
+  o.dst_ld = dst_ld;
+  o.rows = rows;
+  o.cols = cols;
+  o.a_buf = o.b_buf = o.c_buf = -1;
+  return o;
+}
+
 struct Builder {
   Plan* P;
   // GEMM: root-tier regions of different siblings are disjoint by construction,
@@ -100,27 +118,30 @@ struct Builder {
       op.deps[op.ndeps++] = kv.second;
     }
     P->ops.push_back(op);
+    if (!replica.empty() && op.op == NU_OP_COPY && P->bufs[op.dst_buf].kind == B_USER_C &&
+        P->bufs[op.src_buf].kind == B_ARENA)
+      push_replicas(op);
   }
   bool overflow = false;
+
+  // replicate_result (S§8(e)) carried by the plan: every drain of a finished C
+  // piece from a sibling's HBM to the root is followed by copies of the same
+  // HBM region into every sibling's replica (peers first, its own last) on that
+  // sibling's device-to-device stream, so the NVLink transfers overlap the
+  // compute and drains still to come instead of running after the join.
+  // replica[w] = plan buffer of sibling w's replica (M x N, ld = the root C's).
+  std::vector<int> replica;
+  void push_replicas(const northup_op& d) {
+    const int G = static_cast<int>(replica.size());
+    for (int k = 1; k <= G; ++k) {
+      const int q = (d.worker + k) % G;
+      emit(make_copy(d.worker, S_D2D, d.src_buf, d.src_off, d.src_ld, replica[q], d.dst_off, d.dst_ld, d.rows, d.cols),
+           {{d.src_buf, d.src_off, d.src_ld, d.rows, d.cols, false}, {replica[q], d.dst_off, d.dst_ld, d.rows, d.cols, true}});
+      P->stats.bytes_d2d += 4ull * d.rows * d.cols;
+    }
+  }
 };
 
-inline northup_op make_copy(int worker, int stream, int src, int64_t src_off, int64_t src_ld, int dst,
-                     int64_t dst_off, int64_t dst_ld, int64_t rows, int64_t cols) {
-  northup_op o{};
-  o.op = NU_OP_COPY;
-  o.worker = worker;
-  o.stream = stream;
-  o.src_buf = src;
-  o.dst_buf = dst;
-  o.src_off = src_off;
-  o.dst_off = dst_off;
-  o.src_ld = src_ld;
-  o.dst_ld = dst_ld;
-  o.rows = rows;
-  o.cols = cols;
-  o.a_buf = o.b_buf = o.c_buf = -1;
-  return o;
-}
 
 
 }  // namespace nu

@@ -111,7 +111,7 @@ def kpanels(A, P):
     return np.concatenate([A[:, k0:k0 + P].ravel() for k0 in range(0, K, P)]) if K else A.ravel()
 
 
-def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
+def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None, replicas=None):
     """Replay the plan's ops on host arrays (float64, exact on integers).
     With `rng`, ops run in a random order consistent with the dependencies
     and with in-order execution per (worker, stream)."""
@@ -199,6 +199,8 @@ def simulate(plan: nu.Plan, A, B, M, N, K, rng=None, a_layout=None):
             i = q.pop(0)
             run(ops[i])
             done.add(i)
+    if replicas is not None:
+        replicas.extend(mem[i].reshape(M, N) for i, b in enumerate(bufs) if b["kind"] == 5)
     return mem[[b["kind"] for b in bufs].index(2)].reshape(M, N)
 
 
@@ -620,4 +622,46 @@ def test_file_direct_plan_simulation(M, N, K, G, cap, panel):
     assert p.stats()["bytes_file_write"] == 4 * M * N
     if cap:
         assert all(b["bytes"] <= cap for b in p.bufs() if b["kind"] == 3)
+    t.destroy()
+
+
+@pytest.mark.parametrize("M,N,K,G,cap,block,sched,kc", [
+    (300, 200, 130, 1, 0, None, nu.NU_SCHED_AUTO, 0),             # S2, one sibling
+    (513, 300, 777, 2, 0, None, nu.NU_SCHED_S2, 64),              # S2 with shared staging
+    (400, 520, 1000, 2, 600_000, None, nu.NU_SCHED_S2, 32),       # several C blocks per sibling
+    (200, 300, 150, 4, 0, (64, 96, 40), nu.NU_SCHED_S1, 0),       # S1 blocks on 4 siblings
+    (700, 300, 520, 2, 0, None, nu.NU_SCHED_S2B, 64),             # B-first strips
+])
+def test_replicate_result_plan_pushes_every_piece(M, N, K, G, cap, block, sched, kc):
+    """replicate_result in one process: after each drain of a finished C piece
+    the plan copies the same HBM region into every sibling's replica (S§8(e)),
+    on the sibling's device-to-device stream.  Replayed in random dependency-
+    respecting orders, every replica equals C exactly (integer inputs), and a
+    replica push never waits on the D2H drain it shadows."""
+    A = nugen.fill(M, K, 4, 1, "int")
+    B = nugen.fill(K, N, 4, 2, "int")
+    ref = A.astype(np.float64) @ B.astype(np.float64)
+    t, hbm = nu.host_tree(G, cap)
+    if block:
+        t.set_block(0, *block)
+    for h in hbm:
+        t.set_replica(h, 0x1000, 4 * M * N)   # plan-time check only: never dereferenced here
+    p = t.plan(M, N, K, nu.make_opts(schedule=sched, k_chunk=kc, replicate_result=True))
+    bufs, ops = p.bufs(), p.ops()
+    rep = [i for i, b in enumerate(bufs) if b["kind"] == 5]
+    assert [bufs[i]["worker"] for i in rep] == list(range(G))
+    drains = [o for o in ops if o["op"] == nu.NU_OP_COPY and bufs[o["dst_buf"]]["kind"] == 2]
+    pushes = [o for o in ops if o["op"] == nu.NU_OP_COPY and o["dst_buf"] in rep]
+    assert len(pushes) == G * len(drains) > 0
+    assert {o["stream"] for o in pushes} == {4}                    # S_D2D
+    assert p.stats()["bytes_d2d"] >= G * 4 * M * N
+    for seed in range(3):
+        reps = []
+        C = simulate(p, A, B, M, N, K, rng=random.Random(seed), replicas=reps)
+        assert np.array_equal(C, ref)
+        assert len(reps) == G and all(np.array_equal(r, ref) for r in reps), f"seed {seed}"
+    # without a registered replica the plan refuses replicate_result
+    t.set_replica(hbm[-1], 0, 0)
+    with pytest.raises(nu.NorthupError):
+        t.plan(M, N, K, nu.make_opts(schedule=sched, k_chunk=kc, replicate_result=True))
     t.destroy()

@@ -204,22 +204,50 @@ def test_hbm_capacity_enforced():
     t.destroy()
 
 
-@pytest.mark.parametrize("G", [1, 2, 4])
-def test_replicate_result(G):
+@pytest.mark.parametrize("G,sched,block", [(1, nu.NU_SCHED_AUTO, None), (2, nu.NU_SCHED_AUTO, None),
+                                            (4, nu.NU_SCHED_AUTO, None), (2, nu.NU_SCHED_S1, (64, 96, 128)),
+                                            (2, nu.NU_SCHED_S2B, None), (1, nu.NU_SCHED_S2B, None)])
+def test_replicate_result(G, sched, block):
     """S§8(e) replicate_result: every sibling's HBM replica holds the whole C
-    (G = 1; G > 1 as virtual siblings on one device -> device-copy gather)."""
+    (G = 1; G > 1 as virtual siblings on one device).  The plan pushes each
+    drained C piece into every replica on the device-to-device stream while
+    the rest of the GEMM runs (no gather after the join)."""
     M, N, K = 700, 520, 900
     t, hbm = nu.host_tree(G, devices=[0] * G)
+    if block:
+        t.set_block(0, *block)
     t.finalize()
     p = HostProblem(t, M, N, K, 3, "int")
     reps = [torch.full((M, N), float("nan"), device="cuda:0") for _ in range(G)]
     for h, r in zip(hbm, reps):
         t.set_replica(h, r.data_ptr(), r.numel() * 4)
-    st = t.gemm(p.A, p.B, p.C, M, N, K, nu.make_opts(replicate_result=True))
+    st = t.gemm(p.A, p.B, p.C, M, N, K, nu.make_opts(schedule=sched, replicate_result=True))
     ref = oracle.gemm(p.a, p.b)
     assert np.array_equal(p.c.astype(np.float64), ref)
     for r in reps:
         assert np.array_equal(r.cpu().numpy().astype(np.float64), ref)
+    assert st["bytes_d2d"] >= G * 4 * M * N        # the plan's pushes carried every replica
+    t.destroy()
+
+
+def test_replicate_result_in_hbm_root_gathers():
+    """A single-node HBM tree has no drains to piggy-back on: replicate_result
+    copies the finished C into the replica after the join."""
+    M, N, K = 300, 260, 200
+    a = nugen.fill(M, K, 5, 1, "int")
+    b = nugen.fill(K, N, 5, 2, "int")
+    t = nu.hbm_tree(0)
+    t.finalize()
+    dev = torch.device("cuda", 0)
+    A, B = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
+    C = torch.full((M, N), float("nan"), device=dev)
+    rep = torch.full((M, N), float("nan"), device=dev)
+    t.set_replica(0, rep.data_ptr(), rep.numel() * 4)
+    bA, bB, bC = (t.wrap_device(0, x.data_ptr(), x.numel() * 4) for x in (A, B, C))
+    t.gemm(bA, bB, bC, M, N, K, nu.make_opts(replicate_result=True))
+    ref = oracle.gemm(a, b)
+    assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+    assert np.array_equal(rep.cpu().numpy().astype(np.float64), ref)
     t.destroy()
 
 
