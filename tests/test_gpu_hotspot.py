@@ -179,3 +179,31 @@ def test_leaf_bitwise_vs_emulation(R, C, iters, layout):
         nu.hotspot_leaf(tw, pw, ow, iters, gy0=y0, gx0=x0, rows=R, cols=C)
         out = ow.cpu().numpy()
         assert np.array_equal(out[iters:-iters, iters:-iters], full[y0 + iters:y1 - iters, x0 + iters:x1 - iters])
+
+
+def test_leaf_concurrent_streams_and_tile_counts():
+    """The persistent leaf claims tiles from a per-(device, stream) counter that
+    its last CTA re-arms: launches on several streams at once, back-to-back
+    launches on one stream, and windows whose tile-column count equals half the
+    grid of CTAs (the shape that once concentrated a clamped edge column on two
+    CTAs) all give the emulation's result bit for bit."""
+    dev = torch.device("cuda", 0)
+    n_sm = torch.cuda.get_device_properties(dev).multi_processor_count
+    iters = 8
+    # tile columns = ceil((wn - iters) / 112) for a window at the grid's west edge
+    shapes = [(300, 112 * (n_sm // 2) + iters - 4), (260, 112 * (n_sm // 2) + 20), (390, 1000), (129, 517)]
+    cases = []
+    for i, (R, C) in enumerate(shapes):
+        T, P = grids(R, C, seed=40 + i)
+        t, p = torch.from_numpy(T).to(dev), torch.from_numpy(P).to(dev)
+        cases.append((T, P, t, p, [torch.full_like(t, float("nan")) for _ in range(2)]))
+    streams = [torch.cuda.Stream(dev) for _ in cases]
+    torch.cuda.synchronize(dev)
+    for rep in range(3):                       # counters must be re-armed after every launch
+        for (T, P, t, p, outs), s in zip(cases, streams):
+            with torch.cuda.stream(s):
+                nu.hotspot_leaf(t, p, outs[0], iters, stream=s)
+                nu.hotspot_leaf(outs[0], p, outs[1], iters, stream=s)
+    torch.cuda.synchronize(dev)
+    for T, P, t, p, outs in cases:
+        assert np.array_equal(outs[1].cpu().numpy(), emulate_fp32(T, P, 2 * iters))
