@@ -35,3 +35,38 @@ res = {"total_ms": st["t_total_ms"], "timeline_end_ms": float(end),
        "d2h_GBps": st["bytes_d2h"] / max(1e-9, (d2h[:, 4] - d2h[:, 3]).sum()) / 1e6,
        "launches": int(len(comp))}
 print(json.dumps(res, indent=1, default=float))
+
+# Coarse utilisation profile: per 10 ms bucket, busy fraction of H2D / compute / D2H.
+def busy_in(rows, a, b):
+    return float(np.clip(np.minimum(b, rows[:, 4]) - np.maximum(a, rows[:, 3]), 0, None).sum()) / (b - a)
+
+prof = []
+for a in np.arange(0.0, end, 10.0):
+    b = a + 10.0
+    prof.append([round(float(a)), round(busy_in(h2d, a, b), 2), round(busy_in(comp, a, b), 2), round(busy_in(d2h, a, b), 2)])
+print("bucket_ms h2d comp d2h")
+for r in prof:
+    print(*r)
+print("first_d2h_start_ms", float(d2h[:, 3].min()) if len(d2h) else None, "last_h2d_end_ms", float(h2d[:, 4].max()))
+
+# leaf ops: TF/s per op (2 m n k / duration), early ops vs strips
+lr = []
+for row in comp:
+    op = ops[int(row[0])]
+    if op["op"] == nu.NU_OP_LEAF:
+        d = float(row[4] - row[3])
+        lr.append((float(row[3]), op["m"], op["n"], op["k"], d, 2.0 * op["m"] * op["n"] * op["k"] / d / 1e9))
+lr = np.array(lr)
+if len(lr):
+    for lab, sel in (("m>=8192", lr[:, 1] >= 8192), ("m<8192", lr[:, 1] < 8192)):
+        if sel.any():
+            x = lr[sel]
+            print(lab, "ops", int(sel.sum()), "busy_ms", round(float(x[:, 4].sum()), 2),
+                  "tflops_total", round(float((2 * x[:, 1] * x[:, 2] * x[:, 3]).sum() / x[:, 4].sum() / 1e9), 1),
+                  "shape", x[0, 1:4].astype(int).tolist(), "rate_min/med/max",
+                  [round(float(v), 1) for v in np.percentile(x[:, 5], [0, 50, 100])])
+if len(lr):
+    big_k = lr[lr[:, 3] >= 16384]
+    print("strip ops (k >= 16384): start_ms m n k ms TF/s")
+    for r in big_k:
+        print(round(r[0], 1), int(r[1]), int(r[2]), int(r[3]), round(r[4], 2), round(r[5], 1))
