@@ -206,7 +206,8 @@ def test_hbm_capacity_enforced():
 
 @pytest.mark.parametrize("G,sched,block", [(1, nu.NU_SCHED_AUTO, None), (2, nu.NU_SCHED_AUTO, None),
                                             (4, nu.NU_SCHED_AUTO, None), (2, nu.NU_SCHED_S1, (64, 96, 128)),
-                                            (2, nu.NU_SCHED_S2B, None), (1, nu.NU_SCHED_S2B, None)])
+                                            (2, nu.NU_SCHED_S2B, None), (1, nu.NU_SCHED_S2B, None),
+                                            (2, nu.NU_SCHED_QUEUE, None)])
 def test_replicate_result(G, sched, block):
     """S§8(e) replicate_result: every sibling's HBM replica holds the whole C
     (G = 1; G > 1 as virtual siblings on one device).  The plan pushes each
@@ -226,7 +227,31 @@ def test_replicate_result(G, sched, block):
     assert np.array_equal(p.c.astype(np.float64), ref)
     for r in reps:
         assert np.array_equal(r.cpu().numpy().astype(np.float64), ref)
-    assert st["bytes_d2d"] >= G * 4 * M * N        # the plan's pushes carried every replica
+    if sched != nu.NU_SCHED_QUEUE:                 # the queue schedule gathers after the join
+        assert st["bytes_d2d"] >= G * 4 * M * N    # the plan's pushes carried every replica
+    t.destroy()
+
+
+def test_replicate_result_graph_replay():
+    """opts.graph with replicate_result: the captured op lists include the
+    replica pushes, so a replayed call refreshes every replica."""
+    M, N, K, G = 640, 384, 512, 2
+    t, hbm = nu.host_tree(G, devices=[0] * G)
+    t.finalize()
+    p = HostProblem(t, M, N, K, 9, "int")
+    reps = [torch.full((M, N), float("nan"), device="cuda:0") for _ in range(G)]
+    for h, r in zip(hbm, reps):
+        t.set_replica(h, r.data_ptr(), r.numel() * 4)
+    o = nu.make_opts(replicate_result=True, graph=True, shared_staging=-1)
+    ref = oracle.gemm(p.a, p.b)
+    st1 = t.gemm(p.A, p.B, p.C, M, N, K, o)
+    for r in reps:
+        r.fill_(float("nan"))
+    st2 = t.gemm(p.A, p.B, p.C, M, N, K, o)
+    assert st2["graph_replayed"] == 1
+    assert np.array_equal(p.c.astype(np.float64), ref)
+    for r in reps:
+        assert np.array_equal(r.cpu().numpy().astype(np.float64), ref)
     t.destroy()
 
 
