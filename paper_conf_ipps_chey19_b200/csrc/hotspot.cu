@@ -12,15 +12,22 @@
 // TMA while the current one iterates; hotspot_kernel_v5 (128 x 96 tiles, plain
 // loads) serves windows whose base or leading dimension is not 16-byte aligned.
 //
-// Arithmetic contract (RH4): every cell update is the fixed fp32
-// sequence (round-to-nearest, fma = one rounding)
-//     a = fma(-2, t, s + n);  b = fma(-2, t, e + w)
-//     d = fma(a, ry_1, p);  d = fma(b, rx_1, d);  d = fma(amb - t, rz_1, d)
-//     t' = fma(cap_1, d, t)
+// Arithmetic contract (RH4, revised): the update
+//     T' = T + cap_1 (P + (S + N - 2T) ry_1 + (E + W - 2T) rx_1 + (amb - T) rz_1)
+// is evaluated in the expanded form
+//     T' = kt T + kx (E + W) + ky (S + N) + q,   q = cap_1 P + cap_1 rz_1 amb
+// with kt = 1 - cap_1 (2 rx_1 + 2 ry_1 + rz_1), kx = cap_1 rx_1, ky = cap_1 ry_1
+// (rounded to fp32 once on the host from the fp32 coefficients) and q
+// computed once per cell and tile, q = fma(cap_1, P, kq).  Per cell update one
+// fixed fp32 sequence (round-to-nearest, fma = one rounding):
+//     u = fma(kt, t, q);  u = fma(kx, e + w, u);  t' = fma(ky, s + n, u)
 // written with __fadd_rn/__fmaf_rn so the compiler cannot reassociate or
-// re-fuse it: 3 FADD + 6 FFMA per update.  The result of a cell is therefore
-// independent of tiling, iterations per launch and launch order: in-HBM and
-// out-of-core runs agree bit for bit, and so does an exact fp32 emulation.
+// re-fuse it: 2 FADD + 3 FFMA per update (the first form took 3 FADD + 6
+// FFMA).  The weights kt, kx, kx, ky, ky are positive and sum to 1 - cap_1
+// rz_1, so rounding errors do not grow (RH3's bound holds).  The result of a
+// cell is independent of tiling, iterations per launch and launch order:
+// in-HBM and out-of-core runs agree bit for bit, and so does an exact fp32
+// emulation of this sequence.
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -46,17 +53,18 @@ struct Args {
   int64_t R, C;              // grid
   int64_t vy0, vy1, vx0, vx1;  // valid output region (window coordinates)
   int iters;
-  float cap_1, rx_1, ry_1, rz_1, amb;
+  float kt, kx, ky;          // expanded-form weights (see the contract above)
+  float kc, kq;              // q = fma(kc, P, kq): kc = cap_1, kq = cap_1 rz_1 amb
 };
 
-__device__ __forceinline__ float update(float t, float p, float n, float s, float e, float w,
+// q = the update's constant part of one cell (P and the ambient term)
+__device__ __forceinline__ float q_of(float p, const Args& a) { return __fmaf_rn(a.kc, p, a.kq); }
+
+__device__ __forceinline__ float update(float t, float q, float n, float s, float e, float w,
                                         const Args& a) {
-  const float ay = __fmaf_rn(-2.0f, t, __fadd_rn(s, n));
-  const float ax = __fmaf_rn(-2.0f, t, __fadd_rn(e, w));
-  float d = __fmaf_rn(ay, a.ry_1, p);
-  d = __fmaf_rn(ax, a.rx_1, d);
-  d = __fmaf_rn(__fsub_rn(a.amb, t), a.rz_1, d);
-  return __fmaf_rn(a.cap_1, d, t);
+  float u = __fmaf_rn(a.kt, t, q);
+  u = __fmaf_rn(a.kx, __fadd_rn(e, w), u);
+  return __fmaf_rn(a.ky, __fadd_rn(s, n), u);
 }
 
 // ---------------------------------------------------------------------------
@@ -164,7 +172,7 @@ template <int V, int NW>
 __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
   constexpr int RW = 128, RH = NW * V;
   extern __shared__ float sm5[];
-  float* ps = sm5;                 // power tile RH x RW
+  float* ps = sm5;                 // q = fma(cap_1, power, kq) of the tile, RH x RW
   float* hb = sm5 + RH * RW;       // 2 parities x NW warps x {first, last} row x RW
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int h = a.iters;
@@ -187,7 +195,8 @@ __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
       p[j] = in ? __ldg(a.pw + wy * a.ldp + wx) : 0.0f;
     }
     v[r] = make_float4(t[0], t[1], t[2], t[3]);
-    *reinterpret_cast<float4*>(ps + (r0 + r) * RW + x0) = make_float4(p[0], p[1], p[2], p[3]);
+    *reinterpret_cast<float4*>(ps + (r0 + r) * RW + x0) =
+        make_float4(q_of(p[0], a), q_of(p[1], a), q_of(p[2], a), q_of(p[3], a));
   }
   // (the first iteration's barrier also orders these power stores)
   const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
@@ -323,7 +332,17 @@ __global__ void __launch_bounds__(kPW * 32, 1)
       }
     }
     __syncwarp();
-    const float* ps = pb + (i & 1) * kPRH * kPRW;
+    // power -> q of this lane's own cells (the only ones it reads back), in
+    // place; the fence orders these generic writes before the TMA that will
+    // refill the buffer once every warp has released it (pempty)
+    float* ps = pb + (i & 1) * kPRH * kPRW;
+#pragma unroll
+    for (int r = 0; r < kPV; ++r) {
+      float* q = ps + (r0 + r) * kPRW + x0;
+      const float4 pv = ld_power(q);
+      *reinterpret_cast<float4*>(q) = make_float4(q_of(pv.x, a), q_of(pv.y, a), q_of(pv.z, a), q_of(pv.w, a));
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
     const bool edge = gy_top <= 0 || gy_top + kPRH >= a.R || gx_left <= 0 || gx_left + kPRW >= a.C;
     if (edge) {
@@ -436,11 +455,13 @@ int hotspot_launch(const float* tin, int64_t ldt, const float* pw, int64_t ldp, 
   a.vx0 = gx0 == 0 ? 0 : iters;
   a.vx1 = wn - (gx0 + wn == C ? 0 : iters);
   if (a.vy1 <= a.vy0 || a.vx1 <= a.vx0) return 0;
-  a.cap_1 = coef[0];
-  a.rx_1 = coef[1];
-  a.ry_1 = coef[2];
-  a.rz_1 = coef[3];
-  a.amb = coef[4];
+  // expanded-form weights, each rounded once from the fp32 coefficients (RH4)
+  const double cap = coef[0], rx = coef[1], ry = coef[2], rz = coef[3], amb = coef[4];
+  a.kt = static_cast<float>(1.0 - cap * (2.0 * rx + 2.0 * ry + rz));
+  a.kx = static_cast<float>(cap * rx);
+  a.ky = static_cast<float>(cap * ry);
+  a.kc = coef[0];
+  a.kq = static_cast<float>(cap * rz * amb);
   const bool aligned = (reinterpret_cast<uintptr_t>(tin) & 15) == 0 && (reinterpret_cast<uintptr_t>(pw) & 15) == 0 &&
                        ldt % 4 == 0 && ldp % 4 == 0 && wm < (1ll << 30) && wn < (1ll << 30);
   if (aligned) {

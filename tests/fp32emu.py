@@ -22,24 +22,24 @@ def fma32(a, b, c):
 
 
 def emulate_fp32(T, P, iters, k=None):
-    """The update in fp32 in the kernel's fixed sequence (test-side check,
-    independent of the CUDA code): a = fma(-2, t, s + n), b = fma(-2, t, e + w),
-    d = fma(a, ry, p), d = fma(b, rx, d), d = fma(amb - t, rz, d), t' = fma(cap, d, t)."""
+    """The update in fp32 in the kernel's fixed sequence (RH4, the
+    expanded form; test-side check, independent of the CUDA code):
+        kt = 1 - cap (2 rx + 2 ry + rz), kx = cap rx, ky = cap ry, kq = cap rz amb
+        (each computed in float64 from the fp32 coefficients, rounded once)
+        q = fma(cap, p, kq)                                   once per cell
+        u = fma(kt, t, q); u = fma(kx, e + w, u); t' = fma(ky, s + n, u)"""
     k = nu.hotspot_coeffs(*T.shape) if k is None else k
     f = np.float32
-    cap, rx, ry, rz, amb = f(k.cap_1), f(k.rx_1), f(k.ry_1), f(k.rz_1), f(k.amb)
-    t = T.astype(np.float32).copy()
-    p = P.astype(np.float32)
-    m2 = np.float32(-2)
+    cap, rx, ry, rz, amb = (float(f(x)) for x in (k.cap_1, k.rx_1, k.ry_1, k.rz_1, k.amb))
+    kt = np.full(T.shape, f(1.0 - cap * (2.0 * rx + 2.0 * ry + rz)), dtype=f)
+    kx = np.full(T.shape, f(cap * rx), dtype=f)
+    ky = np.full(T.shape, f(cap * ry), dtype=f)
+    q = fma32(np.full(T.shape, f(cap), dtype=f), P.astype(f), f(cap * rz * amb))
+    t = T.astype(f).copy()
     for _ in range(iters):
         g = np.pad(t, 1, mode="edge")
         n, s, e, w = g[:-2, 1:-1], g[2:, 1:-1], g[1:-1, 2:], g[1:-1, :-2]
-        ay = fma32(np.full_like(t, m2), t, s + n)
-        ax = fma32(np.full_like(t, m2), t, e + w)
-        d = fma32(ay, np.full_like(t, ry), p)
-        d = fma32(ax, np.full_like(t, rx), d)
-        d = fma32(amb - t, np.full_like(t, rz), d)
-        t = fma32(np.full_like(t, cap), d, t)
+        u = fma32(kt, t, q)
+        u = fma32(kx, e + w, u)
+        t = fma32(ky, s + n, u)
     return t
-
-

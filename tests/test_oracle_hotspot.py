@@ -127,6 +127,32 @@ def test_tolerance_model_against_fp32_emulation():
     assert err > 0   # fp32 really differs (the bound is exercised)
 
 
+def test_expanded_form_equals_definition_and_stays_within_bound():
+    """RH4 (revised): the kernel evaluates T' = kt T + kx (E + W) + ky (S + N) + q,
+    q = cap_1 P + cap_1 rz_1 amb.  In fp64 that is the definition up to
+    rounding; its fixed fp32 sequence (the test-side emulation of the kernel)
+    stays within RH3's bound of the fp64 oracle after 256 iterations, and its
+    weights are positive (a convex combination: errors do not grow)."""
+    from fp32emu import emulate_fp32
+    import paper_conf_ipps_chey19_b200 as nu
+    T, P = grids(40, 56, seed=6)
+    k = K
+    kt = 1.0 - k["cap_1"] * (2 * k["rx_1"] + 2 * k["ry_1"] + k["rz_1"])
+    kx, ky = k["cap_1"] * k["rx_1"], k["cap_1"] * k["ry_1"]
+    assert kt > 0 and kx > 0 and ky > 0
+    t = T.astype(np.float64)
+    q = k["cap_1"] * P.astype(np.float64) + k["cap_1"] * k["rz_1"] * k["amb"]
+    for _ in range(5):
+        g = np.pad(t, 1, mode="edge")
+        n, s, e, w = g[:-2, 1:-1], g[2:, 1:-1], g[1:-1, 2:], g[1:-1, :-2]
+        t = kt * t + kx * (e + w) + ky * (s + n) + q
+    assert np.abs(t - hs.run(T, P, 5, K)).max() <= 1e-10
+    out = emulate_fp32(T, P, 256, nu.hotspot_coeffs(40, 56))
+    ref = hs.run(T, P, 256, K)
+    err = np.abs(out.astype(np.float64) - ref).max()
+    assert 0 < err <= hs.tolerance(256, np.abs(ref).max())
+
+
 def test_fma32_emulation_is_exact():
     """Pin of the test-side fma (tests/fp32emu.py) against exact rational
     arithmetic, including sums that land on float32 rounding boundaries."""
