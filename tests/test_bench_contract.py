@@ -61,6 +61,21 @@ def test_ours_quick_json_line():
 
 
 @pytest.mark.gpu
+def test_hotspot_quick_json_line():
+    """--config hotspot: the NEXT-3 line with its alu roofline, the out-of-core
+    roofline from the link rates measured in the same run, and a stream breakdown."""
+    d = run_bench("--config", "hotspot", "--quick", "--steps", "2", "--warmup", "3")
+    assert d["unit"] == "Gcell-updates/s" and d["value"] > 0 and d["in_hbm"]["value"] > 0
+    assert d["roofline"]["bound"] == "alu" and 0 < d["roofline"]["frac"] < 1
+    er = d["e2e_roofline"]
+    assert er["bound"] in ("pcie_h2d", "pcie_d2h", "in_hbm") and 0 < er["frac"] < 1.2
+    assert set(er["terms"]) == {"pcie_h2d", "pcie_d2h", "in_hbm"}
+    assert d["e2e"]["pcie_measured"]["bidir_h2d_gbs"] > 1
+    assert d["breakdown"]["compute_busy_ms"] > 0 and d["breakdown"]["h2d_busy_ms"] > 0
+    assert d["parity"]["bitwise_in_hbm_vs_out_of_core"] and d["parity"]["oracle_ok"]
+
+
+@pytest.mark.gpu
 def test_ours_spawns_ranks_for_gpus_n():
     """`python bench.py --gpus 4` outside torchrun starts the 4 ranks itself
     (here 4 processes share the one GPU: --device-mod 1, gloo)."""
