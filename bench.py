@@ -768,6 +768,14 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
     t_d2h = st_o.get("bytes_d2h", 0) / (pcie["bidir_d2h_gbs"] * 1e9)
     pcie_gcups = cells / max(t_h2d, t_d2h, 1e-12) / 1e9
     pcie_bound = "pcie_h2d" if t_h2d >= t_d2h else "pcie_d2h"
+    # DRAM bytes per launch from the committed ncu capture of the same launch shape
+    hs_traffic = None
+    tp = os.path.join(ROOT, "profiles", "hotspot_traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tj = json.load(f)
+        if (tj.get("R"), tj.get("C"), tj.get("leaf_iters")) == (R, C, st_h.get("bk", 8)):
+            hs_traffic = tj.get("dram_bytes")
     result = {
         "metric": "out-of-core HotSpot-2D cell updates/s (S§8(f) NEXT-3); % slowdown vs in-HBM; roofline frac",
         "value": round(value, 3), "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
@@ -802,7 +810,7 @@ def run_hotspot(args, rank: int, world: int, local_rank: int):
                      "of op durations per stream"},
         "paper_context": {"hotspot_ooc_gap_pct": 15, "note": "APU + SSD vs DRAM (PAPER.md P:381); context only"},
         "roofline": {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "TFLOP/s",
-                     "frac": round(achieved / peak, 4), "traffic": None,
+                     "frac": round(achieved / peak, 4), "traffic": hs_traffic,
                      "peak_basis": f"dense fp32 peak: {N_SMS} SMs x {FP32_LANES_PER_SM} lanes x 2 flops (FMA) x "
                                    f"clocks.max.sm {f_max / 1e6:.0f} MHz",
                      "kernel": "nu::hs::hotspot_kernel_tma", "launch": [R, C, li],

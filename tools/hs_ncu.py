@@ -4,7 +4,7 @@ import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch, nugen
 import paper_conf_ipps_chey19_b200 as nu
-R = C = 16384
+R = C = int(os.environ.get("HS_N", "16384"))
 li = int(sys.argv[1]) if len(sys.argv) > 1 else 8
 T = torch.from_numpy(nugen.fill(R, C, 7, nugen.MAT_T, "temp")).cuda()
 P = torch.from_numpy(nugen.fill(R, C, 7, nugen.MAT_P, "power")).cuda()
