@@ -88,14 +88,14 @@ def host_view(buf, rows, cols):
     return np.ctypeslib.as_array((ctypes.c_float * (rows * cols)).from_address(buf.ptr)).reshape(rows, cols)
 
 
-def run_tree(R, C, iters, G=1, cap=0, **opt):
+def run_tree(R, C, iters, G=1, cap=0, coeffs=None, **opt):
     t, _ = nu.host_tree(G, cap, devices=[0] * G)
     t.finalize()
     Tb, Pb, Ob = t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0), t.alloc(4 * R * C, 0)
     T, P = host_view(Tb, R, C), host_view(Pb, R, C)
     T[...], P[...] = grids(R, C, seed=R + C)
     host_view(Ob, R, C)[...] = np.nan
-    st = t.hotspot(Tb, Pb, Ob, R, C, iters, nu.hotspot_opts(**opt))
+    st = t.hotspot(Tb, Pb, Ob, R, C, iters, nu.hotspot_opts(**opt), coeffs=coeffs)
     out, Tc, Pc = host_view(Ob, R, C).copy(), T.copy(), P.copy()
     assert np.array_equal(T, grids(R, C, seed=R + C)[0])      # T is not modified
     t.destroy()
@@ -129,6 +129,19 @@ def test_tree_out_of_core_matches_in_hbm_and_oracle(R, C, iters, G, cap, opt):
     assert np.array_equal(out, emulate_fp32(T, P, iters))
     check(out, T, P, iters)
     assert st["leaf_launches"] > 0 and st["bytes_h2d"] >= 8 * R * C
+
+
+def test_tree_out_of_core_caller_coefficients():
+    """Caller coefficients through the tree (the plan carries them to every
+    leaf launch): bitwise equal to the fp32 emulation with the same set and
+    within RH3 of the fp64 oracle."""
+    kc = nu.HotspotCoeffs(1.1, 0.12, 0.08, 2e-4, 70.0)
+    R, C, iters = 900, 1100, 19
+    out, T, P, st = run_tree(R, C, iters, 2, 0, coeffs=kc, block=256, halo=10, leaf_iters=5)
+    assert np.array_equal(out, emulate_fp32(T, P, iters, kc))
+    kd = {n: float(getattr(kc, n)) for n in ("cap_1", "rx_1", "ry_1", "rz_1", "amb")}
+    ref = hs.run(T, P, iters, kd)
+    assert np.abs(out.astype(np.float64) - ref).max() <= hs.tolerance(iters, np.abs(ref).max())
 
 
 def test_in_hbm_leaf_iters_invariance():
