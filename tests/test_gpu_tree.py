@@ -90,6 +90,23 @@ def test_host_root_gemm(M, N, K, G, cap, sched, kc, kind):
     assert st["num_gpus"] == G
 
 
+@pytest.mark.parametrize("M,N,K,G,cap,sched,kc,block", [
+    (1000, 1200, 3000, 1, 6_000_000, nu.NU_SCHED_S2, 256, None),     # several C blocks, slots reused
+    (2048, 1536, 6144, 1, 0, nu.NU_SCHED_S2B, 512, None),            # B-first strips and C-strip slots
+    (640, 900, 1500, 2, 0, nu.NU_SCHED_S2, 256, None),               # shared staging between siblings
+    (512, 512, 512, 1, 0, nu.NU_SCHED_S1, 0, (128, 128, 128)),       # S1: row shard kept, blocks drained
+])
+def test_slot_reuse_under_slow_compute(monkeypatch, M, N, K, G, cap, sched, kc, block):
+    """SURVEY T2's race test: sibling 0's compute stream is held for 50x each
+    leaf's nominal time (NORTHUP_DEBUG_SLOW_SIBLING), so the copy streams run far
+    ahead of the leaves and every slot reuse, C-strip drain and shared-staging
+    pull must wait on its recorded dependency; integer inputs stay exact."""
+    monkeypatch.setenv("NORTHUP_DEBUG_SLOW_SIBLING", "0,5000")
+    C, a, b, st = run_host(M, N, K, G=G, cap=cap, block=block, schedule=sched, k_chunk=kc, kind="int", seed=7)
+    check(C, a, b, "int")
+    assert st["copies"] > 3
+
+
 @pytest.mark.parametrize("M,N,K", [(1, 4097, 300), (4097, 1, 300), (257, 3, 1), (3, 5, 70000), (33, 2049, 7)])
 def test_host_root_skinny_and_ragged(M, N, K):
     """Degenerate shapes through the HOST -> HBM tree (vectors, K = 1, a long K
