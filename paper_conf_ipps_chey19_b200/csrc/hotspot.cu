@@ -118,10 +118,12 @@ __device__ __forceinline__ float4 v5_row(const float4 c, const float4 p, const f
 // run's first and last rows first, compute the interior, wait at the next
 // iteration (1507 vs 1674 GCUPS): the mbarrier polling costs more issue slots
 // than the barrier skew it removes.)
+// qv: the lane's q per row in registers (the persistent kernel), else NULL and
+// q is read from the shared-memory tile `ps` one row ahead (v5).
 template <int V, int NW, bool EDGE, bool NAMED = false>
 __device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const float* __restrict__ ps,
                                            float* __restrict__ hb, int lane, int warp, int rtop, int rbot,
-                                           int cl, int cr, int k0 = 0) {
+                                           int cl, int cr, int k0 = 0, const float4* qv = nullptr) {
   constexpr int RW = 128;
   // The persistent kernel unrolls the iteration loop by two: the new rows then
   // alternate between two register sets instead of being moved back into the
@@ -149,7 +151,7 @@ __device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const 
     // are too few to cover it otherwise).
     float wl_n = __shfl_up_sync(0xffffffffu, v[0].w, 1);
     float er_n = __shfl_down_sync(0xffffffffu, v[0].x, 1);
-    float4 p_n = ld_power(ps + (warp * V) * RW + 4 * lane);
+    float4 p_n = NAMED ? qv[0] : ld_power(ps + (warp * V) * RW + 4 * lane);
 #pragma unroll
     for (int r = 0; r < V; ++r) {
       const float4 c = v[r];
@@ -159,7 +161,7 @@ __device__ __forceinline__ void v5_iterate(const Args& a, float4 (&v)[V], const 
       if (r + 1 < V) {
         wl_n = __shfl_up_sync(0xffffffffu, v[r + 1].w, 1);
         er_n = __shfl_down_sync(0xffffffffu, v[r + 1].x, 1);
-        p_n = ld_power(ps + (warp * V + r + 1) * RW + 4 * lane);
+        p_n = NAMED ? qv[r + 1] : ld_power(ps + (warp * V + r + 1) * RW + 4 * lane);
       }
       v[r] = v5_row<EDGE>(c, p, prev, s, wl, er, a, EDGE && r == rtop, EDGE && r == rbot, cl, cr);
       prev = c;
@@ -230,17 +232,19 @@ __global__ void __launch_bounds__(NW * 32, 2) hotspot_kernel_v5(Args a) {
 
 // ---------------------------------------------------------------------------
 // Persistent TMA leaf (the product kernel when the window's base and leading
-// dimensions are 16-byte aligned): one CTA per SM walks the tiles
-// (128 columns x 132 rows, output 112 x 116 at 8 iterations) with 12 warps, 3
-// per SM sub-partition (a lane owns 4 columns x 11 rows, the v5 scheme above:
-// measured 1766 GCUPS against 1675 for 16 warps x 8 rows, 1709 for 12 x 10,
-// 1566 for 8 x 16 and 1493 for 10 x 12); thread 0 also issues the
-// loads.  While the warps iterate tile i, TMA brings tile i+1's
-// temperature (single buffer, freed as soon as the compute warps have copied
-// it into registers) and power (double buffer) into shared memory, so HBM
-// traffic overlaps the arithmetic instead of alternating with it.  Out-of-window
-// cells are zero-filled by TMA, as v5's predicated loads do.
-constexpr int kPW = 12, kPV = 11, kPRH = kPW * kPV, kPRW = 128;
+// dimensions are 16-byte aligned): one CTA per SM claims tiles (128 columns x
+// 128 rows, output 112 x 112 at 8 iterations) and runs them with 16 warps, 4
+// per SM sub-partition; a lane owns 4 columns x 8 rows (the v5 scheme above)
+// and keeps their temperature AND their q (RH4) in registers, so an
+// update reads nothing from shared memory but the two halo rows per iteration
+// (128 registers; measured 2379 GCUPS against 2330 for 12 warps x 10 rows, 2235
+// for 16 x 7, 2219 for 8 x 15, and 2022 with q read from shared memory).
+// Thread 0 also issues the loads.  While the warps iterate tile i, TMA brings
+// tile i+1's temperature (single buffer, freed as soon as the compute warps
+// have copied it into registers) and power (double buffer) into shared memory,
+// so HBM traffic overlaps the arithmetic instead of alternating with it.
+// Out-of-window cells are zero-filled by TMA, as v5's predicated loads do.
+constexpr int kPW = 16, kPV = 8, kPRH = kPW * kPV, kPRW = 128;
 
 // Tile t -> (tile row, tile column), row-major.  CTAs CLAIM tiles in this
 // order from a counter (atomicAdd) instead of taking a static t = c, c + grid,
@@ -254,8 +258,8 @@ __device__ __forceinline__ void tile_of(int t, int tiles_x, int& by, int& bx) {
   by = t / tiles_x;
   bx = t - by * tiles_x;
 }
-constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 66 KiB
-constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 24 KiB
+constexpr int kPTileBytes = kPRH * kPRW * 4;                    // 64 KiB
+constexpr int kPHaloFloats = 2 * kPW * 2 * kPRW;               // 32 KiB
 constexpr int kPSmem = 3 * kPTileBytes + kPHaloFloats * 4 + 64;   // T | P[2] | halo | barriers, tile ids
 
 __device__ __forceinline__ void tma_load_tile(uint32_t dst, const CUtensorMap* map, int x, int y, uint32_t bar) {
@@ -335,14 +339,13 @@ __global__ void __launch_bounds__(kPW * 32, 1)
     // power -> q of this lane's own cells (the only ones it reads back), in
     // place; the fence orders these generic writes before the TMA that will
     // refill the buffer once every warp has released it (pempty)
-    float* ps = pb + (i & 1) * kPRH * kPRW;
+    const float* ps = pb + (i & 1) * kPRH * kPRW;
+    float4 qv[kPV];
 #pragma unroll
     for (int r = 0; r < kPV; ++r) {
-      float* q = ps + (r0 + r) * kPRW + x0;
-      const float4 pv = ld_power(q);
-      *reinterpret_cast<float4*>(q) = make_float4(q_of(pv.x, a), q_of(pv.y, a), q_of(pv.z, a), q_of(pv.w, a));
+      const float4 pv = ld_power(ps + (r0 + r) * kPRW + x0);
+      qv[r] = make_float4(q_of(pv.x, a), q_of(pv.y, a), q_of(pv.z, a), q_of(pv.w, a));
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const int64_t gy_top = a.gy0 + ry, gx_left = a.gx0 + rx;
     const bool edge = gy_top <= 0 || gy_top + kPRH >= a.R || gx_left <= 0 || gx_left + kPRW >= a.C;
     if (edge) {
@@ -352,9 +355,9 @@ __global__ void __launch_bounds__(kPW * 32, 1)
       const int64_t gy = gy_top + r0;
       const int rtop = (gy <= 0 && gy > -kPV) ? static_cast<int>(-gy) : -1;
       const int rbot = (a.R - 1 - gy >= 0 && a.R - 1 - gy < kPV) ? static_cast<int>(a.R - 1 - gy) : -1;
-      v5_iterate<kPV, kPW, true, true>(a, v, ps, hb, lane, warp, rtop, rbot, cl, cr, i * h);
+      v5_iterate<kPV, kPW, true, true>(a, v, ps, hb, lane, warp, rtop, rbot, cl, cr, i * h, qv);
     } else {
-      v5_iterate<kPV, kPW, false, true>(a, v, ps, hb, lane, warp, -1, -1, -1, -1, i * h);
+      v5_iterate<kPV, kPW, false, true>(a, v, ps, hb, lane, warp, -1, -1, -1, -1, i * h, qv);
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(pempty0 + 8 * (i & 1));
