@@ -23,6 +23,7 @@
 #include <string.h>
 #include <unistd.h>
 
+#include <algorithm>
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
@@ -103,14 +104,16 @@ void bind_worker_thread(const northup_tree_s* t, int node) {
 }
 
 // The planner's PCIe term (S§8(d) "BW_e = the concurrently measured per-GPU
-// bandwidth with all links active"): every local GPU copies 64 MiB H2D and
-// 64 MiB D2H at once, twice; the slowest GPU's H2D rate of the second round.
+// bandwidth with all links active"): every local GPU copies 128 MiB H2D and
+// 128 MiB D2H at once, one warm-up round and four timed ones; each GPU's best
+// H2D rate (a single short round once read 27 instead of ~50 GB/s on a box,
+// and the planner then chose a much worse S2B split), the slowest GPU's.
 // Skipped for HBM roots (no host edge) and with NORTHUP_CALIBRATE=0.
 int calibrate_pcie(northup_tree_s* t) {
   t->pcie_gbs = 0.0;
   const char* env = getenv("NORTHUP_CALIBRATE");
   if ((env && env[0] == '0') || t->workers.empty() || t->nodes[0].storage == NU_HBM) return 0;
-  const size_t bytes = 64ull << 20;
+  const size_t bytes = 128ull << 20;
   const size_t W = t->workers.size();
   std::vector<void*> hin(W, nullptr), hout(W, nullptr), din(W, nullptr), dout(W, nullptr);
   std::vector<cudaEvent_t> ev(4 * W, nullptr);
@@ -124,8 +127,8 @@ int calibrate_pcie(northup_tree_s* t) {
     for (int k = 0; k < 4 && !rc; ++k)
       if (cudaEventCreate(&ev[4 * i + k]) != cudaSuccess) rc = 1;
   }
-  double worst = 0.0;
-  for (int round = 0; round < 2 && !rc; ++round) {
+  std::vector<double> best(W, 0.0);
+  for (int round = 0; round < 5 && !rc; ++round) {
     for (size_t i = 0; i < W; ++i) {
       WorkerState* w = t->workers[i];
       cudaSetDevice(w->device);
@@ -136,19 +139,19 @@ int calibrate_pcie(northup_tree_s* t) {
       cudaMemcpyAsync(hout[i], dout[i], bytes, cudaMemcpyDeviceToHost, w->streams[S_D2H]);
       cudaEventRecord(ev[4 * i + 3], w->streams[S_D2H]);
     }
-    worst = 1e30;
     for (size_t i = 0; i < W; ++i) {
       cudaSetDevice(t->workers[i]->device);
       float ms = 0.f;
       if (cudaEventSynchronize(ev[4 * i + 1]) != cudaSuccess ||
           cudaEventElapsedTime(&ms, ev[4 * i + 0], ev[4 * i + 1]) != cudaSuccess || ms <= 0.f) {
-        worst = 0.0;
+        rc = 1;
         break;
       }
-      worst = std::min(worst, bytes / (ms * 1e-3) / 1e9);
+      if (round > 0) best[i] = std::max(best[i], bytes / (ms * 1e-3) / 1e9);   // round 0: warm-up
       cudaEventSynchronize(ev[4 * i + 3]);
     }
   }
+  double worst = rc || W == 0 ? 0.0 : *std::min_element(best.begin(), best.end());
   for (size_t i = 0; i < W; ++i) {
     cudaSetDevice(t->workers[i]->device);
     if (hin[i]) cudaFreeHost(hin[i]);
