@@ -231,6 +231,44 @@ __global__ void __launch_bounds__(1024) split_b_kernel(const float* B, int64_t l
   }
 }
 
+// In place, vectorised (N % 4 == 0, 16-B aligned rows): one CTA of 1024
+// threads per row holds the whole row in registers (float4 loads, at most 12
+// per thread for N <= 49152), then writes the hi and lo halves as 8-byte
+// stores.  The shared-memory version above (scalar 2-byte stores) moved a
+// 32768-wide panel at ~1.5 TB/s.
+constexpr int kSplitVecPerThread = 12;
+__global__ void __launch_bounds__(1024) split_b_inplace_vec_kernel(float* B, int64_t ldb, int Kl, int N,
+                                                                   const int* __restrict__ eb) {
+  const int k = blockIdx.x;
+  const int N4 = N / 4;
+  float4* row = reinterpret_cast<float4*>(B + static_cast<int64_t>(k) * ldb);
+  float4 x[kSplitVecPerThread];
+#pragma unroll
+  for (int j = 0; j < kSplitVecPerThread; ++j) {
+    const int i = threadIdx.x + j * 1024;
+    x[j] = (k < Kl && i < N4) ? row[i] : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  __syncthreads();                                   // the whole row is read before any of it is overwritten
+  __half* hi_row = reinterpret_cast<__half*>(row);
+#pragma unroll
+  for (int j = 0; j < kSplitVecPerThread; ++j) {
+    const int i = threadIdx.x + j * 1024;
+    if (i >= N4) break;
+    const int n = 4 * i;
+    __half h[4], l[4];
+    split1(x[j].x, pow2(-eb[n]), h[0], l[0]);
+    split1(x[j].y, pow2(-eb[n + 1]), h[1], l[1]);
+    split1(x[j].z, pow2(-eb[n + 2]), h[2], l[2]);
+    split1(x[j].w, pow2(-eb[n + 3]), h[3], l[3]);
+    *reinterpret_cast<uint2*>(hi_row + n) =
+        make_uint2(__half_as_ushort(h[0]) | (static_cast<uint32_t>(__half_as_ushort(h[1])) << 16),
+                   __half_as_ushort(h[2]) | (static_cast<uint32_t>(__half_as_ushort(h[3])) << 16));
+    *reinterpret_cast<uint2*>(hi_row + ldb + n) =
+        make_uint2(__half_as_ushort(l[0]) | (static_cast<uint32_t>(__half_as_ushort(l[1])) << 16),
+                   __half_as_ushort(l[2]) | (static_cast<uint32_t>(__half_as_ushort(l[3])) << 16));
+  }
+}
+
 int64_t split_b_max_n() { return kSplitRowMaxN; }
 
 int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64_t ldd, int* ea, int sms,
@@ -263,6 +301,9 @@ int split_b_launch(const float* B, int64_t ldb, int Kl, int N, float* dst, int64
                    reinterpret_cast<uintptr_t>(B) % 16 == 0 && reinterpret_cast<uintptr_t>(dst) % 16 == 0;
   if (vec) {
     split_b_oop_kernel<<<dim3((N / 4 + 255) / 256, (Kp + 7) / 8), 256, 0, s>>>(B, ldb, Kl, Kp, N, eb, dst, ldd);
+  } else if (dst == B && ldd == ldb && N % 4 == 0 && ldb % 4 == 0 && reinterpret_cast<uintptr_t>(B) % 16 == 0 &&
+             N <= 4 * 1024 * kSplitVecPerThread) {
+    split_b_inplace_vec_kernel<<<Kp, 1024, 0, s>>>(const_cast<float*>(B), ldb, Kl, N, eb);
   } else {
     static bool configured[kMaxDevices];
     int dev = 0;
@@ -300,6 +341,7 @@ void preload_split() {
   cudaFuncGetAttributes(&fa, colmax_kernel);
   cudaFuncGetAttributes(&fa, split_b_kernel);
   cudaFuncGetAttributes(&fa, split_b_oop_kernel);
+  cudaFuncGetAttributes(&fa, split_b_inplace_vec_kernel);
   cudaFuncGetAttributes(&fa, col_exps_kernel);
   cudaFuncGetAttributes(&fa, split_ab_small_kernel);
 }
