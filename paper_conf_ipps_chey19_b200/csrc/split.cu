@@ -125,6 +125,63 @@ __global__ void __launch_bounds__(256) split_a_kernel(const float* A, int64_t ld
   split_a_rows(A, lda, M, Kl, Kp, dst, ldd, ea, vec, blockIdx.x, gridDim.x);
 }
 
+// Few rows (a 1024-row strip of S2B's second phase): four warps per row, each
+// over a quarter of the panel's K (a multiple of 32 k, so no 32-k group is
+// shared), the row maximum combined through shared memory.  The same exponent
+// and the same per-element conversion as split_a_rows: bitwise the same split,
+// with four times the warps in flight (a warp per row left ~7 per SM).
+__global__ void __launch_bounds__(256) split_a_quarters_kernel(const float* A, int64_t lda, int M, int Kl, int Kp,
+                                                               int Q, float* dst, int64_t ldd, int* ea, int vec) {
+  __shared__ float mx[2][4];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int r = blockIdx.x * 2 + (warp >> 2), q = warp & 3;
+  const int k0 = q * Q, k1 = min(Kp, k0 + Q), kl1 = min(Kl, k1);
+  const float* a = A + static_cast<int64_t>(min(r, M - 1)) * lda;
+  float m = 0.f;
+  if (r < M) {
+    int k = k0;
+    if (vec)
+      for (; k + 128 <= kl1; k += 128) {
+        const float4 x = *reinterpret_cast<const float4*>(a + k + 4 * lane);
+        m = fmaxf(fmaxf(m, fmaxf(fabsf(x.x), fabsf(x.y))), fmaxf(fabsf(x.z), fabsf(x.w)));
+      }
+    for (k += lane; k < kl1; k += 32) m = fmaxf(m, fabsf(a[k]));
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if (lane == 0) mx[warp >> 2][q] = m;
+  __syncthreads();
+  if (r >= M) return;
+  const float* mr = mx[warp >> 2];
+  const int e = split_exponent(fmaxf(fmaxf(mr[0], mr[1]), fmaxf(mr[2], mr[3])));
+  if (q == 0 && lane == 0) ea[r] = e;
+  const float s = pow2(-e);
+  __half* out = reinterpret_cast<__half*>(dst + static_cast<int64_t>(r) * ldd);
+  int kv = k0;
+  if (vec) {
+    for (; kv + 128 <= kl1; kv += 128) {
+      const float4 x = *reinterpret_cast<const float4*>(a + kv + 4 * lane);
+      __syncwarp();                            // the 512 bytes are read before they are overwritten
+      uint2 hi, lo;
+      split4(x, s, hi, lo);
+      const int g = lane >> 3, c = 4 * (lane & 7);
+      *reinterpret_cast<uint2*>(out + 2 * (kv + 32 * g) + c) = hi;
+      *reinterpret_cast<uint2*>(out + 2 * (kv + 32 * g) + 32 + c) = lo;
+      __syncwarp();
+    }
+  }
+  for (int g0 = kv; g0 < k1; g0 += 32) {
+    const int k = g0 + lane;
+    const float x = k < Kl ? a[k] : 0.f;
+    __syncwarp();                              // the group is read before it is overwritten
+    __half hi, lo;
+    split1(x, s, hi, lo);
+    out[2 * g0 + lane] = hi;
+    out[2 * g0 + 32 + lane] = lo;
+    __syncwarp();
+  }
+}
+
 // Small panels (cfg1-like leaf calls): the A split and the whole B split
 // (column maxima, exponents, hi / lo) in ONE launch instead of five.  Blocks
 // [0, ga) split rows of A as split_a_kernel does; each further block takes 32
@@ -278,7 +335,12 @@ int split_a_launch(const float* A, int64_t lda, int M, int Kl, float* dst, int64
   const int grid = static_cast<int>(std::min<int64_t>((M + 7) / 8, 32LL * sms));
   const int vec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && lda % 4 == 0 &&
                   (reinterpret_cast<uintptr_t>(dst) % 16 == 0) && ldd % 4 == 0;
-  split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea, vec);
+  if (M < 8 * sms && Kp >= 4 * 128) {
+    const int Q = (Kp / 4 + 127) / 128 * 128;   // a multiple of 128 k (the vector step) and of 32
+    split_a_quarters_kernel<<<(M + 1) / 2, 256, 0, s>>>(A, lda, M, Kl, Kp, Q, dst, ldd, ea, vec);
+  } else {
+    split_a_kernel<<<grid, 256, 0, s>>>(A, lda, M, Kl, Kp, dst, ldd, ea, vec);
+  }
   count_launches(1);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 0 : fail(NU_ECUDA, "split_a launch: %s", cudaGetErrorString(e));
@@ -338,6 +400,7 @@ int split_ab_small_launch(const float* A, int64_t lda, int M, int Kl, float* ads
 void preload_split() {
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, split_a_kernel);
+  cudaFuncGetAttributes(&fa, split_a_quarters_kernel);
   cudaFuncGetAttributes(&fa, colmax_kernel);
   cudaFuncGetAttributes(&fa, split_b_kernel);
   cudaFuncGetAttributes(&fa, split_b_oop_kernel);
