@@ -388,7 +388,12 @@ int northup_peer_import(northup_tree_t t, int worker, const void* blob, uint64_t
  *   T'[r,c] = T + cap_1 * (P + (T[r+1,c] + T[r-1,c] - 2T) * ry_1
  *                            + (T[r,c+1] + T[r,c-1] - 2T) * rx_1 + (amb - T) * rz_1)
  * with out-of-grid neighbours replaced by the cell itself (RH1), in
- * fp32, evaluated left to right with round-to-nearest and no contraction. */
+ * fp32 through one fixed sequence of the expanded form (RH4):
+ *   kt = 1 - cap_1 (2 rx_1 + 2 ry_1 + rz_1), kx = cap_1 rx_1, ky = cap_1 ry_1,
+ *   kq = cap_1 rz_1 amb (each rounded once to fp32), q = fma(cap_1, P, kq),
+ *   T' = fma(ky, S + N, fma(kx, E + W, fma(kt, T, q)))
+ * (round-to-nearest; identical on every path, so in-HBM and out-of-core runs
+ * agree bit for bit; within RH3's bound of the fp64 definition). */
 typedef struct {
   float cap_1, rx_1, ry_1, rz_1, amb;
 } northup_hotspot_coeffs;
