@@ -224,6 +224,15 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   st.bk = h;
   st.hbm_peak_bytes = arena_bytes(b, h);
   std::vector<int64_t> slot_ctr(G, 0);
+  // Each sibling's previous window of the same pass: a window that shares its
+  // rows takes the power columns it has in common with it from that window's
+  // slot (a device copy) instead of over PCIe again (2h columns per block; P is
+  // read-only, unlike the temperature windows, which the iterations overwrite).
+  struct PrevWin {
+    bool valid = false;
+    int64_t q = -1, y0 = 0, y1 = 0, x0 = 0, x1 = 0, poff = 0;
+  };
+  std::vector<PrevWin> prevw(G);
   int src = T;
   for (int64_t q = 0; q < Q; ++q) {
     const int64_t itq = std::min(h, iters - q * h);
@@ -273,9 +282,21 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
         const int64_t go = win_g.y0 * C + win_g.x0;
         B.emit(make_copy(w, S_H2D, src, go, ldg_src, arena[w], off[0], LD, wm, wn),
                {{src, go, ldg_src, wm, wn, false}, {arena[w], off[0], LD, wm, wn, true}});
-        B.emit(make_copy(w, S_H2D, PW, go, C, arena[w], poff, LD, wm, wn),
-               {{PW, go, C, wm, wn, false}, {arena[w], poff, LD, wm, wn, true}});
-        st.bytes_h2d += 8ull * wm * wn;
+        int64_t pc0 = 0;   // P columns [0, pc0) of this window come from the previous window's slot
+        const PrevWin& pv = prevw[w];
+        if (pv.valid && pv.q == q && pv.y0 == win_g.y0 && pv.y1 == win_g.y1 && pv.x0 < win_g.x0 &&
+            pv.x1 > win_g.x0) {
+          pc0 = std::min(pv.x1, win_g.x1) - win_g.x0;
+          const int64_t so = pv.poff + (win_g.x0 - pv.x0);
+          B.emit(make_copy(w, S_D2D, arena[w], so, LD, arena[w], poff, LD, wm, pc0),
+                 {{arena[w], so, LD, wm, pc0, false}, {arena[w], poff, LD, wm, pc0, true}});
+          st.bytes_d2d += 4ull * wm * pc0;
+        }
+        if (wn > pc0)
+          B.emit(make_copy(w, S_H2D, PW, go + pc0, C, arena[w], poff + pc0, LD, wm, wn - pc0),
+                 {{PW, go + pc0, C, wm, wn - pc0, false}, {arena[w], poff + pc0, LD, wm, wn - pc0, true}});
+        st.bytes_h2d += 4ull * wm * wn + 4ull * wm * (wn - pc0);
+        prevw[w] = PrevWin{true, q, win_g.y0, win_g.y1, win_g.x0, win_g.x1, poff};
         const int fin = emit_iterations(B, w, win_g, itq, hl, bufs, off, arena[w], poff, LD, win_g.y0,
                                         win_g.x0, R, C, &st);
         // data_up: the block

@@ -96,6 +96,14 @@ def test_hotspot_plan_replays_exactly(R, C, iters, G, cap, block, halo, leaf):
         nwin = sum(1 for o in p.ops() if o["op"] == nu.NU_OP_COPY and o["stream"] == 0) // 2
         assert nwin > -(-R // b) * -(-C // b) * -(-iters // h)
     assert s["bytes_d2h"] == 4 * R * C * -(-iters // h)          # every pass writes the grid once
+    # every window byte arrives once: over PCIe, or (power columns shared with the
+    # sibling's previous window of the same rows) by a device copy from its slot
+    bufs = p.bufs()
+    into_arena = sum(4 * o["rows"] * o["cols"] for o in p.ops()
+                     if o["op"] == nu.NU_OP_COPY and bufs[o["dst_buf"]]["kind"] == 3)
+    assert s["bytes_h2d"] + s["bytes_d2d"] == into_arena
+    if -(-C // b) > 1:
+        assert s["bytes_d2d"] > 0
     if cap:
         assert all(x["bytes"] <= cap for x in p.bufs() if x["kind"] == 3)
     t.destroy()
