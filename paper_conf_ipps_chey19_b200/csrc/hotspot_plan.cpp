@@ -187,9 +187,13 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
     if (t->nodes[h].capacity) cap = cap ? std::min(cap, t->nodes[h].capacity) : t->nodes[h].capacity;
   constexpr int kS = kSlots;
   // slot footprint: three windows (temperature ping, pong, power), (b + 2h) square
+  // slots of three windows (temperature ping, pong, power), (b + 2h) square,
+  // plus two staging strips (window rows x 2h) for the temperature columns a
+  // window shares with the next one (see below)
   auto arena_bytes = [&](int64_t b, int64_t h) {
     const int64_t W = std::min(b + 2 * h, std::max(R, C));
-    return 4ull * kS * 3 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(std::min(W, C));
+    return 4ull * kS * 3 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(std::min(W, C)) +
+           4ull * 2 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(2 * h);
   };
   const int64_t edge = std::max(R, C);
   int64_t b = o && o->block > 0 ? o->block : std::min<int64_t>(edge, 8192);   // P:325 8k blocking
@@ -233,6 +237,18 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
     int64_t q = -1, y0 = 0, y1 = 0, x0 = 0, x1 = 0, poff = 0;
   };
   std::vector<PrevWin> prevw(G);
+  // The temperature columns two such windows share are copied out of the
+  // earlier window (into one of two staging strips after its slot is loaded,
+  // before its second launch overwrites them) and into the later one, so they
+  // do not cross PCIe twice either.
+  const int64_t SLD = pad_ld(2 * h);                                // staging strip leading dimension
+  const int64_t stg0 = static_cast<int64_t>(kS) * 3 * win;          // first strip (elements)
+  std::vector<int> stg_next(G, 0);                                  // strip the next hand-off uses
+  std::vector<int> stg_have(G, -1);                                 // strip holding the hand-off for the next window
+  auto window_of = [&](const Win& blk, int64_t itq) {
+    return Win{std::max<int64_t>(0, blk.y0 - itq), std::min(R, blk.y1 + itq), std::max<int64_t>(0, blk.x0 - itq),
+               std::min(C, blk.x1 + itq)};
+  };
   int src = T;
   for (int64_t q = 0; q < Q; ++q) {
     const int64_t itq = std::min(h, iters - q * h);
@@ -270,8 +286,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
       const int w = owner[bi];
       {
         const Win blk = blks[bi];
-        const Win win_g{std::max<int64_t>(0, blk.y0 - itq), std::min(R, blk.y1 + itq),
-                        std::max<int64_t>(0, blk.x0 - itq), std::min(C, blk.x1 + itq)};
+        const Win win_g = window_of(blk, itq);
         const int64_t wm = win_g.y1 - win_g.y0, wn = win_g.x1 - win_g.x0;
         const int sl = static_cast<int>(slot_ctr[w]++ % kS);
         const int64_t base = static_cast<int64_t>(sl) * 3 * win;
@@ -280,13 +295,42 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
         const int bufs[2] = {arena[w], arena[w]};
         // data_down: window of the current grid and of P (block + borders)
         const int64_t go = win_g.y0 * C + win_g.x0;
-        B.emit(make_copy(w, S_H2D, src, go, ldg_src, arena[w], off[0], LD, wm, wn),
-               {{src, go, ldg_src, wm, wn, false}, {arena[w], off[0], LD, wm, wn, true}});
-        int64_t pc0 = 0;   // P columns [0, pc0) of this window come from the previous window's slot
         const PrevWin& pv = prevw[w];
-        if (pv.valid && pv.q == q && pv.y0 == win_g.y0 && pv.y1 == win_g.y1 && pv.x0 < win_g.x0 &&
-            pv.x1 > win_g.x0) {
-          pc0 = std::min(pv.x1, win_g.x1) - win_g.x0;
+        const bool shares = pv.valid && pv.q == q && pv.y0 == win_g.y0 && pv.y1 == win_g.y1 && pv.x0 < win_g.x0 &&
+                            pv.x1 > win_g.x0;
+        const int64_t ov = shares ? std::min(pv.x1, win_g.x1) - win_g.x0 : 0;   // shared columns
+        int64_t tc0 = 0;   // T columns [0, tc0) of this window come from a staging strip
+        if (shares && stg_have[w] >= 0 && ov <= 2 * h) {
+          tc0 = ov;
+          const int64_t so = stg0 + static_cast<int64_t>(stg_have[w]) * WR * SLD;
+          B.emit(make_copy(w, S_D2D, arena[w], so, SLD, arena[w], off[0], LD, wm, tc0),
+                 {{arena[w], so, SLD, wm, tc0, false}, {arena[w], off[0], LD, wm, tc0, true}});
+          st.bytes_d2d += 4ull * wm * tc0;
+        }
+        stg_have[w] = -1;
+        if (wn > tc0)
+          B.emit(make_copy(w, S_H2D, src, go + tc0, ldg_src, arena[w], off[0] + tc0, LD, wm, wn - tc0),
+                 {{src, go + tc0, ldg_src, wm, wn - tc0, false}, {arena[w], off[0] + tc0, LD, wm, wn - tc0, true}});
+        // hand the columns this window shares with the sibling's next window
+        // (same pass, same rows) to a staging strip before the iterations
+        // overwrite them
+        if (bi + 1 < blks.size() && owner[bi + 1] == w) {
+          const Win nx = window_of(blks[bi + 1], itq);
+          const int64_t ovn = nx.y0 == win_g.y0 && nx.y1 == win_g.y1 && nx.x0 > win_g.x0 && nx.x0 < win_g.x1
+                                  ? std::min(win_g.x1, nx.x1) - nx.x0 : 0;
+          if (ovn > 0 && ovn <= 2 * h) {
+            const int sidx = stg_next[w];
+            stg_next[w] ^= 1;
+            const int64_t so = off[0] + (nx.x0 - win_g.x0), dso = stg0 + static_cast<int64_t>(sidx) * WR * SLD;
+            B.emit(make_copy(w, S_D2D, arena[w], so, LD, arena[w], dso, SLD, wm, ovn),
+                   {{arena[w], so, LD, wm, ovn, false}, {arena[w], dso, SLD, wm, ovn, true}});
+            st.bytes_d2d += 4ull * wm * ovn;
+            stg_have[w] = sidx;
+          }
+        }
+        int64_t pc0 = 0;   // P columns [0, pc0) of this window come from the previous window's slot
+        if (shares) {
+          pc0 = ov;
           const int64_t so = pv.poff + (win_g.x0 - pv.x0);
           B.emit(make_copy(w, S_D2D, arena[w], so, LD, arena[w], poff, LD, wm, pc0),
                  {{arena[w], so, LD, wm, pc0, false}, {arena[w], poff, LD, wm, pc0, true}});
@@ -295,7 +339,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
         if (wn > pc0)
           B.emit(make_copy(w, S_H2D, PW, go + pc0, C, arena[w], poff + pc0, LD, wm, wn - pc0),
                  {{PW, go + pc0, C, wm, wn - pc0, false}, {arena[w], poff + pc0, LD, wm, wn - pc0, true}});
-        st.bytes_h2d += 4ull * wm * wn + 4ull * wm * (wn - pc0);
+        st.bytes_h2d += 4ull * wm * (wn - tc0) + 4ull * wm * (wn - pc0);
         prevw[w] = PrevWin{true, q, win_g.y0, win_g.y1, win_g.x0, win_g.x1, poff};
         const int fin = emit_iterations(B, w, win_g, itq, hl, bufs, off, arena[w], poff, LD, win_g.y0,
                                         win_g.x0, R, C, &st);
