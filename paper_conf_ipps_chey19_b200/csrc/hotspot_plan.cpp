@@ -186,6 +186,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   for (int h : hbm)
     if (t->nodes[h].capacity) cap = cap ? std::min(cap, t->nodes[h].capacity) : t->nodes[h].capacity;
   constexpr int kS = kSlots;
+  constexpr int kRowBands = 3;   // row-band staging buffers per sibling (T and P, full grid width)
   // slot footprint: three windows (temperature ping, pong, power), (b + 2h) square
   // slots of three windows (temperature ping, pong, power), (b + 2h) square,
   // plus two staging strips (window rows x 2h) for the temperature columns a
@@ -193,7 +194,8 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   auto arena_bytes = [&](int64_t b, int64_t h) {
     const int64_t W = std::min(b + 2 * h, std::max(R, C));
     return 4ull * kS * 3 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(std::min(W, C)) +
-           4ull * 2 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(2 * h);
+           4ull * 2 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(2 * h) +
+           4ull * kRowBands * 2 * static_cast<uint64_t>(2 * h) * pad_ld(C);
   };
   const int64_t edge = std::max(R, C);
   int64_t b = o && o->block > 0 ? o->block : std::min<int64_t>(edge, 8192);   // P:325 8k blocking
@@ -245,6 +247,32 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   const int64_t stg0 = static_cast<int64_t>(kS) * 3 * win;          // first strip (elements)
   std::vector<int> stg_next(G, 0);                                  // strip the next hand-off uses
   std::vector<int> stg_have(G, -1);                                 // strip holding the hand-off for the next window
+  // Row bands: the 2 itq rows a window shares with the sibling's window below
+  // it (same pass, same columns or a subset) are copied, T and P, into a
+  // full-width band buffer after the upper window lands (before its second
+  // launch overwrites T) and from there into the lower window.
+  const int64_t LDC = pad_ld(C), rs0 = stg0 + 2 * WR * SLD;
+  auto rs_t = [&](int buf) { return rs0 + static_cast<int64_t>(buf) * 2 * (2 * h) * LDC; };
+  auto rs_p = [&](int buf) { return rs_t(buf) + (2 * h) * LDC; };
+  struct Band {
+    int64_t row = -1, q = -1;
+    int buf = -1;
+    std::vector<std::pair<int64_t, int64_t>> cov;   // grid columns staged so far
+    bool covers(int64_t x0, int64_t x1) const {
+      int64_t at = x0;   // intervals arrive left to right per block row
+      for (bool grew = true; grew && at < x1;) {
+        grew = false;
+        for (const auto& c : cov)
+          if (c.first <= at && c.second > at) {
+            at = c.second;
+            grew = true;
+          }
+      }
+      return at >= x1;
+    }
+  };
+  std::vector<std::vector<Band>> bands(G);
+  std::vector<int> rs_next(G, 0);
   auto window_of = [&](const Win& blk, int64_t itq) {
     return Win{std::max<int64_t>(0, blk.y0 - itq), std::min(R, blk.y1 + itq), std::max<int64_t>(0, blk.x0 - itq),
                std::min(C, blk.x1 + itq)};
@@ -259,6 +287,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
     // last block of the last pass are split 2 x 2: the pipeline fills after a
     // quarter-size window and drains a quarter-size block (a little more border
     // recomputation on those two blocks only).
+    for (auto& bl : bands) bl.clear();
     std::vector<Win> blks;
     std::vector<int> owner;
     for (int64_t by = 0; by < nby; ++by) {
@@ -293,24 +322,54 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
         const int64_t off[2] = {base, base + win};
         const int64_t poff = base + 2 * win;
         const int bufs[2] = {arena[w], arena[w]};
-        // data_down: window of the current grid and of P (block + borders)
-        const int64_t go = win_g.y0 * C + win_g.x0;
+        // data_down: window of the current grid and of P (block + borders).
+        // Rows [0, r_lo) may come from a row band, columns [0, tc0) / [0, pc0)
+        // of the other rows from the sibling's previous window; the rest over PCIe.
+        const int64_t bh = 2 * itq;
+        int64_t r_lo = 0;
+        if (win_g.y0 > 0 && wm > bh) {
+          for (const Band& bd : bands[w])
+            if (bd.q == q && bd.row == win_g.y0 && bd.covers(win_g.x0, win_g.x1)) {
+              r_lo = bh;
+              B.emit(make_copy(w, S_D2D, arena[w], rs_t(bd.buf) + win_g.x0, LDC, arena[w], off[0], LD, bh, wn),
+                     {{arena[w], rs_t(bd.buf) + win_g.x0, LDC, bh, wn, false}, {arena[w], off[0], LD, bh, wn, true}});
+              B.emit(make_copy(w, S_D2D, arena[w], rs_p(bd.buf) + win_g.x0, LDC, arena[w], poff, LD, bh, wn),
+                     {{arena[w], rs_p(bd.buf) + win_g.x0, LDC, bh, wn, false}, {arena[w], poff, LD, bh, wn, true}});
+              st.bytes_d2d += 8ull * bh * wn;
+              break;
+            }
+        }
+        const int64_t rm = wm - r_lo;                                  // rows not from a band
+        const int64_t go = (win_g.y0 + r_lo) * C + win_g.x0;
+        const int64_t to = off[0] + r_lo * LD, po = poff + r_lo * LD;   // their start in the slot
         const PrevWin& pv = prevw[w];
         const bool shares = pv.valid && pv.q == q && pv.y0 == win_g.y0 && pv.y1 == win_g.y1 && pv.x0 < win_g.x0 &&
                             pv.x1 > win_g.x0;
         const int64_t ov = shares ? std::min(pv.x1, win_g.x1) - win_g.x0 : 0;   // shared columns
-        int64_t tc0 = 0;   // T columns [0, tc0) of this window come from a staging strip
+        int64_t tc0 = 0;   // T columns [0, tc0) of those rows come from a staging strip
         if (shares && stg_have[w] >= 0 && ov <= 2 * h) {
           tc0 = ov;
-          const int64_t so = stg0 + static_cast<int64_t>(stg_have[w]) * WR * SLD;
-          B.emit(make_copy(w, S_D2D, arena[w], so, SLD, arena[w], off[0], LD, wm, tc0),
-                 {{arena[w], so, SLD, wm, tc0, false}, {arena[w], off[0], LD, wm, tc0, true}});
-          st.bytes_d2d += 4ull * wm * tc0;
+          const int64_t so = stg0 + static_cast<int64_t>(stg_have[w]) * WR * SLD + r_lo * SLD;
+          B.emit(make_copy(w, S_D2D, arena[w], so, SLD, arena[w], to, LD, rm, tc0),
+                 {{arena[w], so, SLD, rm, tc0, false}, {arena[w], to, LD, rm, tc0, true}});
+          st.bytes_d2d += 4ull * rm * tc0;
         }
         stg_have[w] = -1;
         if (wn > tc0)
-          B.emit(make_copy(w, S_H2D, src, go + tc0, ldg_src, arena[w], off[0] + tc0, LD, wm, wn - tc0),
-                 {{src, go + tc0, ldg_src, wm, wn - tc0, false}, {arena[w], off[0] + tc0, LD, wm, wn - tc0, true}});
+          B.emit(make_copy(w, S_H2D, src, go + tc0, ldg_src, arena[w], to + tc0, LD, rm, wn - tc0),
+                 {{src, go + tc0, ldg_src, rm, wn - tc0, false}, {arena[w], to + tc0, LD, rm, wn - tc0, true}});
+        int64_t pc0 = 0;   // P columns [0, pc0) of those rows come from the previous window's slot
+        if (shares) {
+          pc0 = ov;
+          const int64_t so = pv.poff + r_lo * LD + (win_g.x0 - pv.x0);
+          B.emit(make_copy(w, S_D2D, arena[w], so, LD, arena[w], po, LD, rm, pc0),
+                 {{arena[w], so, LD, rm, pc0, false}, {arena[w], po, LD, rm, pc0, true}});
+          st.bytes_d2d += 4ull * rm * pc0;
+        }
+        if (wn > pc0)
+          B.emit(make_copy(w, S_H2D, PW, go + pc0, C, arena[w], po + pc0, LD, rm, wn - pc0),
+                 {{PW, go + pc0, C, rm, wn - pc0, false}, {arena[w], po + pc0, LD, rm, wn - pc0, true}});
+        st.bytes_h2d += 4ull * rm * (wn - tc0) + 4ull * rm * (wn - pc0);
         // hand the columns this window shares with the sibling's next window
         // (same pass, same rows) to a staging strip before the iterations
         // overwrite them
@@ -328,18 +387,36 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
             stg_have[w] = sidx;
           }
         }
-        int64_t pc0 = 0;   // P columns [0, pc0) of this window come from the previous window's slot
-        if (shares) {
-          pc0 = ov;
-          const int64_t so = pv.poff + (win_g.x0 - pv.x0);
-          B.emit(make_copy(w, S_D2D, arena[w], so, LD, arena[w], poff, LD, wm, pc0),
-                 {{arena[w], so, LD, wm, pc0, false}, {arena[w], poff, LD, wm, pc0, true}});
-          st.bytes_d2d += 4ull * wm * pc0;
+        // and the rows it shares with a later window of the sibling below it
+        if (win_g.y1 < R && wm > bh) {
+          const int64_t brow = win_g.y1 - bh;
+          bool needed = false;
+          for (size_t bj = bi + 1; bj < blks.size() && !needed; ++bj) {
+            if (owner[bj] != w) continue;
+            const Win lw = window_of(blks[bj], itq);
+            needed = lw.y0 == brow && lw.x0 < win_g.x1 && lw.x1 > win_g.x0;
+          }
+          if (needed) {
+            Band* bd = nullptr;
+            for (Band& x : bands[w])
+              if (x.q == q && x.row == brow) bd = &x;
+            if (!bd) {
+              const int buf = rs_next[w];
+              rs_next[w] = (rs_next[w] + 1) % kRowBands;
+              auto& bl = bands[w];
+              bl.erase(std::remove_if(bl.begin(), bl.end(), [&](const Band& x) { return x.buf == buf; }), bl.end());
+              bl.push_back(Band{brow, q, buf, {}});
+              bd = &bl.back();
+            }
+            const int64_t tso = off[0] + (wm - bh) * LD, pso = poff + (wm - bh) * LD;
+            B.emit(make_copy(w, S_D2D, arena[w], tso, LD, arena[w], rs_t(bd->buf) + win_g.x0, LDC, bh, wn),
+                   {{arena[w], tso, LD, bh, wn, false}, {arena[w], rs_t(bd->buf) + win_g.x0, LDC, bh, wn, true}});
+            B.emit(make_copy(w, S_D2D, arena[w], pso, LD, arena[w], rs_p(bd->buf) + win_g.x0, LDC, bh, wn),
+                   {{arena[w], pso, LD, bh, wn, false}, {arena[w], rs_p(bd->buf) + win_g.x0, LDC, bh, wn, true}});
+            st.bytes_d2d += 8ull * bh * wn;
+            bd->cov.emplace_back(win_g.x0, win_g.x1);
+          }
         }
-        if (wn > pc0)
-          B.emit(make_copy(w, S_H2D, PW, go + pc0, C, arena[w], poff + pc0, LD, wm, wn - pc0),
-                 {{PW, go + pc0, C, wm, wn - pc0, false}, {arena[w], poff + pc0, LD, wm, wn - pc0, true}});
-        st.bytes_h2d += 4ull * wm * (wn - tc0) + 4ull * wm * (wn - pc0);
         prevw[w] = PrevWin{true, q, win_g.y0, win_g.y1, win_g.x0, win_g.x1, poff};
         const int fin = emit_iterations(B, w, win_g, itq, hl, bufs, off, arena[w], poff, LD, win_g.y0,
                                         win_g.x0, R, C, &st);
