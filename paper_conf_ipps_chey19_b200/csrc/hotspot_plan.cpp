@@ -194,9 +194,10 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   auto arena_bytes = [&](int64_t b, int64_t h) {
     const int64_t W = std::min(b + 2 * h, std::max(R, C));
     return 4ull * kS * 3 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(std::min(W, C)) +
-           4ull * 2 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(2 * h) +
-           4ull * kRowBands * 2 * static_cast<uint64_t>(2 * h) * pad_ld(C);
+           4ull * 2 * static_cast<uint64_t>(std::min(W, R)) * pad_ld(2 * h);
   };
+  // the row-band buffers (full grid width) come on top, only when they fit
+  auto band_bytes = [&](int64_t h) { return 4ull * kRowBands * 2 * static_cast<uint64_t>(2 * h) * pad_ld(C); };
   const int64_t edge = std::max(R, C);
   int64_t b = o && o->block > 0 ? o->block : std::min<int64_t>(edge, 8192);   // P:325 8k blocking
   int64_t h = o && o->halo > 0 ? o->halo : 0;
@@ -222,13 +223,15 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
   const int64_t WR = std::min(W, R), LD = pad_ld(std::min(W, C));
   const int64_t win = WR * LD;   // elements per window buffer
   std::vector<int> arena(G);
-  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, arena_bytes(b, h));
+  const bool use_bands = !cap || arena_bytes(b, h) + band_bytes(h) <= cap;
+  const uint64_t abytes = arena_bytes(b, h) + (use_bands ? band_bytes(h) : 0);
+  for (int w = 0; w < G; ++w) arena[w] = B.add_buf(B_ARENA, hbm[w], w, abytes);
   const int64_t Q = cdiv(iters, h);
   const int S = Q > 1 ? B.add_buf(B_DRAM, 0, -1, 4ull * R * C) : -1;   // pinned scratch grid
   const int64_t nby = cdiv(R, b), nbx = cdiv(C, b);
   st.bm = st.bn = b;
   st.bk = h;
-  st.hbm_peak_bytes = arena_bytes(b, h);
+  st.hbm_peak_bytes = abytes;
   std::vector<int64_t> slot_ctr(G, 0);
   // Each sibling's previous window of the same pass: a window that shares its
   // rows takes the power columns it has in common with it from that window's
@@ -327,7 +330,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
         // of the other rows from the sibling's previous window; the rest over PCIe.
         const int64_t bh = 2 * itq;
         int64_t r_lo = 0;
-        if (win_g.y0 > 0 && wm > bh) {
+        if (use_bands && win_g.y0 > 0 && wm > bh) {
           for (const Band& bd : bands[w])
             if (bd.q == q && bd.row == win_g.y0 && bd.covers(win_g.x0, win_g.x1)) {
               r_lo = bh;
@@ -388,7 +391,7 @@ int build_hotspot_plan(const northup_tree_s* t, int64_t R, int64_t C, int64_t it
           }
         }
         // and the rows it shares with a later window of the sibling below it
-        if (win_g.y1 < R && wm > bh) {
+        if (use_bands && win_g.y1 < R && wm > bh) {
           const int64_t brow = win_g.y1 - bh;
           bool needed = false;
           for (size_t bj = bi + 1; bj < blks.size() && !needed; ++bj) {
